@@ -1,0 +1,194 @@
+/*
+ * rtlsim.h — C ABI of the B200-native batch-stimulus RTL simulator.
+ *
+ * The hot path of RTLflow (Lin et al., ICPP'22, PAPER.md): cycle-based
+ * ("full-cycle") simulation of ONE levelized RTL design across a
+ * batch of N independent stimuli, one GPU thread per stimulus,
+ * every partition's combinational and sequential logic evaluated every clock
+ * cycle (Listing 1). Outputs must equal the plain definition
+ * (the CPU oracle, oracle/) bit for bit ("all signal outputs
+ * match the golden reference").
+ *
+ * Conventions (all calls):
+ *  - Every function returns RTLSIM_OK (0) or a negative rtlsim_status. No C++
+ *    exception crosses the ABI. rtlsim_last_error() gives a message.
+ *  - A value of width w is ceil(w/32) little-endian u32 words; bits >= w are
+ *    zero in every output. IW / OW / RW = sum of ceil(w/32) over the inputs /
+ *    outputs / registers, in IR order.
+ *  - Argument and IR errors leave the ctx unchanged. A CUDA error makes the
+ *    ctx sticky-failed: every later call except rtlsim_free returns
+ *    RTLSIM_E_STATE. A ctx is not thread-safe; use one ctx per device.
+ *  - Pointers documented "host" may be pageable or pinned (pinned buffers are
+ *    copied with async DMA directly; pageable ones through pinned staging).
+ *    Pointers documented "device" are CUDA device pointers on opt->device.
+ */
+#ifndef RTLSIM_H
+#define RTLSIM_H
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef enum {
+  RTLSIM_OK = 0,
+  RTLSIM_E_ARG = -1,         /* bad argument (NULL, size, range)                */
+  RTLSIM_E_IR = -2,          /* malformed IR (driver count, kinds, widths, SLICE) */
+  RTLSIM_E_COMB_LOOP = -3,   /* combinational cycle among ops (reading 13)      */
+  RTLSIM_E_UNSUPPORTED = -4, /* MUL/DIVU/MODU wider than 64 bits (reading 11)   */
+  RTLSIM_E_NOMEM = -5,       /* host or device allocation failed                */
+  RTLSIM_E_CUDA = -6,        /* CUDA runtime error (ctx becomes sticky-failed)  */
+  RTLSIM_E_STATE = -7,       /* wrong call order, or sticky failure             */
+  RTLSIM_E_RANGE = -8        /* cycles beyond the bound stimulus (reading 14)   */
+} rtlsim_status;
+
+/* Signal kinds (§2: nodes of the RTL graph). */
+enum { RTLSIM_INPUT = 0, RTLSIM_REG = 1, RTLSIM_COMB = 2, RTLSIM_CONST = 3 };
+
+/* Opcodes (DESIGN.md §3 gives the exact two-state semantics; operands are
+ * zero-extended to W = max(wd, wa, wb) unless stated, and every result is
+ * truncated to the destination width). Numbering is the IR
+ * interchange format (mirrored in rtlgen/ir.py). */
+enum rtlsim_opcode {
+  RTLSIM_OP_COPY = 0,   /* zext/trunc(a)                                     */
+  RTLSIM_OP_SEXT = 1,   /* sext_{wa}(a)                                      */
+  RTLSIM_OP_NOT = 2,    /* ~zext_W(a): high bits become 1 when wd > wa       */
+  RTLSIM_OP_AND = 3, RTLSIM_OP_OR = 4, RTLSIM_OP_XOR = 5,
+  RTLSIM_OP_ADD = 6, RTLSIM_OP_SUB = 7, RTLSIM_OP_NEG = 8,
+  RTLSIM_OP_MUL = 9,    /* all widths <= 64                                  */
+  RTLSIM_OP_DIVU = 10,  /* <= 64; b == 0 gives 0                             */
+  RTLSIM_OP_MODU = 11,  /* <= 64; b == 0 gives 0                             */
+  RTLSIM_OP_EQ = 12, RTLSIM_OP_NE = 13,                  /* 1-bit results   */
+  RTLSIM_OP_LTU = 14, RTLSIM_OP_LEU = 15, RTLSIM_OP_GTU = 16, RTLSIM_OP_GEU = 17,
+  RTLSIM_OP_LTS = 18, RTLSIM_OP_LES = 19, RTLSIM_OP_GTS = 20, RTLSIM_OP_GES = 21,
+  RTLSIM_OP_SHL = 22,   /* b self-determined; b >= wd gives 0                */
+  RTLSIM_OP_SHRL = 23,  /* b >= max(wd,wa) gives 0                           */
+  RTLSIM_OP_SHRA = 24,  /* sext to max(wd,wa), b >= that width gives sign fill */
+  RTLSIM_OP_MUX = 25,   /* a = select (any width, != 0), b = then, c = else  */
+  RTLSIM_OP_CONCAT = 26,/* {a, b}: (a << wb) | b                             */
+  RTLSIM_OP_SLICE = 27, /* a[imm + wd - 1 : imm]; imm + wd <= wa             */
+  RTLSIM_OP_REDAND = 28, RTLSIM_OP_REDOR = 29, RTLSIM_OP_REDXOR = 30
+};
+#define RTLSIM_NONE 0xFFFFFFFFu
+#define RTLSIM_MAX_WIDTH 1024
+
+/* One op: V[dst] := EVAL(opcode, V[a], V[b], V[c], imm) mod 2^w_dst.
+ * Unused operand fields are RTLSIM_NONE. `part` is the op's partition
+ * (§3.2: macro tasks / partitions of the RTL graph). */
+typedef struct {
+  uint16_t opcode, part;
+  uint32_t dst, a, b, c, imm;
+} rtlsim_op;
+
+/* The levelized design (borrowed only during rtlsim_load; copied). */
+typedef struct {
+  uint32_t n_signals;
+  const uint16_t *width;       /* [n_signals], 1..1024                        */
+  const uint8_t *kind;         /* [n_signals], RTLSIM_INPUT..RTLSIM_CONST     */
+  uint32_t n_ops;
+  const rtlsim_op *ops;        /* any order; must be acyclic, one driver per COMB */
+  uint32_t n_regs;
+  const uint32_t *reg_q;       /* [n_regs] REG signals                        */
+  const uint32_t *reg_d;       /* [n_regs] any signal; q <= d mod 2^w_q       */
+  const uint32_t *reg_init;    /* [RW] initial register words (all stimuli)   */
+  uint32_t n_consts;
+  const uint32_t *const_sig;   /* [n_consts] CONST signals                    */
+  const uint32_t *const_words; /* [sum ceil(w/32)] constant words             */
+  uint32_t n_inputs;
+  const uint32_t *input_sig;   /* [n_inputs] INPUT signals: stimulus word order */
+  uint32_t n_outputs;
+  const uint32_t *output_sig;  /* [n_outputs] any signals: output word order  */
+  uint32_t n_partitions;       /* ops[i].part < n_partitions; partition DAG acyclic */
+} rtlsim_ir;
+
+/* Option flags */
+#define RTLSIM_F_DIGEST 0x1u      /* compute the per-(stimulus, cycle) digest   */
+#define RTLSIM_F_NO_PIPELINE 0x2u /* host-buffer runs: serialise copy/compute   */
+#define RTLSIM_F_GRAPH 0x4u       /* per-(cycle, partition) kernel nodes in a CUDA
+                                     graph instead of one fused chunk kernel   */
+#define RTLSIM_F_HOST_ONLY 0x8u   /* compile the schedule only; no device work
+                                     (load/stats only; bind/run return E_STATE) */
+
+typedef struct {
+  int device;                /* CUDA device ordinal                           */
+  void *cuda_stream;         /* cudaStream_t for compute, or NULL (own stream) */
+  uint32_t op_lanes;         /* warps per CTA sharing one stimulus tile (0 = auto) */
+  uint32_t chunk_cycles;     /* cycles per launch / pipeline chunk (0 = auto) */
+  uint32_t flags;            /* RTLSIM_F_*                                    */
+  uint32_t smem_limit;       /* bytes of shared memory per CTA (0 = device max) */
+} rtlsim_options;
+
+typedef struct {
+  uint64_t n_ops, n_signals, n_regs;   /* design                              */
+  uint64_t word_ops;         /* sum over ops of ceil(max(wd,wa,wb)/32)        */
+  uint64_t n_desc;           /* descriptors incl. loads/stores per cycle      */
+  uint64_t n_steps;          /* barrier-separated steps per cycle             */
+  uint64_t n_partitions;
+  double b_floor;            /* algorithmic HBM bytes per stimulus-cycle:
+                                sum_regs 2 b(w) + sum_in b(w) + sum_out b(w)  */
+  double b_state;            /* bytes the schedule moves per stimulus-cycle  */
+  double b_part;             /* of which cross-partition nets                 */
+  uint64_t rows_bit, rows_u8, rows_u16, rows_u32;    /* state arena rows      */
+  uint64_t xrows_bit, xrows_u8, xrows_u16, xrows_u32;/* cross-partition rows  */
+  uint64_t smem_words;       /* shared words per tile (per stimulus warp)     */
+  uint32_t op_lanes, chunk_cycles, tile_stimuli, iw, ow, rw;
+  uint64_t device_bytes;     /* device memory held by the ctx                 */
+} rtlsim_stats_t;
+
+typedef struct rtlsim_ctx rtlsim_ctx;
+
+/* Called by rtlsim_run_stream / bind_stream in cycle order.
+ * producer: fill dst[N][nc][IW] (host, pinned) with stimulus cycles c0..c0+nc-1.
+ * consumer: read out[N][nc][OW] (host) and digest[N][nc] (or NULL).
+ * A non-zero return aborts the run with RTLSIM_E_ARG. */
+typedef int (*rtlsim_producer)(void *user, uint64_t c0, uint64_t nc, uint32_t *dst);
+typedef int (*rtlsim_consumer)(void *user, uint64_t c0, uint64_t nc, const uint32_t *out,
+                               const uint64_t *digest);
+
+/* Validate, levelize and compile the design (the paper's
+ * transpilation step, here a schedule + layout compiler), allocate device
+ * state and upload descriptors. opt may be NULL (defaults). */
+int rtlsim_load(const rtlsim_ir *ir, const rtlsim_options *opt, rtlsim_ctx **out);
+
+/* Bind N stimuli x T cycles, host stimulus stim[N][T][IW] (borrowed until the
+ * last run that reads it returns). Input bits above each input's width are
+ * ignored (reading 15). Resets registers to reg_init and the cycle cursor to 0.
+ * The stimulus is staged chunk by chunk (P:L919-963 pipeline), never copied
+ * whole. */
+int rtlsim_bind(rtlsim_ctx *ctx, uint64_t N, uint64_t T, const uint32_t *stim);
+/* Same with a DEVICE pointer to stim[N][T][IW] (resident in HBM). */
+int rtlsim_bind_device(rtlsim_ctx *ctx, uint64_t N, uint64_t T, const uint32_t *stim_dev);
+/* Same with a producer callback instead of a buffer. */
+int rtlsim_bind_stream(rtlsim_ctx *ctx, uint64_t N, uint64_t T, rtlsim_producer prod, void *user);
+
+/* Simulate `cycles` cycles c0..c0+cycles-1 from the ctx's cycle cursor c0
+ * (E_RANGE if c0 + cycles > T; nothing is simulated). Host outputs (each may
+ * be NULL): out[N][cycles][OW] (outputs sampled before the clock edge,
+ * reading 3), regs[N][RW] after the last cycle, digest[N][cycles]. Blocking. */
+int rtlsim_run(rtlsim_ctx *ctx, uint64_t cycles, uint32_t *out, uint32_t *regs, uint64_t *digest);
+/* Same with DEVICE output buffers (either may be NULL). Asynchronous on the
+ * ctx's stream: call rtlsim_sync before reading them. */
+int rtlsim_run_device(rtlsim_ctx *ctx, uint64_t cycles, uint32_t *out_dev, uint64_t *digest_dev);
+/* Same with a consumer callback receiving each chunk. */
+int rtlsim_run_stream(rtlsim_ctx *ctx, uint64_t cycles, rtlsim_consumer cons, void *user);
+int rtlsim_sync(rtlsim_ctx *ctx);
+
+/* Register state checkpoint: regs[N][RW] host (get/set), or reset to reg_init
+ * and cycle 0. */
+int rtlsim_get_regs(rtlsim_ctx *ctx, uint32_t *regs);
+int rtlsim_set_regs(rtlsim_ctx *ctx, const uint32_t *regs);
+int rtlsim_reset(rtlsim_ctx *ctx);
+
+int rtlsim_stats(const rtlsim_ctx *ctx, rtlsim_stats_t *st);
+/* Kernel launches issued by this ctx since load (for the bench's gpu_launches). */
+uint64_t rtlsim_launch_count(const rtlsim_ctx *ctx);
+/* Message for the last failing call on ctx (NULL: the thread's last
+ * rtlsim_load failure). Owned by the library; valid until the next call. */
+const char *rtlsim_last_error(const rtlsim_ctx *ctx);
+void rtlsim_free(rtlsim_ctx *ctx); /* NULL-safe */
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* RTLSIM_H */
