@@ -1,0 +1,476 @@
+// kernels.cu — hand-written sm_100a kernels of the simulator.
+//
+// N1 rtl_eval: the op-stream evaluator. One CTA = one tile of 32 stimuli
+// (one thread per stimulus) x L op-lanes (warps that
+// split the independent ops of each level, the paper's structure-level
+// parallelism P:L159-162). Combinational values live in shared-memory slots,
+// signal-major / stimulus-minor (slot word k of stimulus lane l at
+// smem[k + l], the index mapping of P:L623-638 moved on-chip): every warp
+// access is conflict-free. 1-bit values are packed, one u32 per 32 stimuli,
+// written with __ballot_sync. Registers stream from width-class arenas in HBM
+// (ping-pong buffers, non-blocking update). No tensor cores:
+// nothing here is a dense contraction.
+//
+// N2/N3: stimulus / output transposes between the user layout [N][T][W]
+// (stimulus-major) and the device layout [T][W][N] (coalesced per warp).
+// N4: register init / import / export.
+#include <cstdint>
+
+#include "kernels.h"
+#include "program.h"
+
+namespace rtlsim {
+
+// ------------------------------------------------------------- helpers --
+__device__ __forceinline__ uint32_t nw_of(uint32_t w) { return (w + 31u) >> 5; }
+
+// Slot layouts in shared memory (per 32-stimulus tile, chosen by width):
+//   w == 1      one packed word, bit `lane` = stimulus lane
+//   w in 2..8   32 byte lanes (8 words)
+//   w in 9..16  32 half-word lanes (16 words)
+//   w > 16      one 32-word row per 32-bit word: word i of lane l at off+32i+l
+//   constants (off & kConstSlot): one broadcast copy of the words
+// Values are canonical (bits >= w are zero).
+
+// word i of the value at slot `off` (width w), zero- or sign-extended to
+// infinite precision
+__device__ __forceinline__ uint32_t getw(const uint32_t *sm, uint32_t off, uint32_t w, uint32_t i,
+                                         bool sx, uint32_t lane) {
+  if (w == 1) {
+    const uint32_t b = (sm[off] >> lane) & 1u;
+    return sx ? (0u - b) : (i == 0 ? b : 0u);
+  }
+  const uint32_t n = nw_of(w), rem = w & 31u;
+  uint32_t x;
+  if (off & kConstSlot) {
+    x = sm[(off & ~kConstSlot) + (i < n ? i : n - 1)];
+  } else if (w <= 8) {
+    x = reinterpret_cast<const uint8_t *>(sm)[4u * off + lane];
+  } else if (w <= 16) {
+    x = reinterpret_cast<const uint16_t *>(sm)[2u * off + lane];
+  } else {
+    x = sm[off + 32u * (i < n ? i : n - 1) + lane];
+  }
+  if (i < n) {
+    if (sx && i == n - 1 && rem && ((x >> (rem - 1)) & 1u)) x |= ~((1u << rem) - 1u);
+    return x;
+  }
+  return sx ? 0u - ((x >> ((w - 1) & 31u)) & 1u) : 0u;   // x is the top word here
+}
+
+// store word i of a width-wd value (masking the top word); 1-bit values are
+// packed with a warp ballot and written by lane 0 (all lanes must call)
+__device__ __forceinline__ void putw(uint32_t *sm, uint32_t off, uint32_t wd, uint32_t i, uint32_t x,
+                                     uint32_t lane) {
+  if (wd == 1) {
+    const uint32_t m = __ballot_sync(0xFFFFFFFFu, x & 1u);
+    if (lane == 0) sm[off] = m;
+    return;
+  }
+  const uint32_t n = nw_of(wd), rem = wd & 31u;
+  if (i == n - 1 && rem) x &= (1u << rem) - 1u;
+  if (wd <= 8) reinterpret_cast<uint8_t *>(sm)[4u * off + lane] = (uint8_t)x;
+  else if (wd <= 16) reinterpret_cast<uint16_t *>(sm)[2u * off + lane] = (uint16_t)x;
+  else sm[off + 32u * i + lane] = x;
+}
+
+// shift amount (self-determined, unsigned), saturated when >= 2^32
+__device__ __forceinline__ uint32_t shamt(const uint32_t *sm, uint32_t off, uint32_t w, uint32_t lane) {
+  uint32_t s = getw(sm, off, w, 0, false, lane);
+  for (uint32_t i = 1; i < nw_of(w); i++)
+    if (getw(sm, off, w, i, false, lane)) s = 0xFFFFFFFFu;
+  return s;
+}
+
+__device__ __forceinline__ unsigned long long mix64(unsigned long long z) {
+  z ^= z >> 30;
+  z *= 0xBF58476D1CE4E5B9ull;
+  z ^= z >> 27;
+  z *= 0x94D049BB133111EBull;
+  z ^= z >> 31;
+  return z;
+}
+
+// --------------------------------------------------------------- N1 --
+__global__ void __launch_bounds__(1024) rtl_eval_kernel(const EvalParams p) {
+  extern __shared__ uint32_t sm[];
+  const uint32_t lane = threadIdx.x & 31u, wl = threadIdx.x >> 5;
+  const uint32_t tile = blockIdx.x;
+  const uint32_t s = tile * 32u + lane;
+  const uint32_t N = p.N_pad, N32 = p.N_pad >> 5;
+
+  for (uint32_t c = 0; c < p.n_cycles; c++) {
+    const uint32_t par = (uint32_t)((p.cycle0 + c) & 1ull);
+    const Arena cur = p.state[par], nxt = p.state[par ^ 1u];
+    const uint32_t *in = p.in + (size_t)c * p.IW * N;
+    uint32_t *out = p.out + (size_t)c * p.OW * N;
+    unsigned long long dig = 0ull;
+
+    for (uint32_t step = p.step_begin; step < p.step_end; step++) {
+      const uint32_t kb = __ldg(p.step_ptr + step * p.L + wl);
+      const uint32_t ke = __ldg(p.step_ptr + step * p.L + wl + 1);
+      for (uint32_t k = kb; k < ke; k++) {
+        const uint4 q0 = __ldg(p.desc + 2 * k);
+        const uint4 q1 = __ldg(p.desc + 2 * k + 1);
+        const uint32_t op = q0.x & 0xFFFFu, imm = q0.x >> 16;
+        const uint32_t wd = q0.y & 0xFFFFu, wa = q0.y >> 16;
+        const uint32_t wb = q0.z & 0xFFFFu, wc = q0.z >> 16;
+        const uint32_t d = q0.w, a = q1.x, b = q1.y, cc = q1.z;
+        const uint32_t nd = nw_of(wd);
+        switch (op) {
+          case RTLSIM_OP_COPY:
+            for (uint32_t i = 0; i < nd; i++) putw(sm, d, wd, i, getw(sm, a, wa, i, false, lane), lane);
+            break;
+          case RTLSIM_OP_SEXT:
+            for (uint32_t i = 0; i < nd; i++) putw(sm, d, wd, i, getw(sm, a, wa, i, true, lane), lane);
+            break;
+          case RTLSIM_OP_NOT:
+            for (uint32_t i = 0; i < nd; i++) putw(sm, d, wd, i, ~getw(sm, a, wa, i, false, lane), lane);
+            break;
+          case RTLSIM_OP_AND:
+            for (uint32_t i = 0; i < nd; i++)
+              putw(sm, d, wd, i, getw(sm, a, wa, i, false, lane) & getw(sm, b, wb, i, false, lane), lane);
+            break;
+          case RTLSIM_OP_OR:
+            for (uint32_t i = 0; i < nd; i++)
+              putw(sm, d, wd, i, getw(sm, a, wa, i, false, lane) | getw(sm, b, wb, i, false, lane), lane);
+            break;
+          case RTLSIM_OP_XOR:
+            for (uint32_t i = 0; i < nd; i++)
+              putw(sm, d, wd, i, getw(sm, a, wa, i, false, lane) ^ getw(sm, b, wb, i, false, lane), lane);
+            break;
+          case RTLSIM_OP_ADD:
+          case RTLSIM_OP_SUB: {
+            unsigned long long carry = (op == RTLSIM_OP_SUB) ? 1ull : 0ull;
+            for (uint32_t i = 0; i < nd; i++) {
+              uint32_t x = getw(sm, a, wa, i, false, lane), y = getw(sm, b, wb, i, false, lane);
+              if (op == RTLSIM_OP_SUB) y = ~y;
+              unsigned long long t = (unsigned long long)x + y + carry;
+              carry = t >> 32;
+              putw(sm, d, wd, i, (uint32_t)t, lane);
+            }
+            break;
+          }
+          case RTLSIM_OP_NEG: {
+            unsigned long long carry = 1ull;
+            for (uint32_t i = 0; i < nd; i++) {
+              unsigned long long t = (unsigned long long)(uint32_t)~getw(sm, a, wa, i, false, lane) + carry;
+              carry = t >> 32;
+              putw(sm, d, wd, i, (uint32_t)t, lane);
+            }
+            break;
+          }
+          case RTLSIM_OP_MUL:
+          case RTLSIM_OP_DIVU:
+          case RTLSIM_OP_MODU: {
+            unsigned long long x = getw(sm, a, wa, 0, false, lane) |
+                                   ((unsigned long long)getw(sm, a, wa, 1, false, lane) << 32);
+            unsigned long long y = getw(sm, b, wb, 0, false, lane) |
+                                   ((unsigned long long)getw(sm, b, wb, 1, false, lane) << 32);
+            unsigned long long r = op == RTLSIM_OP_MUL ? x * y : (y == 0ull ? 0ull : (op == RTLSIM_OP_DIVU ? x / y : x % y));
+            putw(sm, d, wd, 0, (uint32_t)r, lane);
+            if (nd > 1) putw(sm, d, wd, 1, (uint32_t)(r >> 32), lane);
+            break;
+          }
+          case RTLSIM_OP_EQ: case RTLSIM_OP_NE: case RTLSIM_OP_LTU: case RTLSIM_OP_LEU:
+          case RTLSIM_OP_GTU: case RTLSIM_OP_GEU: case RTLSIM_OP_LTS: case RTLSIM_OP_LES:
+          case RTLSIM_OP_GTS: case RTLSIM_OP_GES: {
+            const bool sg = op >= RTLSIM_OP_LTS;
+            const uint32_t n = nw_of(wa > wb ? wa : wb);
+            int cmp = 0;
+            for (int i = (int)n - 1; i >= 0 && cmp == 0; i--) {
+              uint32_t x = getw(sm, a, wa, (uint32_t)i, sg, lane), y = getw(sm, b, wb, (uint32_t)i, sg, lane);
+              if (x != y) {
+                if (sg && i == (int)n - 1) cmp = ((int32_t)x < (int32_t)y) ? -1 : 1;
+                else cmp = x < y ? -1 : 1;
+              }
+            }
+            uint32_t t;
+            switch (op) {
+              case RTLSIM_OP_EQ: t = cmp == 0; break;
+              case RTLSIM_OP_NE: t = cmp != 0; break;
+              case RTLSIM_OP_LTU: case RTLSIM_OP_LTS: t = cmp < 0; break;
+              case RTLSIM_OP_LEU: case RTLSIM_OP_LES: t = cmp <= 0; break;
+              case RTLSIM_OP_GTU: case RTLSIM_OP_GTS: t = cmp > 0; break;
+              default: t = cmp >= 0; break;
+            }
+            for (uint32_t i = 0; i < nd; i++) putw(sm, d, wd, i, i == 0 ? t : 0u, lane);
+            break;
+          }
+          case RTLSIM_OP_SHL: {
+            const uint32_t sa = shamt(sm, b, wb, lane);
+            const uint32_t ws = sa >> 5, bs = sa & 31u;
+            for (uint32_t i = 0; i < nd; i++) {
+              uint32_t x = 0;
+              if (sa < wd && i >= ws) {
+                x = getw(sm, a, wa, i - ws, false, lane) << bs;
+                if (bs && i > ws) x |= getw(sm, a, wa, i - ws - 1, false, lane) >> (32u - bs);
+              }
+              putw(sm, d, wd, i, x, lane);
+            }
+            break;
+          }
+          case RTLSIM_OP_SHRL:
+          case RTLSIM_OP_SHRA: {
+            const bool sx = op == RTLSIM_OP_SHRA;
+            const uint32_t W = wd > wa ? wd : wa;
+            uint32_t sa = shamt(sm, b, wb, lane);
+            if (sa > W) sa = W;   // beyond the context width: 0 / sign fill
+            const uint32_t ws = sa >> 5, bs = sa & 31u;
+            for (uint32_t i = 0; i < nd; i++) {
+              uint32_t x = getw(sm, a, wa, i + ws, sx, lane) >> bs;
+              if (bs) x |= getw(sm, a, wa, i + ws + 1, sx, lane) << (32u - bs);
+              putw(sm, d, wd, i, x, lane);
+            }
+            break;
+          }
+          case RTLSIM_OP_MUX: {
+            uint32_t sel = 0;
+            for (uint32_t i = 0; i < nw_of(wa); i++) sel |= getw(sm, a, wa, i, false, lane);
+            const uint32_t src = sel ? b : cc, wsrc = sel ? wb : wc;
+            for (uint32_t i = 0; i < nd; i++) putw(sm, d, wd, i, getw(sm, src, wsrc, i, false, lane), lane);
+            break;
+          }
+          case RTLSIM_OP_CONCAT: {
+            const uint32_t ws = wb >> 5, bs = wb & 31u;
+            for (uint32_t i = 0; i < nd; i++) {
+              uint32_t x = getw(sm, b, wb, i, false, lane);
+              if (i >= ws) {
+                x |= getw(sm, a, wa, i - ws, false, lane) << bs;
+                if (bs && i > ws) x |= getw(sm, a, wa, i - ws - 1, false, lane) >> (32u - bs);
+              }
+              putw(sm, d, wd, i, x, lane);
+            }
+            break;
+          }
+          case RTLSIM_OP_SLICE: {
+            const uint32_t ws = imm >> 5, bs = imm & 31u;
+            for (uint32_t i = 0; i < nd; i++) {
+              uint32_t x = getw(sm, a, wa, i + ws, false, lane) >> bs;
+              if (bs) x |= getw(sm, a, wa, i + ws + 1, false, lane) << (32u - bs);
+              putw(sm, d, wd, i, x, lane);
+            }
+            break;
+          }
+          case RTLSIM_OP_REDAND:
+          case RTLSIM_OP_REDOR:
+          case RTLSIM_OP_REDXOR: {
+            const uint32_t n = nw_of(wa), rem = wa & 31u;
+            uint32_t t = op == RTLSIM_OP_REDAND ? 1u : 0u;
+            for (uint32_t i = 0; i < n; i++) {
+              uint32_t x = getw(sm, a, wa, i, false, lane);
+              if (op == RTLSIM_OP_REDAND) t &= (x == ((i == n - 1 && rem) ? ((1u << rem) - 1u) : 0xFFFFFFFFu));
+              else if (op == RTLSIM_OP_REDOR) t |= (x != 0u);
+              else t ^= (__popc(x) & 1u);
+            }
+            for (uint32_t i = 0; i < nd; i++) putw(sm, d, wd, i, i == 0 ? t : 0u, lane);
+            break;
+          }
+          // ------------------------------------------------ loads --
+          case OP_LD_REG:
+          case OP_LD_X: {
+            const Arena &ar = op == OP_LD_REG ? cur : p.xnet;
+            if (imm == CLS_BIT) {
+              if (lane == 0) sm[d] = ar.bit[(size_t)a * N32 + tile];
+            } else if (imm == CLS_U8) {
+              reinterpret_cast<uint8_t *>(sm)[4u * d + lane] = ar.u8[(size_t)a * N + s];
+            } else if (imm == CLS_U16) {
+              reinterpret_cast<uint16_t *>(sm)[2u * d + lane] = ar.u16[(size_t)a * N + s];
+            } else {
+              for (uint32_t i = 0; i < nd; i++) sm[d + 32u * i + lane] = ar.u32[(size_t)(a + i) * N + s];
+            }
+            break;
+          }
+          case OP_LD_IN:
+            for (uint32_t i = 0; i < nd; i++) putw(sm, d, wd, i, in[(size_t)(a + i) * N + s], lane);
+            break;
+          case OP_LD_CONST:   // broadcast layout: one copy of the words per tile
+            if (lane == 0) {
+              if (wd == 1) sm[d] = (__ldg(p.consts + a) & 1u) ? 0xFFFFFFFFu : 0u;
+              else
+                for (uint32_t i = 0; i < nd; i++) sm[d + i] = __ldg(p.consts + a + i);
+            }
+            break;
+          // ----------------------------------------------- stores --
+          case OP_ST_REG:
+          case OP_ST_X: {
+            const Arena &ar = op == OP_ST_REG ? nxt : p.xnet;
+            const uint32_t aux = q1.w;
+            if (imm == CLS_BIT) {
+              const uint32_t m = sm[a];
+              if (lane == 0) ar.bit[(size_t)d * N32 + tile] = m;
+              if (op == OP_ST_REG && p.digest)
+                dig ^= mix64(((unsigned long long)(aux + 1u + 0x80000000u) << 32) | ((m >> lane) & 1u));
+            } else {
+              for (uint32_t i = 0; i < nd; i++) {
+                const uint32_t v = getw(sm, a, wd, i, false, lane);
+                if (imm == CLS_U8) ar.u8[(size_t)d * N + s] = (uint8_t)v;
+                else if (imm == CLS_U16) ar.u16[(size_t)d * N + s] = (uint16_t)v;
+                else ar.u32[(size_t)(d + i) * N + s] = v;
+                if (op == OP_ST_REG && p.digest)
+                  dig ^= mix64(((unsigned long long)(aux + i + 1u + 0x80000000u) << 32) | v);
+              }
+            }
+            break;
+          }
+          case OP_ST_OUT:
+            for (uint32_t i = 0; i < nd; i++) {
+              const uint32_t v = getw(sm, a, wd, i, false, lane);
+              out[(size_t)(d + i) * N + s] = v;
+              if (p.digest) dig ^= mix64(((unsigned long long)(d + i + 1u) << 32) | v);
+            }
+            break;
+          default:
+            break;
+        }
+      }
+      __syncthreads();
+    }
+    if (p.digest && dig) atomicXor(p.digest + (size_t)c * N + s, dig);
+  }
+}
+
+cudaError_t eval_set_smem(uint32_t smem_bytes) {
+  return cudaFuncSetAttribute(rtl_eval_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem_bytes);
+}
+
+cudaError_t launch_eval(const EvalParams &p, uint32_t smem_bytes, cudaStream_t st) {
+  dim3 grid(p.N_pad / 32u), block(32u * p.L);
+  rtl_eval_kernel<<<grid, block, smem_bytes, st>>>(p);
+  return cudaGetLastError();
+}
+
+// ------------------------------------------------------------ N2 / N3 --
+// 32x32 tiled transposes through shared memory (coalesced on both sides).
+__global__ void stim_transpose_kernel(const uint32_t *__restrict__ src, uint64_t src_pitch, uint32_t N,
+                                      uint32_t nc, uint32_t IW, const uint32_t *__restrict__ mask,
+                                      uint32_t *__restrict__ dst, uint32_t N_pad) {
+  __shared__ uint32_t t[32][33];
+  const uint32_t cols = nc * IW;                       // (cycle, word) pairs
+  const uint32_t j0 = blockIdx.x * 32u, s0 = blockIdx.y * 32u;
+  for (uint32_t r = threadIdx.y; r < 32u; r += blockDim.y) {
+    const uint32_t s = s0 + r, j = j0 + threadIdx.x;
+    uint32_t v = 0;
+    if (s < N && j < cols) v = src[(size_t)s * src_pitch + j] & __ldg(mask + (j % IW));
+    t[r][threadIdx.x] = v;
+  }
+  __syncthreads();
+  for (uint32_t r = threadIdx.y; r < 32u; r += blockDim.y) {
+    const uint32_t j = j0 + r, s = s0 + threadIdx.x;
+    if (j < cols && s < N_pad) dst[(size_t)j * N_pad + s] = t[threadIdx.x][r];
+  }
+}
+
+cudaError_t launch_stim_transpose(const uint32_t *src, uint64_t src_pitch, uint32_t N, uint32_t N_pad,
+                                  uint32_t nc, uint32_t IW, const uint32_t *mask, uint32_t *dst,
+                                  cudaStream_t st) {
+  if (nc == 0 || IW == 0) return cudaSuccess;
+  dim3 grid((nc * IW + 31u) / 32u, N_pad / 32u), block(32, 8);
+  stim_transpose_kernel<<<grid, block, 0, st>>>(src, src_pitch, N, nc, IW, mask, dst, N_pad);
+  return cudaGetLastError();
+}
+
+__global__ void out_transpose_kernel(const uint32_t *__restrict__ src, uint32_t N, uint32_t N_pad,
+                                     uint32_t cols, uint32_t *__restrict__ dst, uint64_t dst_pitch) {
+  __shared__ uint32_t t[32][33];
+  const uint32_t j0 = blockIdx.x * 32u, s0 = blockIdx.y * 32u;
+  for (uint32_t r = threadIdx.y; r < 32u; r += blockDim.y) {
+    const uint32_t j = j0 + r, s = s0 + threadIdx.x;
+    t[r][threadIdx.x] = (j < cols && s < N_pad) ? src[(size_t)j * N_pad + s] : 0u;
+  }
+  __syncthreads();
+  for (uint32_t r = threadIdx.y; r < 32u; r += blockDim.y) {
+    const uint32_t s = s0 + r, j = j0 + threadIdx.x;
+    if (s < N && j < cols) dst[(size_t)s * dst_pitch + j] = t[threadIdx.x][r];
+  }
+}
+
+cudaError_t launch_out_transpose(const uint32_t *src, uint32_t N, uint32_t N_pad, uint32_t nc,
+                                 uint32_t OW, uint32_t *dst, uint64_t dst_pitch, cudaStream_t st) {
+  if (nc == 0 || OW == 0) return cudaSuccess;
+  dim3 grid((nc * OW + 31u) / 32u, N_pad / 32u), block(32, 8);
+  out_transpose_kernel<<<grid, block, 0, st>>>(src, N, N_pad, nc * OW, dst, dst_pitch);
+  return cudaGetLastError();
+}
+
+__global__ void digest_transpose_kernel(const unsigned long long *__restrict__ src, uint32_t N,
+                                        uint32_t N_pad, uint32_t nc, unsigned long long *__restrict__ dst,
+                                        uint64_t dst_pitch) {
+  __shared__ unsigned long long t[32][33];
+  const uint32_t j0 = blockIdx.x * 32u, s0 = blockIdx.y * 32u;
+  for (uint32_t r = threadIdx.y; r < 32u; r += blockDim.y) {
+    const uint32_t j = j0 + r, s = s0 + threadIdx.x;
+    t[r][threadIdx.x] = (j < nc && s < N_pad) ? src[(size_t)j * N_pad + s] : 0ull;
+  }
+  __syncthreads();
+  for (uint32_t r = threadIdx.y; r < 32u; r += blockDim.y) {
+    const uint32_t s = s0 + r, j = j0 + threadIdx.x;
+    if (s < N && j < nc) dst[(size_t)s * dst_pitch + j] = t[threadIdx.x][r];
+  }
+}
+
+cudaError_t launch_digest_transpose(const unsigned long long *src, uint32_t N, uint32_t N_pad, uint32_t nc,
+                                    unsigned long long *dst, uint64_t dst_pitch, cudaStream_t st) {
+  if (nc == 0) return cudaSuccess;
+  dim3 grid((nc + 31u) / 32u, N_pad / 32u), block(32, 8);
+  digest_transpose_kernel<<<grid, block, 0, st>>>(src, N, N_pad, nc, dst, dst_pitch);
+  return cudaGetLastError();
+}
+
+// ----------------------------------------------------------------- N4 --
+// one warp per (register word, 32-stimulus tile)
+__global__ void regs_import_kernel(const uint32_t *__restrict__ src, uint64_t src_stride,
+                                   const RegWord *__restrict__ map, uint32_t RW, uint32_t N,
+                                   uint32_t N_pad, Arena a) {
+  const uint32_t k = blockIdx.y;
+  const uint32_t s = blockIdx.x * blockDim.x + threadIdx.x;
+  if (s >= N_pad) return;
+  const uint32_t lane = threadIdx.x & 31u;
+  const RegWord m = map[k];
+  const uint32_t si = s < N ? s : (N ? N - 1 : 0);   // padding stimuli mirror the last one
+  const uint32_t v = src[(size_t)si * src_stride + k];
+  switch (m.cls) {
+    case CLS_BIT: {
+      const uint32_t bits = __ballot_sync(0xFFFFFFFFu, v & 1u);
+      if (lane == 0) a.bit[(size_t)m.row * (N_pad >> 5) + (s >> 5)] = bits;
+      break;
+    }
+    case CLS_U8: a.u8[(size_t)m.row * N_pad + s] = (uint8_t)v; break;
+    case CLS_U16: a.u16[(size_t)m.row * N_pad + s] = (uint16_t)v; break;
+    default: a.u32[(size_t)m.row * N_pad + s] = v; break;
+  }
+}
+
+cudaError_t launch_regs_import(const uint32_t *src, uint64_t src_stride, const RegWord *map, uint32_t RW,
+                               uint32_t N, uint32_t N_pad, Arena a, cudaStream_t st) {
+  if (RW == 0) return cudaSuccess;
+  dim3 grid(N_pad / 256u + ((N_pad % 256u) ? 1u : 0u), RW), block(256);
+  regs_import_kernel<<<grid, block, 0, st>>>(src, src_stride, map, RW, N, N_pad, a);
+  return cudaGetLastError();
+}
+
+__global__ void regs_export_kernel(Arena a, const RegWord *__restrict__ map, uint32_t RW, uint32_t N,
+                                   uint32_t N_pad, uint32_t *__restrict__ dst) {
+  const uint32_t k = blockIdx.y;
+  const uint32_t s = blockIdx.x * blockDim.x + threadIdx.x;
+  if (s >= N) return;
+  const RegWord m = map[k];
+  uint32_t v;
+  switch (m.cls) {
+    case CLS_BIT: v = (a.bit[(size_t)m.row * (N_pad >> 5) + (s >> 5)] >> (s & 31u)) & 1u; break;
+    case CLS_U8: v = a.u8[(size_t)m.row * N_pad + s]; break;
+    case CLS_U16: v = a.u16[(size_t)m.row * N_pad + s]; break;
+    default: v = a.u32[(size_t)m.row * N_pad + s]; break;
+  }
+  dst[(size_t)s * RW + k] = v;
+}
+
+cudaError_t launch_regs_export(Arena a, const RegWord *map, uint32_t RW, uint32_t N, uint32_t N_pad,
+                               uint32_t *dst, cudaStream_t st) {
+  if (RW == 0 || N == 0) return cudaSuccess;
+  dim3 grid((N + 255u) / 256u, RW), block(256);
+  regs_export_kernel<<<grid, block, 0, st>>>(a, map, RW, N, N_pad, dst);
+  return cudaGetLastError();
+}
+
+}  // namespace rtlsim

@@ -1,0 +1,705 @@
+// runtime.cu — the C ABI (include/rtlsim.h): context lifecycle, device
+// memory, the per-chunk schedule and the pipelined stimulus upload / output
+// drain.
+//
+// PAPER.md mapping:
+//   * CUDA Graph execution (§3.2.2): the per-cycle partition
+//     schedule is either one fused chunk kernel that walks every partition's
+//     steps for Tc cycles per launch (default: no per-cycle launch at all), or,
+//     with RTLSIM_F_GRAPH, Tc x P per-(cycle, partition) kernel nodes captured
+//     once into a CUDA graph and replayed.
+//   * Pipeline scheduling (§3.2.3): stimulus chunks are uploaded
+//     and transposed (N2) on one side stream while the previous chunk is
+//     simulated and the one before is transposed back (N3) and drained on
+//     another; double-buffered, chained by events.
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <cstdio>
+#include <cstring>
+#include <map>
+#include <string>
+#include <vector>
+
+#include "../../include/rtlsim.h"
+#include "kernels.h"
+#include "program.h"
+
+using namespace rtlsim;
+
+namespace {
+thread_local std::string g_load_error;
+
+enum SrcKind { SRC_NONE = 0, SRC_HOST, SRC_DEVICE, SRC_PRODUCER };
+
+struct Dest {
+  uint32_t *out_host = nullptr, *out_dev = nullptr;
+  uint64_t *dig_host = nullptr, *dig_dev = nullptr;
+  rtlsim_consumer cons = nullptr;
+  void *user = nullptr;
+  uint64_t cycles = 0;   // total cycles of this run (output pitch)
+};
+
+bool is_pinned(const void *p) {
+  if (!p) return false;
+  cudaPointerAttributes a;
+  if (cudaPointerGetAttributes(&a, p) != cudaSuccess) {
+    cudaGetLastError();
+    return false;
+  }
+  return a.type == cudaMemoryTypeHost;
+}
+}  // namespace
+
+struct rtlsim_ctx {
+  Program prog;
+  rtlsim_options opt{};
+  bool host_only = false, failed = false;
+  std::string err;
+  int device = 0;
+  cudaStream_t st = nullptr, st_h2d = nullptr, st_d2h = nullptr;
+  bool own_stream = false;
+  uint32_t smem_bytes = 0;
+  uint64_t launches = 0;
+  uint64_t device_bytes = 0;
+  std::vector<void *> dev_allocs;     // freed at rtlsim_free
+  std::vector<void *> bind_allocs;    // freed at re-bind
+  std::vector<void *> host_allocs;    // pinned, freed at re-bind
+  // static device data
+  uint4 *d_desc = nullptr;
+  uint32_t *d_step = nullptr, *d_consts = nullptr, *d_mask = nullptr, *d_reginit = nullptr;
+  RegWord *d_regmap = nullptr;
+  // binding
+  SrcKind src = SRC_NONE;
+  const uint32_t *stim = nullptr;
+  bool stim_pinned = false;
+  rtlsim_producer prod = nullptr;
+  void *prod_user = nullptr;
+  uint64_t N = 0, T = 0, cycle = 0, cycle0_run = 0;
+  uint64_t static_bytes = 0;
+  uint32_t N_pad = 0, Tc = 64;
+  Arena state[2]{}, xnet{};
+  uint32_t *d_in[2]{}, *d_out[2]{}, *d_raw[2]{}, *d_outu[2]{};
+  unsigned long long *d_dig[2]{}, *d_digu[2]{};
+  uint32_t *h_in[2]{}, *h_out[2]{};
+  unsigned long long *h_dig[2]{};
+  cudaEvent_t ev_in_ready[2]{}, ev_comp_done[2]{}, ev_drain_done[2]{}, ev_h2d_copied[2]{}, ev_start = nullptr;
+  bool ev_used[2] = {false, false};
+  std::map<uint64_t, cudaGraphExec_t> graphs;   // graph mode: key (buf, parity, nc)
+};
+
+#define CK(call)                                                                       \
+  do {                                                                                 \
+    cudaError_t e_ = (call);                                                           \
+    if (e_ != cudaSuccess) return cuda_fail(ctx, e_, #call, __LINE__);                 \
+  } while (0)
+
+static int cuda_fail(rtlsim_ctx *ctx, cudaError_t e, const char *what, int line) {
+  ctx->failed = true;
+  ctx->err = std::string("CUDA error ") + cudaGetErrorString(e) + " at runtime.cu:" + std::to_string(line) +
+             " (" + what + ")";
+  return RTLSIM_E_CUDA;
+}
+
+static int arg_fail(rtlsim_ctx *ctx, int code, const std::string &msg) {
+  ctx->err = msg;
+  return code;
+}
+
+static cudaError_t dalloc(rtlsim_ctx *ctx, void **p, size_t bytes, bool bind_scope) {
+  *p = nullptr;
+  if (bytes == 0) return cudaSuccess;
+  cudaError_t e = cudaMalloc(p, bytes);
+  if (e != cudaSuccess) return e;
+  ctx->device_bytes += bytes;
+  (bind_scope ? ctx->bind_allocs : ctx->dev_allocs).push_back(*p);
+  return cudaSuccess;
+}
+
+static void free_binding(rtlsim_ctx *ctx) {
+  for (void *p : ctx->bind_allocs) cudaFree(p);
+  ctx->bind_allocs.clear();
+  for (void *p : ctx->host_allocs) cudaFreeHost(p);
+  ctx->host_allocs.clear();
+  for (auto &kv : ctx->graphs) cudaGraphExecDestroy(kv.second);
+  ctx->graphs.clear();
+  for (int b = 0; b < 2; b++) {
+    ctx->d_in[b] = ctx->d_out[b] = ctx->d_raw[b] = ctx->d_outu[b] = nullptr;
+    ctx->d_dig[b] = ctx->d_digu[b] = nullptr;
+    ctx->h_in[b] = ctx->h_out[b] = nullptr;
+    ctx->h_dig[b] = nullptr;
+    ctx->ev_used[b] = false;
+  }
+  ctx->src = SRC_NONE;
+  ctx->N = ctx->T = ctx->cycle = 0;
+  ctx->device_bytes = ctx->static_bytes;
+}
+
+
+// ------------------------------------------------------------------ load --
+extern "C" int rtlsim_load(const rtlsim_ir *ir, const rtlsim_options *opt, rtlsim_ctx **out) {
+  if (!out) {
+    g_load_error = "NULL out";
+    return RTLSIM_E_ARG;
+  }
+  *out = nullptr;
+  rtlsim_ctx *ctx = new (std::nothrow) rtlsim_ctx();
+  if (!ctx) return RTLSIM_E_NOMEM;
+  if (opt) ctx->opt = *opt;
+  ctx->host_only = (ctx->opt.flags & RTLSIM_F_HOST_ONLY) != 0;
+  ctx->device = ctx->opt.device;
+  uint32_t smem_limit = ctx->opt.smem_limit;
+  if (!ctx->host_only) {
+    cudaError_t e = cudaSetDevice(ctx->device);
+    if (e == cudaSuccess) {
+      int optin = 0;
+      e = cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, ctx->device);
+      if (!smem_limit) smem_limit = (uint32_t)optin;
+      smem_limit = std::min<uint32_t>(smem_limit, (uint32_t)optin);
+    }
+    if (e != cudaSuccess) {
+      g_load_error = std::string("CUDA device unavailable: ") + cudaGetErrorString(e);
+      cudaGetLastError();
+      delete ctx;
+      return RTLSIM_E_CUDA;
+    }
+  } else if (!smem_limit) {
+    smem_limit = 232448;   // sm_100 opt-in maximum (227 KB)
+  }
+  std::string err;
+  int rc = compile_program(ir, ctx->opt.op_lanes, smem_limit / 4u, &ctx->prog, &err);
+  if (rc != RTLSIM_OK) {
+    g_load_error = err;
+    delete ctx;
+    return rc;
+  }
+  Program &G = ctx->prog;
+  ctx->smem_bytes = G.smem_words * 4u;
+  if (ctx->opt.chunk_cycles) ctx->Tc = ctx->opt.chunk_cycles;
+  if (ctx->host_only) {
+    *out = ctx;
+    return RTLSIM_OK;
+  }
+  // device-side static data
+  auto up = [&](void **dst, const void *src, size_t bytes) -> cudaError_t {
+    cudaError_t e = dalloc(ctx, dst, std::max<size_t>(bytes, 16), false);
+    if (e != cudaSuccess || !bytes) return e;
+    return cudaMemcpy(*dst, src, bytes, cudaMemcpyHostToDevice);
+  };
+  std::vector<RegWord> regmap(G.RW);
+  for (const RegInfo &ri : G.regs)
+    for (uint32_t t = 0; t < (ri.cls == CLS_U32 ? nwords(ri.width) : 1u); t++)
+      regmap[ri.word + t] = RegWord{ri.cls, ri.row + t};
+  cudaError_t e = cudaSuccess;
+  if (e == cudaSuccess) e = up((void **)&ctx->d_desc, G.desc.data(), G.desc.size() * sizeof(Desc));
+  if (e == cudaSuccess) e = up((void **)&ctx->d_step, G.step_ptr.data(), G.step_ptr.size() * 4);
+  if (e == cudaSuccess) e = up((void **)&ctx->d_consts, G.const_pool.data(), G.const_pool.size() * 4);
+  if (e == cudaSuccess) e = up((void **)&ctx->d_mask, G.in_mask.data(), G.in_mask.size() * 4);
+  if (e == cudaSuccess) e = up((void **)&ctx->d_regmap, regmap.data(), regmap.size() * sizeof(RegWord));
+  if (e == cudaSuccess) e = up((void **)&ctx->d_reginit, G.reg_init.data(), G.reg_init.size() * 4);
+  if (e == cudaSuccess) e = eval_set_smem(std::max<uint32_t>(ctx->smem_bytes, 1024));
+  if (e == cudaSuccess) {
+    if (ctx->opt.cuda_stream) {
+      ctx->st = (cudaStream_t)ctx->opt.cuda_stream;
+    } else {
+      e = cudaStreamCreateWithFlags(&ctx->st, cudaStreamNonBlocking);
+      ctx->own_stream = true;
+    }
+  }
+  if (e == cudaSuccess) e = cudaStreamCreateWithFlags(&ctx->st_h2d, cudaStreamNonBlocking);
+  if (e == cudaSuccess) e = cudaStreamCreateWithFlags(&ctx->st_d2h, cudaStreamNonBlocking);
+  for (int b = 0; b < 2 && e == cudaSuccess; b++) {
+    e = cudaEventCreateWithFlags(&ctx->ev_in_ready[b], cudaEventDisableTiming);
+    if (e == cudaSuccess) e = cudaEventCreateWithFlags(&ctx->ev_comp_done[b], cudaEventDisableTiming);
+    if (e == cudaSuccess) e = cudaEventCreateWithFlags(&ctx->ev_drain_done[b], cudaEventDisableTiming);
+    if (e == cudaSuccess) e = cudaEventCreateWithFlags(&ctx->ev_h2d_copied[b], cudaEventDisableTiming);
+  }
+  if (e == cudaSuccess) e = cudaEventCreateWithFlags(&ctx->ev_start, cudaEventDisableTiming);
+  if (e != cudaSuccess) {
+    g_load_error = std::string("CUDA error during load: ") + cudaGetErrorString(e);
+    cudaGetLastError();
+    rtlsim_free(ctx);
+    return e == cudaErrorMemoryAllocation ? RTLSIM_E_NOMEM : RTLSIM_E_CUDA;
+  }
+  ctx->static_bytes = ctx->device_bytes;
+  *out = ctx;
+  return RTLSIM_OK;
+}
+
+// ------------------------------------------------------------------ bind --
+static int alloc_arena(rtlsim_ctx *ctx, Arena *a, const uint32_t rows[4]) {
+  const size_t N = ctx->N_pad;
+  CK(dalloc(ctx, (void **)&a->bit, (size_t)rows[CLS_BIT] * (N / 32) * 4, true));
+  CK(dalloc(ctx, (void **)&a->u8, (size_t)rows[CLS_U8] * N, true));
+  CK(dalloc(ctx, (void **)&a->u16, (size_t)rows[CLS_U16] * N * 2, true));
+  CK(dalloc(ctx, (void **)&a->u32, (size_t)rows[CLS_U32] * N * 4, true));
+  return RTLSIM_OK;
+}
+
+static int reset_regs(rtlsim_ctx *ctx) {
+  Program &G = ctx->prog;
+  CK(launch_regs_import(ctx->d_reginit, 0, ctx->d_regmap, G.RW, (uint32_t)ctx->N, ctx->N_pad, ctx->state[0],
+                        ctx->st));
+  ctx->launches++;
+  ctx->cycle = 0;
+  return RTLSIM_OK;
+}
+
+static int bind_common(rtlsim_ctx *ctx, uint64_t N, uint64_t T) {
+  if (!ctx) return RTLSIM_E_ARG;
+  if (ctx->failed || ctx->host_only) return arg_fail(ctx, RTLSIM_E_STATE, ctx->failed ? ctx->err : "host-only ctx");
+  if (N == 0 || N > (1ull << 31)) return arg_fail(ctx, RTLSIM_E_ARG, "N out of range");
+  CK(cudaSetDevice(ctx->device));
+  CK(cudaStreamSynchronize(ctx->st));
+  CK(cudaStreamSynchronize(ctx->st_h2d));
+  CK(cudaStreamSynchronize(ctx->st_d2h));
+  free_binding(ctx);
+  ctx->N = N;
+  ctx->T = T;
+  ctx->N_pad = (uint32_t)((N + 31) / 32 * 32);
+  Program &G = ctx->prog;
+  ctx->Tc = ctx->opt.chunk_cycles ? ctx->opt.chunk_cycles : 64;
+  if (T) ctx->Tc = (uint32_t)std::min<uint64_t>(ctx->Tc, T);
+  ctx->Tc = std::max<uint32_t>(ctx->Tc, 1);
+  int rc;
+  for (int b = 0; b < 2; b++)
+    if ((rc = alloc_arena(ctx, &ctx->state[b], G.rows)) != RTLSIM_OK) return rc;
+  if ((rc = alloc_arena(ctx, &ctx->xnet, G.xrows)) != RTLSIM_OK) return rc;
+  const size_t NP = ctx->N_pad, Tc = ctx->Tc;
+  for (int b = 0; b < 2; b++) {
+    CK(dalloc(ctx, (void **)&ctx->d_in[b], std::max<size_t>(Tc * G.IW * NP * 4, 16), true));
+    CK(dalloc(ctx, (void **)&ctx->d_out[b], std::max<size_t>(Tc * G.OW * NP * 4, 16), true));
+    CK(dalloc(ctx, (void **)&ctx->d_dig[b], Tc * NP * 8, true));
+    ctx->ev_used[b] = false;
+  }
+  return reset_regs(ctx);
+}
+
+// lazily allocated staging used by host-buffer / callback runs
+static int ensure_host_staging(rtlsim_ctx *ctx) {
+  if (ctx->d_raw[0]) return RTLSIM_OK;
+  Program &G = ctx->prog;
+  const size_t N = ctx->N, Tc = ctx->Tc;
+  for (int b = 0; b < 2; b++) {
+    CK(dalloc(ctx, (void **)&ctx->d_raw[b], std::max<size_t>(N * Tc * G.IW * 4, 16), true));
+    CK(dalloc(ctx, (void **)&ctx->d_outu[b], std::max<size_t>(N * Tc * G.OW * 4, 16), true));
+    CK(dalloc(ctx, (void **)&ctx->d_digu[b], N * Tc * 8, true));
+    void *p;
+    CK(cudaMallocHost(&p, std::max<size_t>(N * Tc * G.IW * 4, 16)));
+    ctx->host_allocs.push_back(p);
+    ctx->h_in[b] = (uint32_t *)p;
+    CK(cudaMallocHost(&p, std::max<size_t>(N * Tc * G.OW * 4, 16)));
+    ctx->host_allocs.push_back(p);
+    ctx->h_out[b] = (uint32_t *)p;
+    CK(cudaMallocHost(&p, N * Tc * 8));
+    ctx->host_allocs.push_back(p);
+    ctx->h_dig[b] = (unsigned long long *)p;
+  }
+  return RTLSIM_OK;
+}
+
+extern "C" int rtlsim_bind(rtlsim_ctx *ctx, uint64_t N, uint64_t T, const uint32_t *stim) {
+  if (!ctx) return RTLSIM_E_ARG;
+  if (!stim && ctx->prog.IW && T) return arg_fail(ctx, RTLSIM_E_ARG, "NULL stimulus");
+  int rc = bind_common(ctx, N, T);
+  if (rc) return rc;
+  ctx->src = SRC_HOST;
+  ctx->stim = stim;
+  ctx->stim_pinned = is_pinned(stim);
+  return RTLSIM_OK;
+}
+
+extern "C" int rtlsim_bind_device(rtlsim_ctx *ctx, uint64_t N, uint64_t T, const uint32_t *stim_dev) {
+  if (!ctx) return RTLSIM_E_ARG;
+  if (!stim_dev && ctx->prog.IW && T) return arg_fail(ctx, RTLSIM_E_ARG, "NULL stimulus");
+  int rc = bind_common(ctx, N, T);
+  if (rc) return rc;
+  ctx->src = SRC_DEVICE;
+  ctx->stim = stim_dev;
+  return RTLSIM_OK;
+}
+
+extern "C" int rtlsim_bind_stream(rtlsim_ctx *ctx, uint64_t N, uint64_t T, rtlsim_producer prod, void *user) {
+  if (!ctx) return RTLSIM_E_ARG;
+  if (!prod) return arg_fail(ctx, RTLSIM_E_ARG, "NULL producer");
+  int rc = bind_common(ctx, N, T);
+  if (rc) return rc;
+  ctx->src = SRC_PRODUCER;
+  ctx->prod = prod;
+  ctx->prod_user = user;
+  return RTLSIM_OK;
+}
+
+// ------------------------------------------------------------------- run --
+static EvalParams eval_params(rtlsim_ctx *ctx, int b, uint64_t cycle0, uint32_t nc, bool digest) {
+  Program &G = ctx->prog;
+  EvalParams p{};
+  p.desc = ctx->d_desc;
+  p.step_ptr = ctx->d_step;
+  p.step_begin = 0;
+  p.step_end = G.n_steps;
+  p.L = G.L;
+  p.n_cycles = nc;
+  p.cycle0 = cycle0;
+  p.N_pad = ctx->N_pad;
+  p.IW = G.IW;
+  p.OW = G.OW;
+  p.state[0] = ctx->state[0];
+  p.state[1] = ctx->state[1];
+  p.xnet = ctx->xnet;
+  p.in = ctx->d_in[b];
+  p.out = ctx->d_out[b];
+  p.consts = ctx->d_consts;
+  p.digest = digest ? ctx->d_dig[b] : nullptr;
+  return p;
+}
+
+// simulate chunk (cycle0, nc) from d_in[b] into d_out[b] / d_dig[b] on ctx->st
+static int launch_chunk(rtlsim_ctx *ctx, int b, uint64_t cycle0, uint32_t nc, bool digest) {
+  Program &G = ctx->prog;
+  if (digest) CK(cudaMemsetAsync(ctx->d_dig[b], 0, (size_t)nc * ctx->N_pad * 8, ctx->st));
+  if (G.n_steps == 0) return RTLSIM_OK;
+  if (!(ctx->opt.flags & RTLSIM_F_GRAPH)) {
+    EvalParams p = eval_params(ctx, b, cycle0, nc, digest);
+    CK(launch_eval(p, ctx->smem_bytes, ctx->st));
+    ctx->launches++;
+    return RTLSIM_OK;
+  }
+  // graph mode: Tc x P per-(cycle, partition) nodes, captured once per
+  // (buffer, parity, nc, digest) and replayed
+  const uint64_t key = ((uint64_t)nc << 8) | ((uint64_t)b << 2) | ((cycle0 & 1ull) << 1) | (digest ? 1u : 0u);
+  auto it = ctx->graphs.find(key);
+  if (it == ctx->graphs.end()) {
+    cudaStream_t cap;
+    CK(cudaStreamCreateWithFlags(&cap, cudaStreamNonBlocking));
+    CK(cudaStreamBeginCapture(cap, cudaStreamCaptureModeThreadLocal));
+    const uint32_t NP = (uint32_t)G.part_steps.size() - 1;
+    for (uint32_t c = 0; c < nc; c++) {
+      for (uint32_t q = 0; q < NP; q++) {
+        if (G.part_steps[q] == G.part_steps[q + 1]) continue;
+        EvalParams p = eval_params(ctx, b, (cycle0 & 1ull) + c, 1, digest);
+        p.step_begin = G.part_steps[q];
+        p.step_end = G.part_steps[q + 1];
+        p.in = ctx->d_in[b] + (size_t)c * G.IW * ctx->N_pad;
+        p.out = ctx->d_out[b] + (size_t)c * G.OW * ctx->N_pad;
+        if (digest) p.digest = ctx->d_dig[b] + (size_t)c * ctx->N_pad;
+        cudaError_t e = launch_eval(p, ctx->smem_bytes, cap);
+        if (e != cudaSuccess) {
+          cudaGraph_t g;
+          cudaStreamEndCapture(cap, &g);
+          return cuda_fail(ctx, e, "graph capture", __LINE__);
+        }
+      }
+    }
+    cudaGraph_t g;
+    CK(cudaStreamEndCapture(cap, &g));
+    cudaGraphExec_t ge;
+    CK(cudaGraphInstantiate(&ge, g, 0));
+    CK(cudaGraphDestroy(g));
+    CK(cudaStreamDestroy(cap));
+    it = ctx->graphs.emplace(key, ge).first;
+  }
+  CK(cudaGraphLaunch(it->second, ctx->st));
+  ctx->launches += (uint64_t)nc * (G.part_steps.size() - 1);
+  return RTLSIM_OK;
+}
+
+static int run_impl(rtlsim_ctx *ctx, uint64_t cycles, const Dest &dst, bool digest) {
+  if (!ctx) return RTLSIM_E_ARG;
+  if (ctx->failed) return arg_fail(ctx, RTLSIM_E_STATE, ctx->err);
+  if (ctx->src == SRC_NONE) return arg_fail(ctx, RTLSIM_E_STATE, "run before bind");
+  if (ctx->cycle + cycles > ctx->T) return arg_fail(ctx, RTLSIM_E_RANGE, "cycles beyond the bound stimulus");
+  if (cycles == 0) return RTLSIM_OK;
+  Program &G = ctx->prog;
+  CK(cudaSetDevice(ctx->device));
+  const bool host_side = ctx->src != SRC_DEVICE || dst.out_host || dst.dig_host || dst.cons;
+  if (host_side) {
+    int rc = ensure_host_staging(ctx);
+    if (rc) return rc;
+  }
+  const bool serial = (ctx->opt.flags & RTLSIM_F_NO_PIPELINE) != 0;
+  const uint32_t N = (uint32_t)ctx->N, NP = ctx->N_pad, IW = G.IW, OW = G.OW;
+  const bool out_pinned = dst.out_host && is_pinned(dst.out_host);
+  const bool dig_pinned = dst.dig_host && is_pinned(dst.dig_host);
+  // side streams start after everything already queued on the compute stream
+  CK(cudaEventRecord(ctx->ev_start, ctx->st));
+  CK(cudaStreamWaitEvent(ctx->st_h2d, ctx->ev_start, 0));
+  CK(cudaStreamWaitEvent(ctx->st_d2h, ctx->ev_start, 0));
+
+  const uint64_t nchunks = (cycles + ctx->Tc - 1) / ctx->Tc;
+  std::vector<uint32_t> nc_of(nchunks);
+  // host-side completion of chunk k (pageable outputs / consumer)
+  auto finish_host = [&](uint64_t k) -> int {
+    const int b = (int)(k & 1);
+    const uint64_t c0 = k * ctx->Tc;
+    const uint32_t nc = nc_of[k];
+    if (!((dst.out_host && !out_pinned) || (dst.dig_host && !dig_pinned) || dst.cons)) return RTLSIM_OK;
+    CK(cudaEventSynchronize(ctx->ev_drain_done[b]));
+    if (dst.out_host && !out_pinned)
+      for (uint64_t s = 0; s < N; s++)
+        memcpy(dst.out_host + (s * dst.cycles + c0) * OW, ctx->h_out[b] + s * (uint64_t)nc * OW,
+               (size_t)nc * OW * 4);
+    if (dst.dig_host && !dig_pinned)
+      for (uint64_t s = 0; s < N; s++)
+        memcpy(dst.dig_host + s * dst.cycles + c0, ctx->h_dig[b] + s * (uint64_t)nc, (size_t)nc * 8);
+    if (dst.cons) {
+      if (dst.cons(dst.user, ctx->cycle0_run + c0, nc, ctx->h_out[b], digest ? (const uint64_t *)ctx->h_dig[b] : nullptr))
+        return arg_fail(ctx, RTLSIM_E_ARG, "consumer aborted");
+    }
+    return RTLSIM_OK;
+  };
+  ctx->cycle0_run = ctx->cycle;
+  for (uint64_t k = 0; k < nchunks; k++) {
+    const int b = (int)(k & 1);
+    const uint64_t c0 = k * ctx->Tc;
+    const uint32_t nc = (uint32_t)std::min<uint64_t>(ctx->Tc, cycles - c0);
+    nc_of[k] = nc;
+    const uint64_t abs_c = ctx->cycle + c0;
+    // ---- A: stimulus chunk -> d_in[b] (side stream)
+    if (ctx->ev_used[b]) CK(cudaStreamWaitEvent(ctx->st_h2d, ctx->ev_comp_done[b], 0));
+    if (IW) {
+      const uint32_t *src = nullptr;
+      uint64_t pitch = 0;
+      if (ctx->src == SRC_DEVICE) {
+        src = ctx->stim + abs_c * IW;
+        pitch = ctx->T * IW;
+      } else {
+        const uint32_t *hsrc = nullptr;
+        uint64_t hpitch = 0;
+        if (ctx->src == SRC_HOST && ctx->stim_pinned) {
+          hsrc = ctx->stim + abs_c * IW;
+          hpitch = ctx->T * IW;
+        } else {
+          if (ctx->ev_used[b]) CK(cudaEventSynchronize(ctx->ev_h2d_copied[b]));
+          if (ctx->src == SRC_HOST) {
+            for (uint64_t s = 0; s < N; s++)
+              memcpy(ctx->h_in[b] + s * (uint64_t)nc * IW, ctx->stim + (s * ctx->T + abs_c) * IW,
+                     (size_t)nc * IW * 4);
+          } else if (ctx->prod(ctx->prod_user, abs_c, nc, ctx->h_in[b])) {
+            return arg_fail(ctx, RTLSIM_E_ARG, "producer aborted");
+          }
+          hsrc = ctx->h_in[b];
+          hpitch = (uint64_t)nc * IW;
+        }
+        CK(cudaMemcpy2DAsync(ctx->d_raw[b], (size_t)nc * IW * 4, hsrc, hpitch * 4, (size_t)nc * IW * 4, N,
+                             cudaMemcpyHostToDevice, ctx->st_h2d));
+        CK(cudaEventRecord(ctx->ev_h2d_copied[b], ctx->st_h2d));
+        src = ctx->d_raw[b];
+        pitch = (uint64_t)nc * IW;
+      }
+      CK(launch_stim_transpose(src, pitch, N, NP, nc, IW, ctx->d_mask, ctx->d_in[b], ctx->st_h2d));
+      ctx->launches++;
+    }
+    CK(cudaEventRecord(ctx->ev_in_ready[b], ctx->st_h2d));
+    if (serial) CK(cudaStreamSynchronize(ctx->st_h2d));
+    // ---- B: simulate the chunk (compute stream)
+    CK(cudaStreamWaitEvent(ctx->st, ctx->ev_in_ready[b], 0));
+    if (ctx->ev_used[b]) CK(cudaStreamWaitEvent(ctx->st, ctx->ev_drain_done[b], 0));
+    int rc = launch_chunk(ctx, b, abs_c, nc, digest);
+    if (rc) return rc;
+    CK(cudaEventRecord(ctx->ev_comp_done[b], ctx->st));
+    if (serial) CK(cudaStreamSynchronize(ctx->st));
+    // ---- C: drain (side stream)
+    CK(cudaStreamWaitEvent(ctx->st_d2h, ctx->ev_comp_done[b], 0));
+    if (dst.out_dev) {
+      CK(launch_out_transpose(ctx->d_out[b], N, NP, nc, OW, dst.out_dev + c0 * OW, dst.cycles * OW, ctx->st_d2h));
+      ctx->launches++;
+    }
+    if (dst.dig_dev) {
+      CK(launch_digest_transpose(ctx->d_dig[b], N, NP, nc, (unsigned long long *)dst.dig_dev + c0, dst.cycles,
+                                 ctx->st_d2h));
+      ctx->launches++;
+    }
+    if (dst.out_host || dst.cons) {
+      CK(launch_out_transpose(ctx->d_out[b], N, NP, nc, OW, ctx->d_outu[b], (uint64_t)nc * OW, ctx->st_d2h));
+      ctx->launches++;
+      if (out_pinned)
+        CK(cudaMemcpy2DAsync(dst.out_host + c0 * OW, dst.cycles * OW * 4, ctx->d_outu[b], (size_t)nc * OW * 4,
+                             (size_t)nc * OW * 4, N, cudaMemcpyDeviceToHost, ctx->st_d2h));
+      else
+        CK(cudaMemcpyAsync(ctx->h_out[b], ctx->d_outu[b], (size_t)N * nc * OW * 4, cudaMemcpyDeviceToHost,
+                           ctx->st_d2h));
+    }
+    if (dst.dig_host || (dst.cons && digest)) {
+      CK(launch_digest_transpose(ctx->d_dig[b], N, NP, nc, ctx->d_digu[b], nc, ctx->st_d2h));
+      ctx->launches++;
+      if (dig_pinned)
+        CK(cudaMemcpy2DAsync(dst.dig_host + c0, dst.cycles * 8, ctx->d_digu[b], (size_t)nc * 8, (size_t)nc * 8, N,
+                             cudaMemcpyDeviceToHost, ctx->st_d2h));
+      else
+        CK(cudaMemcpyAsync(ctx->h_dig[b], ctx->d_digu[b], (size_t)N * nc * 8, cudaMemcpyDeviceToHost,
+                           ctx->st_d2h));
+    }
+    CK(cudaEventRecord(ctx->ev_drain_done[b], ctx->st_d2h));
+    ctx->ev_used[b] = true;
+    if (serial) CK(cudaStreamSynchronize(ctx->st_d2h));
+    if (k >= 1) {
+      rc = finish_host(k - 1);
+      if (rc) return rc;
+    }
+  }
+  int rc = finish_host(nchunks - 1);
+  if (rc) return rc;
+  // join the side streams into the compute stream
+  CK(cudaEventRecord(ctx->ev_start, ctx->st_d2h));
+  CK(cudaStreamWaitEvent(ctx->st, ctx->ev_start, 0));
+  ctx->cycle += cycles;
+  return RTLSIM_OK;
+}
+
+static int export_regs(rtlsim_ctx *ctx, uint32_t *regs_host) {
+  Program &G = ctx->prog;
+  if (!G.RW) return RTLSIM_OK;
+  uint32_t *tmp = nullptr;
+  CK(cudaMallocAsync((void **)&tmp, (size_t)ctx->N * G.RW * 4, ctx->st));
+  CK(launch_regs_export(ctx->state[ctx->cycle & 1], ctx->d_regmap, G.RW, (uint32_t)ctx->N, ctx->N_pad, tmp,
+                        ctx->st));
+  ctx->launches++;
+  CK(cudaMemcpyAsync(regs_host, tmp, (size_t)ctx->N * G.RW * 4, cudaMemcpyDeviceToHost, ctx->st));
+  CK(cudaFreeAsync(tmp, ctx->st));
+  CK(cudaStreamSynchronize(ctx->st));
+  return RTLSIM_OK;
+}
+
+extern "C" int rtlsim_run(rtlsim_ctx *ctx, uint64_t cycles, uint32_t *out, uint32_t *regs, uint64_t *digest) {
+  if (!ctx) return RTLSIM_E_ARG;
+  Dest d;
+  d.out_host = out;
+  d.dig_host = digest;
+  d.cycles = cycles;
+  int rc = run_impl(ctx, cycles, d, digest != nullptr || (ctx->opt.flags & RTLSIM_F_DIGEST));
+  if (rc) return rc;
+  if (regs) {
+    rc = export_regs(ctx, regs);
+    if (rc) return rc;
+  }
+  CK(cudaStreamSynchronize(ctx->st));
+  return RTLSIM_OK;
+}
+
+extern "C" int rtlsim_run_device(rtlsim_ctx *ctx, uint64_t cycles, uint32_t *out_dev, uint64_t *digest_dev) {
+  if (!ctx) return RTLSIM_E_ARG;
+  Dest d;
+  d.out_dev = out_dev;
+  d.dig_dev = digest_dev;
+  d.cycles = cycles;
+  return run_impl(ctx, cycles, d, digest_dev != nullptr);
+}
+
+extern "C" int rtlsim_run_stream(rtlsim_ctx *ctx, uint64_t cycles, rtlsim_consumer cons, void *user) {
+  if (!ctx) return RTLSIM_E_ARG;
+  if (!cons) return arg_fail(ctx, RTLSIM_E_ARG, "NULL consumer");
+  Dest d;
+  d.cons = cons;
+  d.user = user;
+  d.cycles = cycles;
+  int rc = run_impl(ctx, cycles, d, (ctx->opt.flags & RTLSIM_F_DIGEST) != 0);
+  if (rc) return rc;
+  CK(cudaStreamSynchronize(ctx->st));
+  return RTLSIM_OK;
+}
+
+extern "C" int rtlsim_sync(rtlsim_ctx *ctx) {
+  if (!ctx) return RTLSIM_E_ARG;
+  if (ctx->failed) return arg_fail(ctx, RTLSIM_E_STATE, ctx->err);
+  if (ctx->host_only) return RTLSIM_OK;
+  CK(cudaStreamSynchronize(ctx->st));
+  CK(cudaStreamSynchronize(ctx->st_h2d));
+  CK(cudaStreamSynchronize(ctx->st_d2h));
+  return RTLSIM_OK;
+}
+
+// ------------------------------------------------------------ registers --
+extern "C" int rtlsim_get_regs(rtlsim_ctx *ctx, uint32_t *regs) {
+  if (!ctx || !regs) return RTLSIM_E_ARG;
+  if (ctx->failed) return arg_fail(ctx, RTLSIM_E_STATE, ctx->err);
+  if (ctx->src == SRC_NONE) return arg_fail(ctx, RTLSIM_E_STATE, "get_regs before bind");
+  return export_regs(ctx, regs);
+}
+
+extern "C" int rtlsim_set_regs(rtlsim_ctx *ctx, const uint32_t *regs) {
+  if (!ctx || !regs) return RTLSIM_E_ARG;
+  if (ctx->failed) return arg_fail(ctx, RTLSIM_E_STATE, ctx->err);
+  if (ctx->src == SRC_NONE) return arg_fail(ctx, RTLSIM_E_STATE, "set_regs before bind");
+  Program &G = ctx->prog;
+  if (!G.RW) return RTLSIM_OK;
+  CK(cudaSetDevice(ctx->device));
+  uint32_t *tmp = nullptr;
+  CK(cudaMallocAsync((void **)&tmp, (size_t)ctx->N * G.RW * 4, ctx->st));
+  CK(cudaMemcpyAsync(tmp, regs, (size_t)ctx->N * G.RW * 4, cudaMemcpyHostToDevice, ctx->st));
+  CK(launch_regs_import(tmp, G.RW, ctx->d_regmap, G.RW, (uint32_t)ctx->N, ctx->N_pad, ctx->state[ctx->cycle & 1],
+                        ctx->st));
+  ctx->launches++;
+  CK(cudaFreeAsync(tmp, ctx->st));
+  CK(cudaStreamSynchronize(ctx->st));
+  return RTLSIM_OK;
+}
+
+extern "C" int rtlsim_reset(rtlsim_ctx *ctx) {
+  if (!ctx) return RTLSIM_E_ARG;
+  if (ctx->failed) return arg_fail(ctx, RTLSIM_E_STATE, ctx->err);
+  if (ctx->src == SRC_NONE) return arg_fail(ctx, RTLSIM_E_STATE, "reset before bind");
+  CK(cudaSetDevice(ctx->device));
+  int rc = reset_regs(ctx);
+  if (rc) return rc;
+  CK(cudaStreamSynchronize(ctx->st));
+  return RTLSIM_OK;
+}
+
+// ---------------------------------------------------------------- misc --
+extern "C" int rtlsim_stats(const rtlsim_ctx *ctx, rtlsim_stats_t *st) {
+  if (!ctx || !st) return RTLSIM_E_ARG;
+  const Program &G = ctx->prog;
+  memset(st, 0, sizeof *st);
+  st->n_ops = G.n_ops;
+  st->n_signals = G.n_signals;
+  st->n_regs = G.reg_q.size();
+  st->word_ops = G.word_ops;
+  st->n_desc = G.desc.size();
+  st->n_steps = G.n_steps;
+  st->n_partitions = G.n_partitions;
+  st->b_floor = G.b_floor;
+  st->b_state = G.b_state;
+  st->b_part = G.b_part;
+  st->rows_bit = G.rows[CLS_BIT]; st->rows_u8 = G.rows[CLS_U8];
+  st->rows_u16 = G.rows[CLS_U16]; st->rows_u32 = G.rows[CLS_U32];
+  st->xrows_bit = G.xrows[CLS_BIT]; st->xrows_u8 = G.xrows[CLS_U8];
+  st->xrows_u16 = G.xrows[CLS_U16]; st->xrows_u32 = G.xrows[CLS_U32];
+  st->smem_words = G.smem_words;
+  st->op_lanes = G.L;
+  st->chunk_cycles = ctx->Tc;
+  st->tile_stimuli = 32;
+  st->iw = G.IW; st->ow = G.OW; st->rw = G.RW;
+  st->device_bytes = ctx->device_bytes;
+  return RTLSIM_OK;
+}
+
+extern "C" uint64_t rtlsim_launch_count(const rtlsim_ctx *ctx) { return ctx ? ctx->launches : 0; }
+
+extern "C" const char *rtlsim_last_error(const rtlsim_ctx *ctx) {
+  return ctx ? ctx->err.c_str() : g_load_error.c_str();
+}
+
+extern "C" void rtlsim_free(rtlsim_ctx *ctx) {
+  if (!ctx) return;
+  if (!ctx->host_only) {
+    cudaSetDevice(ctx->device);
+    if (ctx->st) cudaStreamSynchronize(ctx->st);
+    if (ctx->st_h2d) cudaStreamSynchronize(ctx->st_h2d);
+    if (ctx->st_d2h) cudaStreamSynchronize(ctx->st_d2h);
+    free_binding(ctx);
+    for (void *p : ctx->dev_allocs) cudaFree(p);
+    for (int b = 0; b < 2; b++) {
+      if (ctx->ev_in_ready[b]) cudaEventDestroy(ctx->ev_in_ready[b]);
+      if (ctx->ev_comp_done[b]) cudaEventDestroy(ctx->ev_comp_done[b]);
+      if (ctx->ev_drain_done[b]) cudaEventDestroy(ctx->ev_drain_done[b]);
+      if (ctx->ev_h2d_copied[b]) cudaEventDestroy(ctx->ev_h2d_copied[b]);
+    }
+    if (ctx->ev_start) cudaEventDestroy(ctx->ev_start);
+    if (ctx->st_h2d) cudaStreamDestroy(ctx->st_h2d);
+    if (ctx->st_d2h) cudaStreamDestroy(ctx->st_d2h);
+    if (ctx->own_stream && ctx->st) cudaStreamDestroy(ctx->st);
+    cudaGetLastError();
+  }
+  delete ctx;
+}

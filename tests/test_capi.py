@@ -1,0 +1,133 @@
+"""The C-ABI library on the CPU build host: it loads, exports every symbol
+include/rtlsim.h declares, and its host-side compiler (validation, levelizer,
+layout, byte accounting) behaves — no compute calls without a GPU."""
+import ctypes
+import os
+import re
+
+import numpy as np
+import pytest
+
+from rtlgen import designs, shaped
+from rtlgen import ir as I
+from rtlgen.builder import Builder
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+@pytest.fixture(scope="module")
+def R():
+    from paper_conf_icpp_linrzkh22_b200 import build, rtlsim
+    build.build()
+    return rtlsim
+
+
+def test_exports_every_declared_symbol(R):
+    hdr = open(os.path.join(ROOT, "include", "rtlsim.h")).read()
+    declared = set(re.findall(r"\b(rtlsim_[a-z_]+)\s*\(", hdr))
+    declared -= {"rtlsim_producer", "rtlsim_consumer"}
+    assert {"rtlsim_load", "rtlsim_bind", "rtlsim_run"} <= declared
+    lib = ctypes.CDLL(R.LIB_PATH)
+    for name in sorted(declared):
+        assert hasattr(lib, name), name
+    assert declared == set(R.EXPORTS)
+
+
+def _load(R, ir, **kw):
+    return R.Simulator(ir, flags=R.F_HOST_ONLY, **kw)
+
+
+def test_host_only_compile_and_stats(R):
+    ir = designs.tiny_dut()
+    st = _load(R, ir).stats()
+    assert st["n_ops"] == ir.n_ops and st["iw"] == 5 and st["ow"] == ir.OW and st["rw"] == ir.RW
+    # B_floor = sum_regs 2 b(w) + sum_in b(w) + sum_out b(w), b = 1/8, 1, 2, 4*ceil(w/32)
+    b = lambda w: 0.125 if w == 1 else 1 if w <= 8 else 2 if w <= 16 else 4 * ((w + 31) // 32)
+    want = (sum(2 * b(int(ir.width[q])) for q in ir.reg_q) + sum(b(int(ir.width[s])) for s in ir.input_sig)
+            + sum(b(int(ir.width[s])) for s in ir.output_sig))
+    assert st["b_floor"] == pytest.approx(want)
+    assert st["n_steps"] >= 3 and st["smem_words"] > 0
+
+
+def test_partitioned_design_uses_cross_partition_nets(R):
+    ir = designs.random_dag(5, n_ops=200, n_regs=10, n_partitions=3)
+    st = _load(R, ir).stats()
+    assert st["b_part"] > 0 and st["xrows_bit"] + st["xrows_u8"] + st["xrows_u16"] + st["xrows_u32"] > 0
+
+
+def test_shaped_configs_fit_shared_memory(R):
+    for cid in (2, 3):
+        st = _load(R, shaped.generate(cid)).stats()
+        assert st["smem_words"] * 4 <= 227 * 1024, (cid, st["smem_words"])
+        assert st["op_lanes"] >= 1
+
+
+def _expect_error(R, ir, code):
+    with pytest.raises(R.RtlsimError) as e:
+        _load(R, ir)
+    assert e.value.code == code, (e.value, code)
+
+
+def test_validation_errors(R):
+    # comb loop
+    b = Builder()
+    x = b.input(4)
+    y = b.op("NOT", 4, x)
+    z = b.op("NOT", 4, y)
+    ir = b.build()
+    ir.ops["a"][0] = z          # y = ~z, z = ~y
+    _expect_error(R, ir, -3)
+    # double driver
+    b = Builder()
+    x = b.input(4)
+    y = b.op("NOT", 4, x)
+    ir = b.build()
+    ir.ops = np.concatenate([ir.ops, ir.ops])
+    _expect_error(R, ir, -2)
+    # width 0 / > 1024
+    ir = designs.listing2_dut()
+    ir.width[0] = 0
+    _expect_error(R, ir, -2)
+    ir = designs.listing2_dut()
+    ir.width[0] = 1025
+    _expect_error(R, ir, -2)
+    # MUL wider than 64 bits
+    b = Builder()
+    x = b.input(65)
+    b.op("MUL", 8, x, x)
+    _expect_error(R, b.build(), -4)
+    # SLICE out of range
+    b = Builder()
+    x = b.input(8)
+    b.op("SLICE", 4, x, imm=5)
+    _expect_error(R, b.build(), -2)
+    # partition DAG cycle: p0 -> p1 -> p0
+    b = Builder()
+    x = b.input(4)
+    b.partition(0)
+    u = b.op("NOT", 4, x)
+    b.partition(1)
+    v = b.op("NOT", 4, u)
+    b.partition(0)
+    b.op("NOT", 4, v)
+    _expect_error(R, b.build(), -2)
+    # the last load error is reported with a message
+    assert R.rtlsim_last_error(None)
+
+
+def test_unordered_ops_are_sorted(R):
+    """Ops may be given in any order; the levelizer sorts them."""
+    ir = designs.random_dag(7, n_ops=50)
+    rev = I.IR(**{f: getattr(ir, f) for f in ("width", "kind", "ops", "reg_q", "reg_d", "reg_init", "const_sig",
+                                               "const_words", "input_sig", "output_sig")})
+    rev.ops = ir.ops[::-1].copy()
+    assert _load(R, rev).stats()["n_ops"] == 50
+
+
+def test_product_does_not_import_oracle():
+    pkg = os.path.join(ROOT, "paper_conf_icpp_linrzkh22_b200")
+    for dirpath, _, files in os.walk(pkg):
+        for f in files:
+            if f.endswith((".py", ".cu", ".cpp", ".h")):
+                src = open(os.path.join(dirpath, f)).read()
+                assert "import oracle" not in src and "from oracle" not in src and "oracle.h" not in src, f

@@ -1,0 +1,157 @@
+"""Parity: the CUDA path (through the C ABI) against the CPU oracle, element
+by element, on the same seeded inputs. Integer-only method,
+so the bar is bit-exact equality of every output word, every register word
+and every per-(stimulus, cycle) digest."""
+import numpy as np
+import pytest
+
+from rtlgen import designs, shaped, stim
+from rtlgen import ir as I
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def R():
+    import torch
+    assert torch.cuda.is_available(), "GPU tests need a CUDA device"
+    from paper_conf_icpp_linrzkh22_b200 import build, rtlsim
+    build.build()
+    return rtlsim
+
+
+def gpu_run(R, ir, st, cycles=None, digest=True, **opt):
+    sim = R.Simulator(ir, **opt)
+    sim.bind(st)
+    r = sim.run(cycles or st.shape[1], out=True, regs=True, digest=digest)
+    r["launches"] = sim.launch_count()
+    return r
+
+
+def assert_same(got, want, what=""):
+    for k in ("out", "regs", "digest"):
+        if want.get(k) is None or got.get(k) is None:
+            continue
+        a, b = got[k], want[k]
+        assert a.shape == b.shape, (what, k, a.shape, b.shape)
+        if not np.array_equal(a, b):
+            bad = np.argwhere(a != b)
+            raise AssertionError(f"{what}: {k} differs at {len(bad)} places, first {bad[:5].tolist()} "
+                                 f"got {a[tuple(bad[0])]} want {b[tuple(bad[0])]}")
+
+
+def test_tiny_config1_full(R, oracle_lib):
+    """Config 1: tiny DUT, 1024 stimuli x 100 cycles, mode B, full parity."""
+    ir = designs.tiny_dut()
+    st = stim.tiny_stimulus(stim.STIM_SEED_BASE + 1, np.arange(1024), 100, mode="B")
+    want = oracle_lib.simulate(ir, st, digest=True, threads=8)
+    got = gpu_run(R, ir, st)
+    assert_same(got, want, "tiny")
+    assert got["launches"] > 0
+
+
+def test_tiny_ragged_n(R, oracle_lib):
+    ir = designs.tiny_dut()
+    for N in (1, 31, 33, 100):
+        st = stim.tiny_stimulus(5, np.arange(N), 70, mode="B")
+        assert_same(gpu_run(R, ir, st, chunk_cycles=16), oracle_lib.simulate(ir, st, digest=True), f"N={N}")
+
+
+def test_swap_and_listing2(R, oracle_lib):
+    for ir in (designs.swap_dut(), designs.listing2_dut()):
+        st = stim.stimulus(ir, 3, np.arange(64), 0, 12)
+        assert_same(gpu_run(R, ir, st), oracle_lib.simulate(ir, st, digest=True), ir.name)
+
+
+@pytest.mark.parametrize("seed", range(6))
+def test_comb_dag_exhaustive(R, oracle_lib, seed):
+    ir = designs.random_dag(seed, n_ops=60 + 25 * seed, input_widths=(3, 5, 1, 4, 3))
+    st = designs.exhaustive_stimulus(ir)
+    assert_same(gpu_run(R, ir, st), oracle_lib.simulate(ir, st, digest=True, threads=8), f"dag{seed}")
+
+
+@pytest.mark.parametrize("seed,parts", [(0, 1), (1, 3), (2, 5), (3, 2)])
+def test_sequential_dag_partitions(R, oracle_lib, seed, parts):
+    """Wide registers, cross-partition nets, shuffled partition order."""
+    ir = designs.random_dag(500 + seed, n_ops=300, n_regs=24, n_partitions=parts,
+                            input_widths=(7, 33, 1, 64, 100), max_width=1024)
+    st = stim.stimulus(ir, 11 + seed, np.arange(96), 0, 40, mask=False)
+    assert_same(gpu_run(R, ir, st, chunk_cycles=7), oracle_lib.simulate(ir, st, digest=True, threads=8),
+                f"seq{seed}")
+
+
+@pytest.mark.parametrize("cid,scale,N,T", [(2, 1.0, 256, 60), (3, 0.25, 160, 24), (4, 0.02, 96, 8)])
+def test_shaped_reduced(R, oracle_lib, cid, scale, N, T):
+    ir = shaped.generate(cid, scale=scale)
+    st = stim.stimulus(ir, stim.STIM_SEED_BASE + cid, np.arange(N), 0, T)
+    assert_same(gpu_run(R, ir, st, chunk_cycles=16), oracle_lib.simulate(ir, st, digest=True, threads=16),
+                f"config{cid}@{scale}")
+
+
+def test_modes_agree(R, oracle_lib):
+    """Graph mode, no-pipeline mode, op-lane counts and chunk sizes change only the schedule."""
+    ir = designs.random_dag(600, n_ops=250, n_regs=16, n_partitions=4, input_widths=(9, 40, 1))
+    st = stim.stimulus(ir, 21, np.arange(70), 0, 33)
+    want = oracle_lib.simulate(ir, st, digest=True, threads=8)
+    for opt in (dict(flags=R.F_GRAPH, chunk_cycles=8), dict(flags=R.F_NO_PIPELINE), dict(op_lanes=1),
+                dict(op_lanes=7, chunk_cycles=5), dict(flags=R.F_GRAPH | R.F_NO_PIPELINE, chunk_cycles=33)):
+        assert_same(gpu_run(R, ir, st, **opt), want, str(opt))
+
+
+def test_run_splitting_and_checkpoint(R, oracle_lib):
+    ir = designs.random_dag(700, n_ops=150, n_regs=12, n_partitions=2, input_widths=(9, 40, 1))
+    N, T = 64, 30
+    st = stim.stimulus(ir, 31, np.arange(N), 0, T)
+    want = oracle_lib.simulate(ir, st, digest=True)
+    sim = R.Simulator(ir, chunk_cycles=4)
+    sim.bind(st)
+    a = sim.run(11)
+    b = sim.run(19)
+    assert np.array_equal(np.concatenate([a["out"], b["out"]], axis=1), want["out"])
+    assert np.array_equal(b["regs"], want["regs"])
+    with pytest.raises(R.RtlsimError) as e:
+        sim.run(1)
+    assert e.value.code == -8          # E_RANGE beyond T
+    # checkpoint: reset, restore registers of cycle 11, continue
+    sim.reset()
+    half = oracle_lib.simulate(ir, st[:, :11])
+    sim2 = R.Simulator(ir)
+    sim2.bind(st[:, 11:].copy())
+    sim2.set_regs(half["regs"])
+    c = sim2.run(19)
+    assert np.array_equal(c["out"], want["out"][:, 11:]) and np.array_equal(c["regs"], want["regs"])
+    assert np.array_equal(sim2.get_regs(), want["regs"])
+
+
+def test_device_bind_and_run(R, oracle_lib):
+    import torch
+    ir = designs.tiny_dut()
+    N, T = 256, 50
+    st = stim.tiny_stimulus(9, np.arange(N), T, mode="B")
+    want = oracle_lib.simulate(ir, st, digest=True)
+    d_stim = torch.from_numpy(st.view(np.int32)).cuda()
+    out = torch.zeros((N, T, ir.OW), dtype=torch.int32, device="cuda")
+    dig = torch.zeros((N, T), dtype=torch.int64, device="cuda")
+    sim = R.Simulator(ir, chunk_cycles=13)
+    sim.bind_device(d_stim, N, T)
+    sim.run_device(T, out, dig)
+    sim.sync()
+    assert np.array_equal(out.cpu().numpy().view(np.uint32), want["out"])
+    assert np.array_equal(dig.cpu().numpy().view(np.uint64), want["digest"])
+    assert np.array_equal(sim.get_regs(), want["regs"])
+
+
+def test_pinned_host_buffers(R, oracle_lib):
+    import torch
+    ir = designs.random_dag(800, n_ops=120, n_regs=8, input_widths=(12, 5))
+    N, T = 128, 40
+    st = stim.stimulus(ir, 41, np.arange(N), 0, T)
+    want = oracle_lib.simulate(ir, st, digest=True)
+    pst = torch.from_numpy(st.view(np.int32)).pin_memory()
+    pout = torch.zeros((N, T, ir.OW), dtype=torch.int32).pin_memory()
+    sim = R.Simulator(ir, chunk_cycles=6)
+    sim.bind_device  # noqa: B018 (API presence)
+    R.rtlsim_bind(sim.ctx, pst.numpy())
+    sim.N, sim.T = N, T
+    R.rtlsim_run(sim.ctx, T, pout.numpy(), None, None)
+    assert np.array_equal(pout.numpy().view(np.uint32), want["out"])
