@@ -109,6 +109,9 @@ typedef struct {
                                      graph instead of one fused chunk kernel   */
 #define RTLSIM_F_HOST_ONLY 0x8u   /* compile the schedule only; no device work
                                      (load/stats only; bind/run return E_STATE) */
+#define RTLSIM_F_TIMING 0x10u     /* bracket every evaluator launch with CUDA
+                                     events on the compute stream; totals in
+                                     rtlsim_stats (eval_ms, eval_launches)     */
 
 typedef struct {
   int device;                /* CUDA device ordinal                           */
@@ -134,6 +137,9 @@ typedef struct {
   uint64_t smem_words;       /* shared words per tile (per stimulus warp)     */
   uint32_t op_lanes, chunk_cycles, tile_stimuli, iw, ow, rw;
   uint64_t device_bytes;     /* device memory held by the ctx                 */
+  double eval_ms;            /* RTLSIM_F_TIMING: summed evaluator launch time  */
+  uint64_t eval_launches;    /* RTLSIM_F_TIMING: timed evaluator launches      */
+  uint64_t eval_stim_cycles; /* RTLSIM_F_TIMING: stimulus-cycles they covered  */
 } rtlsim_stats_t;
 
 typedef struct rtlsim_ctx rtlsim_ctx;

@@ -149,11 +149,22 @@ int compile_program(const rtlsim_ir *ir, uint32_t op_lanes, uint32_t smem_limit_
     cw += nwords(G.width[s]);
   }
   G.const_words.assign(ir->const_words, ir->const_words + cw);
+  std::vector<uint32_t> input_row(n, 0);
   for (uint32_t i = 0; i < ir->n_inputs; i++) {
     uint32_t s = G.input_sig[i];
     if (s >= n || G.kind[s] != RTLSIM_INPUT || input_of[s] != -1)
       return fail(err, RTLSIM_E_IR, "input " + std::to_string(i) + ": bad signal");
     input_of[s] = (int32_t)G.IW;
+    {
+      // class-formatted per-cycle input rows (N2 writes them, LD_IN copies)
+      const uint32_t c = width_class(G.width[s]);
+      input_row[s] = G.in_rows[c];
+      for (uint32_t k = 0; k < nwords(G.width[s]); k++) {
+        G.in_map.push_back(c);
+        G.in_map.push_back(G.in_rows[c] + (c == CLS_U32 ? k : 0));
+      }
+      G.in_rows[c] += (c == CLS_U32) ? nwords(G.width[s]) : 1;
+    }
     for (uint32_t k = 0; k < nwords(G.width[s]); k++) {
       uint32_t bits = std::min<uint32_t>(32, G.width[s] - 32 * k);
       G.in_mask.push_back(bits == 32 ? 0xFFFFFFFFu : ((1u << bits) - 1u));
@@ -578,71 +589,87 @@ int compile_program(const rtlsim_ir *ir, uint32_t op_lanes, uint32_t smem_limit_
       Desc d{};
       d.wd = (uint16_t)w;
       d.d = vals[ld.val].slot;   // LD_CONST writes the broadcast layout
+      uint32_t op;
       if (G.kind[s] == RTLSIM_REG) {
         const RegInfo &ri = G.regs[reg_of[s]];
-        d.op = OP_LD_REG; d.imm = (uint16_t)ri.cls; d.a = ri.row;
+        op = OP_LD_REG; d.a = ri.row;
         if (ld.first) bytes_state += lane_bytes(w);
       } else if (G.kind[s] == RTLSIM_INPUT) {
-        d.op = OP_LD_IN; d.a = (uint32_t)input_of[s];
-        if (ld.first) bytes_state += 4.0 * nwords(w);
+        op = OP_LD_IN; d.a = input_row[s];
+        if (ld.first) bytes_state += lane_bytes(w);
       } else if (G.kind[s] == RTLSIM_CONST) {
-        d.op = OP_LD_CONST; d.a = (uint32_t)const_of[s];
+        op = OP_LD_CONST; d.a = (uint32_t)const_of[s];
       } else {
-        d.op = OP_LD_X; d.imm = width_class(w); d.a = xrow.at(s);
+        op = OP_LD_X; d.a = xrow.at(s);
         if (ld.first) {
           bytes_state += lane_bytes(w);
           bytes_part += lane_bytes(w);
         }
       }
+      d.w0 = op | ((uint32_t)width_class(w) << 17);
       steps[ld.step].push_back(StepDesc{d, nwords(w)});
     }
+    // compute descriptor: widths, slot offsets, layout codes and flags
+    auto compute_desc = [&](uint32_t opc, uint32_t wd, int32_t vd, int ar, const int32_t *src,
+                            uint32_t imm) -> Desc {
+      Desc d{};
+      d.wd = (uint16_t)wd;
+      d.d = vals[vd].slot;
+      uint32_t w0 = opc | (layout_code(wd, false) << 17);
+      bool wide = wd > 32;
+      const uint32_t sh[3] = {8, 11, 14};
+      uint16_t *ws[3] = {&d.wa, &d.wb, &d.wc};
+      uint32_t *os[3] = {&d.a, &d.b, &d.c};
+      for (int k = 0; k < ar; k++) {
+        const Value &v = vals[src[k]];
+        *ws[k] = (uint16_t)v.width;
+        *os[k] = operand(src[k]);
+        w0 |= layout_code(v.width, v.bcast) << sh[k];
+        wide = wide || v.width > 32;
+      }
+      if (ar >= 2) w0 |= DF_HAS_B;
+      if (ar >= 3) w0 |= DF_HAS_C;
+      if (wide) w0 |= DF_WIDE;
+      d.w0 = w0;
+      d.aux = imm;
+      return d;
+    };
     for (size_t j = 0; j < ops_p.size(); j++) {
       const uint32_t i = ops_p[j];
       const rtlsim_op &o = G.ops[i];
-      Desc d{};
-      d.op = o.opcode;
-      d.imm = o.opcode == RTLSIM_OP_SLICE ? (uint16_t)o.imm : 0;
-      d.wd = G.width[o.dst];
-      d.d = vals[vid(o.dst)].slot;
-      int ar = arity(o.opcode);
-      d.wa = G.width[o.a];
-      d.a = operand(op_vals[j][0]);
-      if (ar >= 2) { d.wb = G.width[o.b]; d.b = operand(op_vals[j][1]); }
-      if (ar >= 3) { d.wc = G.width[o.c]; d.c = operand(op_vals[j][2]); }
+      const int ar = arity(o.opcode);
+      Desc d = compute_desc(o.opcode, G.width[o.dst], vid(o.dst), ar, op_vals[j].data(),
+                            o.opcode == RTLSIM_OP_SLICE ? o.imm : 0u);
       uint32_t wmax = std::max<uint32_t>(d.wd, std::max<uint32_t>(d.wa, d.wb));
       uint32_t cost = nwords(wmax);
       G.word_ops += cost;
       if (o.opcode == RTLSIM_OP_MUL || o.opcode == RTLSIM_OP_DIVU || o.opcode == RTLSIM_OP_MODU) cost += 4;
-      if (o.opcode == RTLSIM_OP_SHL || o.opcode == RTLSIM_OP_SHRL || o.opcode == RTLSIM_OP_SHRA ||
-          o.opcode == RTLSIM_OP_CONCAT || o.opcode == RTLSIM_OP_SLICE) cost += 1;
+      if (d.w0 & DF_WIDE) cost += 2;
       steps[op_step[i]].push_back(StepDesc{d, cost});
     }
     for (const Synth &sy : synth) {
-      Desc d{};
-      d.op = RTLSIM_OP_COPY;
-      d.wd = (uint16_t)sy.w;
-      d.d = vals[sy.val].slot;
-      d.wa = G.width[sy.src_sig];
-      d.a = operand(is_local(sy.src_sig) ? vid(sy.src_sig) : groups.at(sy.src_sig).front().val);
+      const int32_t src = is_local(sy.src_sig) ? vid(sy.src_sig) : groups.at(sy.src_sig).front().val;
+      Desc d = compute_desc(RTLSIM_OP_COPY, sy.w, sy.val, 1, &src, 0u);
       steps[sy.step].push_back(StepDesc{d, nwords(std::max(sy.w, (uint32_t)d.wa))});
     }
     for (size_t k = 0; k < sinks.size(); k++) {
       const Sink &sk = sinks[k];
       Desc d{};
-      d.op = sk.op;
       d.a = operand(sk.src_val);
+      uint32_t op = sk.op;
       if (sk.op == OP_ST_REG) {
         const RegInfo &ri = G.regs[sk.idx];
-        d.wd = (uint16_t)ri.width; d.imm = (uint16_t)ri.cls; d.d = ri.row; d.aux = ri.word;
+        d.wd = (uint16_t)ri.width; d.d = ri.row; d.aux = ri.word;
         bytes_state += lane_bytes(ri.width);
       } else if (sk.op == OP_ST_OUT) {
         d.wd = G.width[G.output_sig[sk.idx]]; d.d = out_word[sk.idx];
         bytes_state += 4.0 * nwords(d.wd);
       } else {
-        d.wd = G.width[sk.idx]; d.imm = width_class(d.wd); d.d = xrow.at(sk.idx);
+        d.wd = G.width[sk.idx]; d.d = xrow.at(sk.idx);
         bytes_state += lane_bytes(d.wd);
         bytes_part += lane_bytes(d.wd);
       }
+      d.w0 = op | ((uint32_t)width_class(d.wd) << 17);
       steps[sink_step[k]].push_back(StepDesc{d, nwords(d.wd)});
     }
     for (auto &st : steps)
@@ -676,7 +703,8 @@ int compile_program(const rtlsim_ir *ir, uint32_t op_lanes, uint32_t smem_limit_
     }
     for (uint32_t l = 0; l < L; l++) {
       G.step_ptr.push_back((uint32_t)G.desc.size());
-      std::stable_sort(lanes[l].begin(), lanes[l].end(), [](const Desc &x, const Desc &y) { return x.op < y.op; });
+      std::stable_sort(lanes[l].begin(), lanes[l].end(),
+                       [](const Desc &x, const Desc &y) { return (x.w0 & 0xFFu) < (y.w0 & 0xFFu); });
       G.desc.insert(G.desc.end(), lanes[l].begin(), lanes[l].end());
     }
   }

@@ -82,6 +82,32 @@ __device__ __forceinline__ uint32_t shamt(const uint32_t *sm, uint32_t off, uint
   return s;
 }
 
+// 4-byte asynchronous global -> shared copy (LDGSTS); completion is awaited
+// once per step, just before the step barrier
+__device__ __forceinline__ void cp_async4(void *smem_dst, const void *gsrc) {
+  const uint32_t d = (uint32_t)__cvta_generic_to_shared(smem_dst);
+  asm volatile("cp.async.ca.shared.global [%0], [%1], 4;" ::"r"(d), "l"(gsrc) : "memory");
+}
+__device__ __forceinline__ void cp_async_wait_all() { asm volatile("cp.async.wait_all;" ::: "memory"); }
+
+// copy the tile's segment of a class row (or nd consecutive u32 rows) into
+// slot d, in the slot layout of its width class
+__device__ __forceinline__ void ld_class(uint32_t *sm, uint32_t d, uint32_t cls, uint32_t nd, const Arena &ar,
+                                         size_t row, uint32_t N, uint32_t tile, uint32_t lane) {
+  uint8_t *smb = reinterpret_cast<uint8_t *>(sm);
+  if (cls == CLS_BIT) {
+    if (lane == 0) cp_async4(sm + d, ar.bit + row * (N >> 5) + tile);
+  } else if (cls == CLS_U8) {
+    if (lane < 8) cp_async4(smb + 4u * d + 4u * lane, ar.u8 + row * N + tile * 32u + 4u * lane);
+  } else if (cls == CLS_U16) {
+    if (lane < 16)
+      cp_async4(smb + 4u * d + 4u * lane,
+                reinterpret_cast<const uint8_t *>(ar.u16 + row * N + tile * 32u) + 4u * lane);
+  } else {
+    for (uint32_t i = 0; i < nd; i++) cp_async4(sm + d + 32u * i + lane, ar.u32 + (row + i) * N + tile * 32u + lane);
+  }
+}
+
 __device__ __forceinline__ unsigned long long mix64(unsigned long long z) {
   z ^= z >> 30;
   z *= 0xBF58476D1CE4E5B9ull;
@@ -92,32 +118,15 @@ __device__ __forceinline__ unsigned long long mix64(unsigned long long z) {
 }
 
 // --------------------------------------------------------------- N1 --
-__global__ void __launch_bounds__(1024) rtl_eval_kernel(const EvalParams p) {
-  extern __shared__ uint32_t sm[];
-  const uint32_t lane = threadIdx.x & 31u, wl = threadIdx.x >> 5;
-  const uint32_t tile = blockIdx.x;
-  const uint32_t s = tile * 32u + lane;
-  const uint32_t N = p.N_pad, N32 = p.N_pad >> 5;
-
-  for (uint32_t c = 0; c < p.n_cycles; c++) {
-    const uint32_t par = (uint32_t)((p.cycle0 + c) & 1ull);
-    const Arena cur = p.state[par], nxt = p.state[par ^ 1u];
-    const uint32_t *in = p.in + (size_t)c * p.IW * N;
-    uint32_t *out = p.out + (size_t)c * p.OW * N;
-    unsigned long long dig = 0ull;
-
-    for (uint32_t step = p.step_begin; step < p.step_end; step++) {
-      const uint32_t kb = __ldg(p.step_ptr + step * p.L + wl);
-      const uint32_t ke = __ldg(p.step_ptr + step * p.L + wl + 1);
-      for (uint32_t k = kb; k < ke; k++) {
-        const uint4 q0 = __ldg(p.desc + 2 * k);
-        const uint4 q1 = __ldg(p.desc + 2 * k + 1);
-        const uint32_t op = q0.x & 0xFFFFu, imm = q0.x >> 16;
-        const uint32_t wd = q0.y & 0xFFFFu, wa = q0.y >> 16;
-        const uint32_t wb = q0.z & 0xFFFFu, wc = q0.z >> 16;
-        const uint32_t d = q0.w, a = q1.x, b = q1.y, cc = q1.z;
-        const uint32_t nd = nw_of(wd);
-        switch (op) {
+// Generic path: any widths (1..1024), word loops over 32-bit words. Kept out
+// of line so the hot loop below stays small in the instruction cache.
+__device__ __noinline__ void exec_wide(uint32_t *sm, const uint4 q0, const uint4 q1, uint32_t lane) {
+  const uint32_t op = q0.x & 0xFFu;
+  const uint32_t wd = q0.y & 0xFFFFu, wa = q0.y >> 16;
+  const uint32_t wb = q0.z & 0xFFFFu, wc = q0.z >> 16;
+  const uint32_t d = q0.w, a = q1.x, b = q1.y, cc = q1.z, imm = q1.w;
+  const uint32_t nd = nw_of(wd);
+  switch (op) {
           case RTLSIM_OP_COPY:
             for (uint32_t i = 0; i < nd; i++) putw(sm, d, wd, i, getw(sm, a, wa, i, false, lane), lane);
             break;
@@ -266,64 +275,178 @@ __global__ void __launch_bounds__(1024) rtl_eval_kernel(const EvalParams p) {
             for (uint32_t i = 0; i < nd; i++) putw(sm, d, wd, i, i == 0 ? t : 0u, lane);
             break;
           }
-          // ------------------------------------------------ loads --
-          case OP_LD_REG:
-          case OP_LD_X: {
-            const Arena &ar = op == OP_LD_REG ? cur : p.xnet;
-            if (imm == CLS_BIT) {
-              if (lane == 0) sm[d] = ar.bit[(size_t)a * N32 + tile];
-            } else if (imm == CLS_U8) {
-              reinterpret_cast<uint8_t *>(sm)[4u * d + lane] = ar.u8[(size_t)a * N + s];
-            } else if (imm == CLS_U16) {
-              reinterpret_cast<uint16_t *>(sm)[2u * d + lane] = ar.u16[(size_t)a * N + s];
-            } else {
-              for (uint32_t i = 0; i < nd; i++) sm[d + 32u * i + lane] = ar.u32[(size_t)(a + i) * N + s];
-            }
-            break;
-          }
-          case OP_LD_IN:
-            for (uint32_t i = 0; i < nd; i++) putw(sm, d, wd, i, in[(size_t)(a + i) * N + s], lane);
-            break;
-          case OP_LD_CONST:   // broadcast layout: one copy of the words per tile
-            if (lane == 0) {
-              if (wd == 1) sm[d] = (__ldg(p.consts + a) & 1u) ? 0xFFFFFFFFu : 0u;
-              else
-                for (uint32_t i = 0; i < nd; i++) sm[d + i] = __ldg(p.consts + a + i);
-            }
-            break;
-          // ----------------------------------------------- stores --
-          case OP_ST_REG:
-          case OP_ST_X: {
-            const Arena &ar = op == OP_ST_REG ? nxt : p.xnet;
-            const uint32_t aux = q1.w;
-            if (imm == CLS_BIT) {
-              const uint32_t m = sm[a];
-              if (lane == 0) ar.bit[(size_t)d * N32 + tile] = m;
-              if (op == OP_ST_REG && p.digest)
-                dig ^= mix64(((unsigned long long)(aux + 1u + 0x80000000u) << 32) | ((m >> lane) & 1u));
-            } else {
-              for (uint32_t i = 0; i < nd; i++) {
-                const uint32_t v = getw(sm, a, wd, i, false, lane);
-                if (imm == CLS_U8) ar.u8[(size_t)d * N + s] = (uint8_t)v;
-                else if (imm == CLS_U16) ar.u16[(size_t)d * N + s] = (uint16_t)v;
-                else ar.u32[(size_t)(d + i) * N + s] = v;
-                if (op == OP_ST_REG && p.digest)
-                  dig ^= mix64(((unsigned long long)(aux + i + 1u + 0x80000000u) << 32) | v);
-              }
-            }
-            break;
-          }
-          case OP_ST_OUT:
-            for (uint32_t i = 0; i < nd; i++) {
-              const uint32_t v = getw(sm, a, wd, i, false, lane);
-              out[(size_t)(d + i) * N + s] = v;
-              if (p.digest) dig ^= mix64(((unsigned long long)(d + i + 1u) << 32) | v);
-            }
-            break;
           default:
             break;
+  }
+}
+
+// Narrow fast path (every width <= 32): one 32-bit word per operand.
+__device__ __forceinline__ uint32_t fetch1(const uint32_t *sm, uint32_t off, uint32_t lc, uint32_t lane) {
+  const uint32_t o = off & 0xFFFFu;   // strips kConstSlot
+  if (lc == LC_U32) return sm[o + lane];
+  if (lc == LC_BIT) return (sm[o] >> lane) & 1u;
+  if (lc == LC_U8) return reinterpret_cast<const uint8_t *>(sm)[4u * o + lane];
+  if (lc == LC_U16) return reinterpret_cast<const uint16_t *>(sm)[2u * o + lane];
+  return sm[o];   // LC_CONST: broadcast
+}
+
+__device__ __forceinline__ void store1(uint32_t *sm, uint32_t d, uint32_t lc, uint32_t r, uint32_t lane) {
+  if (lc == LC_U32) {
+    sm[d + lane] = r;
+  } else if (lc == LC_BIT) {
+    const uint32_t m = __ballot_sync(0xFFFFFFFFu, r & 1u);
+    if (lane == 0) sm[d] = m;
+  } else if (lc == LC_U8) {
+    reinterpret_cast<uint8_t *>(sm)[4u * d + lane] = (uint8_t)r;
+  } else {
+    reinterpret_cast<uint16_t *>(sm)[2u * d + lane] = (uint16_t)r;
+  }
+}
+
+__device__ __forceinline__ int32_t sx32(uint32_t x, uint32_t w) {
+  const uint32_t sb = 1u << (w - 1u);
+  return (int32_t)((x ^ sb) - sb);
+}
+
+// EVAL for narrow ops on canonical (zero-extended) operands; the caller
+// truncates to wd. Semantics: DESIGN.md §3.
+__device__ __forceinline__ uint32_t alu1(uint32_t op, uint32_t x, uint32_t y, uint32_t z, uint32_t wd, uint32_t wa,
+                                         uint32_t wb, uint32_t imm) {
+  switch (op) {
+    case RTLSIM_OP_COPY: return x;
+    case RTLSIM_OP_SEXT: return (uint32_t)sx32(x, wa);
+    case RTLSIM_OP_NOT: return ~x;
+    case RTLSIM_OP_AND: return x & y;
+    case RTLSIM_OP_OR: return x | y;
+    case RTLSIM_OP_XOR: return x ^ y;
+    case RTLSIM_OP_ADD: return x + y;
+    case RTLSIM_OP_SUB: return x - y;
+    case RTLSIM_OP_NEG: return 0u - x;
+    case RTLSIM_OP_MUL: return x * y;
+    case RTLSIM_OP_DIVU: return y ? x / y : 0u;
+    case RTLSIM_OP_MODU: return y ? x % y : 0u;
+    case RTLSIM_OP_EQ: return x == y;
+    case RTLSIM_OP_NE: return x != y;
+    case RTLSIM_OP_LTU: return x < y;
+    case RTLSIM_OP_LEU: return x <= y;
+    case RTLSIM_OP_GTU: return x > y;
+    case RTLSIM_OP_GEU: return x >= y;
+    case RTLSIM_OP_LTS: return sx32(x, wa) < sx32(y, wb);
+    case RTLSIM_OP_LES: return sx32(x, wa) <= sx32(y, wb);
+    case RTLSIM_OP_GTS: return sx32(x, wa) > sx32(y, wb);
+    case RTLSIM_OP_GES: return sx32(x, wa) >= sx32(y, wb);
+    case RTLSIM_OP_SHL: return y >= wd ? 0u : x << y;
+    case RTLSIM_OP_SHRL: return y >= 32u ? 0u : x >> y;
+    case RTLSIM_OP_SHRA: return (uint32_t)(sx32(x, wa) >> (y > 31u ? 31u : y));
+    case RTLSIM_OP_MUX: return x ? y : z;
+    case RTLSIM_OP_CONCAT: return wb >= 32u ? y : ((x << wb) | y);
+    case RTLSIM_OP_SLICE: return x >> imm;
+    case RTLSIM_OP_REDAND: return x == (0xFFFFFFFFu >> (32u - wa));
+    case RTLSIM_OP_REDOR: return x != 0u;
+    default: return __popc(x) & 1u;   // REDXOR
+  }
+}
+
+// N1: op-stream evaluator.
+__global__ void __launch_bounds__(1024) rtl_eval_kernel(const EvalParams p) {
+  extern __shared__ uint32_t sm[];
+  const uint32_t lane = threadIdx.x & 31u, wl = threadIdx.x >> 5;
+  const uint32_t tile = blockIdx.x;
+  const uint32_t s = tile * 32u + lane;
+  const uint32_t N = p.N_pad, N32 = p.N_pad >> 5;
+  // per-warp descriptor staging buffer: 16 descriptors (512 B), refilled from
+  // registers that were prefetched while the previous chunk executed
+  uint4 *dbuf = reinterpret_cast<uint4 *>(sm + p.desc_smem_off) + wl * 32u;
+  uint4 pf = make_uint4(0, 0, 0, 0);
+  uint32_t pf_k = 0xFFFFFFFFu;
+
+  for (uint32_t c = 0; c < p.n_cycles; c++) {
+    const uint32_t par = (uint32_t)((p.cycle0 + c) & 1ull);
+    const Arena cur = p.state[par], nxt = p.state[par ^ 1u];
+    Arena inp;
+    inp.bit = p.in.bit + (size_t)c * p.in_stride[CLS_BIT];
+    inp.u8 = p.in.u8 + (size_t)c * p.in_stride[CLS_U8];
+    inp.u16 = p.in.u16 + (size_t)c * p.in_stride[CLS_U16];
+    inp.u32 = p.in.u32 + (size_t)c * p.in_stride[CLS_U32];
+    uint32_t *out = p.out + (size_t)c * p.OW * N;
+    unsigned long long dig = 0ull;
+
+    for (uint32_t step = p.step_begin; step < p.step_end; step++) {
+      const uint32_t kb = __ldg(p.step_ptr + step * p.L + wl);
+      const uint32_t ke = __ldg(p.step_ptr + step * p.L + wl + 1);
+      const uint32_t nstep = step + 1 < p.step_end ? step + 1 : p.step_begin;
+      const uint32_t nb = __ldg(p.step_ptr + nstep * p.L + wl);
+      for (uint32_t k0 = kb; k0 < ke; k0 += 16u) {
+        if (pf_k != k0) pf = __ldg(p.desc + 2u * k0 + lane);
+        __syncwarp();
+        dbuf[lane] = pf;
+        __syncwarp();
+        pf_k = (k0 + 16u < ke) ? k0 + 16u : nb;
+        pf = __ldg(p.desc + 2u * pf_k + lane);   // the array is padded by 16 descriptors
+        const uint32_t nk = min(16u, ke - k0);
+        for (uint32_t j = 0; j < nk; j++) {
+          const uint4 q0 = dbuf[2u * j];
+          const uint4 q1 = dbuf[2u * j + 1u];
+          const uint32_t w0 = q0.x, op = w0 & 0xFFu;
+          if (op < 32u) {
+            if (w0 & DF_WIDE) {
+              exec_wide(sm, q0, q1, lane);
+            } else {
+              const uint32_t wd = q0.y & 0xFFFFu, wa = q0.y >> 16, wb = q0.z & 0xFFFFu;
+              const uint32_t x = fetch1(sm, q1.x, (w0 >> 8) & 7u, lane);
+              const uint32_t y = (w0 & DF_HAS_B) ? fetch1(sm, q1.y, (w0 >> 11) & 7u, lane) : 0u;
+              const uint32_t z = (w0 & DF_HAS_C) ? fetch1(sm, q1.z, (w0 >> 14) & 7u, lane) : 0u;
+              const uint32_t r = alu1(op, x, y, z, wd, wa, wb, q1.w) & (0xFFFFFFFFu >> (32u - wd));
+              store1(sm, q0.w, (w0 >> 17) & 7u, r, lane);
+            }
+            continue;
+          }
+          const uint32_t wd = q0.y & 0xFFFFu, nd = nw_of(wd), cls = (w0 >> 17) & 7u;
+          const uint32_t d = q0.w, a = q1.x;
+          switch (op) {
+            case OP_LD_REG: ld_class(sm, d, cls, nd, cur, a, N, tile, lane); break;
+            case OP_LD_X: ld_class(sm, d, cls, nd, p.xnet, a, N, tile, lane); break;
+            case OP_LD_IN: ld_class(sm, d, cls, nd, inp, a, N, tile, lane); break;
+            case OP_LD_CONST:   // broadcast layout: one copy of the words per tile
+              if (lane == 0) {
+                if (wd == 1) sm[d] = (__ldg(p.consts + a) & 1u) ? 0xFFFFFFFFu : 0u;
+                else
+                  for (uint32_t i = 0; i < nd; i++) sm[d + i] = __ldg(p.consts + a + i);
+              }
+              break;
+            case OP_ST_REG:
+            case OP_ST_X: {
+              const Arena ar = op == OP_ST_REG ? nxt : p.xnet;
+              const bool dg = p.digest && op == OP_ST_REG;
+              const uint32_t aux = q1.w;
+              if (cls == CLS_BIT) {
+                const uint32_t word = sm[a];   // packed bits (1-bit constants are stored packed too)
+                if (lane == 0) ar.bit[(size_t)d * N32 + tile] = word;
+                if (dg) dig ^= mix64(((unsigned long long)(aux + 1u + 0x80000000u) << 32) | ((word >> lane) & 1u));
+              } else {
+                for (uint32_t i = 0; i < nd; i++) {
+                  const uint32_t v = getw(sm, a, wd, i, false, lane);
+                  if (cls == CLS_U8) ar.u8[(size_t)d * N + s] = (uint8_t)v;
+                  else if (cls == CLS_U16) ar.u16[(size_t)d * N + s] = (uint16_t)v;
+                  else ar.u32[(size_t)(d + i) * N + s] = v;
+                  if (dg) dig ^= mix64(((unsigned long long)(aux + i + 1u + 0x80000000u) << 32) | v);
+                }
+              }
+              break;
+            }
+            case OP_ST_OUT:
+              for (uint32_t i = 0; i < nd; i++) {
+                const uint32_t v = getw(sm, a, wd, i, false, lane);
+                out[(size_t)(d + i) * N + s] = v;
+                if (p.digest) dig ^= mix64(((unsigned long long)(d + i + 1u) << 32) | v);
+              }
+              break;
+            default:
+              break;
+          }
         }
       }
+      cp_async_wait_all();
       __syncthreads();
     }
     if (p.digest && dig) atomicXor(p.digest + (size_t)c * N + s, dig);
@@ -341,10 +464,14 @@ cudaError_t launch_eval(const EvalParams &p, uint32_t smem_bytes, cudaStream_t s
 }
 
 // ------------------------------------------------------------ N2 / N3 --
-// 32x32 tiled transposes through shared memory (coalesced on both sides).
+// N2: stimulus chunk [N][nc][IW] (user layout, row pitch src_pitch words) ->
+// per-cycle class-formatted input rows (packed bits / u8 / u16 / u32 word
+// rows, [nc][rows][N]) through a 32x32 shared-memory transpose, masking the
+// bits above each input's width (reading 15). Stimuli >= N read as zero.
 __global__ void stim_transpose_kernel(const uint32_t *__restrict__ src, uint64_t src_pitch, uint32_t N,
                                       uint32_t nc, uint32_t IW, const uint32_t *__restrict__ mask,
-                                      uint32_t *__restrict__ dst, uint32_t N_pad) {
+                                      const RegWord *__restrict__ map, Arena dst, InStride st,
+                                      uint32_t N_pad) {
   __shared__ uint32_t t[32][33];
   const uint32_t cols = nc * IW;                       // (cycle, word) pairs
   const uint32_t j0 = blockIdx.x * 32u, s0 = blockIdx.y * 32u;
@@ -355,18 +482,32 @@ __global__ void stim_transpose_kernel(const uint32_t *__restrict__ src, uint64_t
     t[r][threadIdx.x] = v;
   }
   __syncthreads();
+  const uint32_t lane = threadIdx.x;
   for (uint32_t r = threadIdx.y; r < 32u; r += blockDim.y) {
-    const uint32_t j = j0 + r, s = s0 + threadIdx.x;
-    if (j < cols && s < N_pad) dst[(size_t)j * N_pad + s] = t[threadIdx.x][r];
+    const uint32_t j = j0 + r, s = s0 + lane;
+    if (j >= cols) continue;                           // warp-uniform
+    const uint32_t c = j / IW, k = j % IW;
+    const RegWord m = map[k];
+    const uint32_t v = t[lane][r];
+    switch (m.cls) {
+      case CLS_BIT: {
+        const uint32_t bits = __ballot_sync(0xFFFFFFFFu, v & 1u);
+        if (lane == 0) dst.bit[(size_t)c * st.s[CLS_BIT] + (size_t)m.row * (N_pad >> 5) + (s0 >> 5)] = bits;
+        break;
+      }
+      case CLS_U8: dst.u8[(size_t)c * st.s[CLS_U8] + (size_t)m.row * N_pad + s] = (uint8_t)v; break;
+      case CLS_U16: dst.u16[(size_t)c * st.s[CLS_U16] + (size_t)m.row * N_pad + s] = (uint16_t)v; break;
+      default: dst.u32[(size_t)c * st.s[CLS_U32] + (size_t)m.row * N_pad + s] = v; break;
+    }
   }
 }
 
 cudaError_t launch_stim_transpose(const uint32_t *src, uint64_t src_pitch, uint32_t N, uint32_t N_pad,
-                                  uint32_t nc, uint32_t IW, const uint32_t *mask, uint32_t *dst,
-                                  cudaStream_t st) {
+                                  uint32_t nc, uint32_t IW, const uint32_t *mask, const RegWord *map,
+                                  Arena dst, InStride st, cudaStream_t stream) {
   if (nc == 0 || IW == 0) return cudaSuccess;
   dim3 grid((nc * IW + 31u) / 32u, N_pad / 32u), block(32, 8);
-  stim_transpose_kernel<<<grid, block, 0, st>>>(src, src_pitch, N, nc, IW, mask, dst, N_pad);
+  stim_transpose_kernel<<<grid, block, 0, stream>>>(src, src_pitch, N, nc, IW, mask, map, dst, st, N_pad);
   return cudaGetLastError();
 }
 
@@ -422,8 +563,8 @@ cudaError_t launch_digest_transpose(const unsigned long long *src, uint32_t N, u
 __global__ void regs_import_kernel(const uint32_t *__restrict__ src, uint64_t src_stride,
                                    const RegWord *__restrict__ map, uint32_t RW, uint32_t N,
                                    uint32_t N_pad, Arena a) {
-  const uint32_t k = blockIdx.y;
-  const uint32_t s = blockIdx.x * blockDim.x + threadIdx.x;
+  const uint32_t k = blockIdx.x;
+  const uint32_t s = blockIdx.y * blockDim.x + threadIdx.x;
   if (s >= N_pad) return;
   const uint32_t lane = threadIdx.x & 31u;
   const RegWord m = map[k];
@@ -444,15 +585,15 @@ __global__ void regs_import_kernel(const uint32_t *__restrict__ src, uint64_t sr
 cudaError_t launch_regs_import(const uint32_t *src, uint64_t src_stride, const RegWord *map, uint32_t RW,
                                uint32_t N, uint32_t N_pad, Arena a, cudaStream_t st) {
   if (RW == 0) return cudaSuccess;
-  dim3 grid(N_pad / 256u + ((N_pad % 256u) ? 1u : 0u), RW), block(256);
+  dim3 grid(RW, N_pad / 256u + ((N_pad % 256u) ? 1u : 0u)), block(256);
   regs_import_kernel<<<grid, block, 0, st>>>(src, src_stride, map, RW, N, N_pad, a);
   return cudaGetLastError();
 }
 
 __global__ void regs_export_kernel(Arena a, const RegWord *__restrict__ map, uint32_t RW, uint32_t N,
                                    uint32_t N_pad, uint32_t *__restrict__ dst) {
-  const uint32_t k = blockIdx.y;
-  const uint32_t s = blockIdx.x * blockDim.x + threadIdx.x;
+  const uint32_t k = blockIdx.x;
+  const uint32_t s = blockIdx.y * blockDim.x + threadIdx.x;
   if (s >= N) return;
   const RegWord m = map[k];
   uint32_t v;
@@ -468,7 +609,7 @@ __global__ void regs_export_kernel(Arena a, const RegWord *__restrict__ map, uin
 cudaError_t launch_regs_export(Arena a, const RegWord *map, uint32_t RW, uint32_t N, uint32_t N_pad,
                                uint32_t *dst, cudaStream_t st) {
   if (RW == 0 || N == 0) return cudaSuccess;
-  dim3 grid((N + 255u) / 256u, RW), block(256);
+  dim3 grid(RW, (N + 255u) / 256u), block(256);
   regs_export_kernel<<<grid, block, 0, st>>>(a, map, RW, N, N_pad, dst);
   return cudaGetLastError();
 }

@@ -14,6 +14,17 @@ struct Arena {
   uint32_t *u32;   // [rows_u32][N_pad]
 };
 
+// Per-cycle element strides of the input chunk's class arenas.
+struct InStride {
+  uint64_t s[4];
+};
+
+// Per register / input word: arena class and row (bit row / u8 row / u16 row /
+// u32 row).
+struct RegWord {
+  uint32_t cls, row;
+};
+
 struct EvalParams {
   const uint4 *desc;          // 32-byte descriptors = 2 x uint4
   const uint32_t *step_ptr;   // [n_steps * L + 1]: lane l of step s = [p[sL+l], p[sL+l+1])
@@ -23,7 +34,9 @@ struct EvalParams {
   uint32_t N_pad, IW, OW;
   Arena state[2];             // ping-pong register state
   Arena xnet;                 // cross-partition nets
-  const uint32_t *in;         // [n_cycles][IW][N_pad] (cycle 0 of this launch)
+  Arena in;                   // class-formatted input rows of cycle 0 of this launch
+  uint64_t in_stride[4];      // per-cycle element stride of each input class arena
+  uint32_t desc_smem_off;     // word offset of the per-warp descriptor buffers
   uint32_t *out;              // [n_cycles][OW][N_pad]
   const uint32_t *consts;
   unsigned long long *digest; // [n_cycles][N_pad] (XOR-accumulated) or NULL
@@ -33,11 +46,12 @@ struct EvalParams {
 cudaError_t launch_eval(const EvalParams &p, uint32_t smem_bytes, cudaStream_t st);
 cudaError_t eval_set_smem(uint32_t smem_bytes);
 
-// N2: stimulus chunk [N][nc][IW] (row pitch src_pitch words) -> [nc][IW][N_pad],
-// masked per word; stimuli >= N are zero.
+// N2: stimulus chunk [N][nc][IW] (row pitch src_pitch words) -> per-cycle
+// class-formatted input rows (map[k]: class and row of input word k), masked
+// per word; stimuli >= N are zero.
 cudaError_t launch_stim_transpose(const uint32_t *src, uint64_t src_pitch, uint32_t N, uint32_t N_pad,
-                                  uint32_t nc, uint32_t IW, const uint32_t *mask, uint32_t *dst,
-                                  cudaStream_t st);
+                                  uint32_t nc, uint32_t IW, const uint32_t *mask, const RegWord *map,
+                                  Arena dst, InStride st, cudaStream_t stream);
 // N3: [nc][OW][N_pad] -> dst[N][*][OW] rows of nc*OW words at pitch dst_pitch words.
 cudaError_t launch_out_transpose(const uint32_t *src, uint32_t N, uint32_t N_pad, uint32_t nc,
                                  uint32_t OW, uint32_t *dst, uint64_t dst_pitch, cudaStream_t st);
@@ -46,11 +60,6 @@ cudaError_t launch_digest_transpose(const unsigned long long *src, uint32_t N, u
                                     uint32_t nc, unsigned long long *dst, uint64_t dst_pitch,
                                     cudaStream_t st);
 
-// Per register word k of the user layout [N][RW]: arena class and row (bit
-// row / u8 row / u16 row / u32 row).
-struct RegWord {
-  uint32_t cls, row;
-};
 // N4: regs[N][RW] (src_stride 0 = broadcast one [RW] vector) -> arena
 cudaError_t launch_regs_import(const uint32_t *src, uint64_t src_stride, const RegWord *map,
                                uint32_t RW, uint32_t N, uint32_t N_pad, Arena a, cudaStream_t st);

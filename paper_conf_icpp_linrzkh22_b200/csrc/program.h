@@ -27,7 +27,7 @@ namespace rtlsim {
 enum : uint16_t {
   OP_LD_REG = 32,   // slot d <- state_cur[class][row a..] ; wd width
   OP_LD_X = 33,     // slot d <- xnet[class][row a..]
-  OP_LD_IN = 34,    // slot d <- in_chunk[c][word a..]
+  OP_LD_IN = 34,    // slot d <- input class arena of cycle c [class imm][row a..]
   OP_LD_CONST = 35, // slot d <- const_pool[a..] (broadcast)
   OP_ST_REG = 40,   // state_next[class][row d..] <- slot a ; aux = register word index
   OP_ST_X = 41,     // xnet[class][row d..] <- slot a
@@ -60,13 +60,26 @@ inline double lane_bytes(uint32_t w) {
   return w == 1 ? 0.125 : w <= 8 ? 1.0 : w <= 16 ? 2.0 : 4.0 * nwords(w);
 }
 
-// 32-byte descriptor, read by the kernel as two uint4 (kept in sync with
-// kernels.cuh).
+// slot layout codes (operand / destination addressing in shared memory)
+enum : uint32_t { LC_BIT = 0, LC_U8 = 1, LC_U16 = 2, LC_U32 = 3, LC_CONST = 4 };
+inline uint32_t layout_code(uint32_t w, bool bcast) {
+  return bcast ? LC_CONST : w == 1 ? LC_BIT : w <= 8 ? LC_U8 : w <= 16 ? LC_U16 : LC_U32;
+}
+// descriptor flags (word 0)
+constexpr uint32_t DF_WIDE = 1u << 20;   // some width > 32: generic word-loop path
+constexpr uint32_t DF_HAS_B = 1u << 21;
+constexpr uint32_t DF_HAS_C = 1u << 22;
+
+// 32-byte descriptor, read by the kernel as two uint4:
+//   w0 = op | la << 8 | lb << 11 | lc << 14 | ld << 17 | flags   (compute ops)
+//   w0 = op | class << 17                                          (LD / ST)
+//   wd, wa, wb, wc widths; d, a, b, c slot offsets (or arena rows for LD/ST);
+//   aux = SLICE lo, or the register word index of ST_REG (digest)
 struct Desc {
-  uint16_t op, imm;          // opcode; SLICE lo or arena class
-  uint16_t wd, wa, wb, wc;   // widths (1 => packed bit slot)
-  uint32_t d, a, b, c;       // smem word offsets, or global rows for LD/ST
-  uint32_t aux;              // ST_REG: register word index (digest)
+  uint32_t w0;
+  uint16_t wd, wa, wb, wc;
+  uint32_t d, a, b, c;
+  uint32_t aux;
 };
 static_assert(sizeof(Desc) == 32, "descriptor must be 32 bytes");
 
@@ -87,6 +100,8 @@ struct Program {
   uint32_t rows[4] = {0, 0, 0, 0};      // state arena rows per class
   uint32_t xrows[4] = {0, 0, 0, 0};     // cross-partition net rows per class
   std::vector<RegInfo> regs;            // per register, IR order
+  uint32_t in_rows[4] = {0, 0, 0, 0};   // per-cycle input rows per class
+  std::vector<uint32_t> in_map;         // [IW][2]: class, row of each stimulus word
   std::vector<uint32_t> const_pool;     // words
   // ---- schedule
   uint32_t L = 1;                       // op-lanes (warps) per tile

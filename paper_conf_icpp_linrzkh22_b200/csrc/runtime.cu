@@ -79,13 +79,25 @@ struct rtlsim_ctx {
   uint64_t static_bytes = 0;
   uint32_t N_pad = 0, Tc = 64;
   Arena state[2]{}, xnet{};
-  uint32_t *d_in[2]{}, *d_out[2]{}, *d_raw[2]{}, *d_outu[2]{};
+  Arena d_in[2]{};                    // class-formatted input rows [Tc][rows][N]
+  InStride in_stride{};
+  RegWord *d_inmap = nullptr;
+  uint32_t *d_out[2]{}, *d_raw[2]{}, *d_outu[2]{};
   unsigned long long *d_dig[2]{}, *d_digu[2]{};
   uint32_t *h_in[2]{}, *h_out[2]{};
   unsigned long long *h_dig[2]{};
   cudaEvent_t ev_in_ready[2]{}, ev_comp_done[2]{}, ev_drain_done[2]{}, ev_h2d_copied[2]{}, ev_start = nullptr;
   bool ev_used[2] = {false, false};
   std::map<uint64_t, cudaGraphExec_t> graphs;   // graph mode: key (buf, parity, nc)
+  // RTLSIM_F_TIMING: event pairs around evaluator launches, folded lazily
+  struct Timed {
+    cudaEvent_t a, b;
+    uint64_t stim_cycles;
+  };
+  std::vector<Timed> timed_pending;
+  std::vector<cudaEvent_t> event_pool;
+  double eval_ms = 0;
+  uint64_t eval_launches = 0, eval_stim_cycles = 0;
 };
 
 #define CK(call)                                                                       \
@@ -124,7 +136,8 @@ static void free_binding(rtlsim_ctx *ctx) {
   for (auto &kv : ctx->graphs) cudaGraphExecDestroy(kv.second);
   ctx->graphs.clear();
   for (int b = 0; b < 2; b++) {
-    ctx->d_in[b] = ctx->d_out[b] = ctx->d_raw[b] = ctx->d_outu[b] = nullptr;
+    ctx->d_in[b] = Arena{};
+    ctx->d_out[b] = ctx->d_raw[b] = ctx->d_outu[b] = nullptr;
     ctx->d_dig[b] = ctx->d_digu[b] = nullptr;
     ctx->h_in[b] = ctx->h_out[b] = nullptr;
     ctx->h_dig[b] = nullptr;
@@ -135,6 +148,9 @@ static void free_binding(rtlsim_ctx *ctx) {
   ctx->device_bytes = ctx->static_bytes;
 }
 
+
+// descriptor staging buffers start after the slots, 16-byte aligned
+static uint32_t desc_smem_off(const Program &G) { return (G.smem_words + 3u) & ~3u; }
 
 // ------------------------------------------------------------------ load --
 extern "C" int rtlsim_load(const rtlsim_ir *ir, const rtlsim_options *opt, rtlsim_ctx **out) {
@@ -174,7 +190,14 @@ extern "C" int rtlsim_load(const rtlsim_ir *ir, const rtlsim_options *opt, rtlsi
     return rc;
   }
   Program &G = ctx->prog;
-  ctx->smem_bytes = G.smem_words * 4u;
+  // slots + one 512-byte descriptor staging buffer per op-lane warp
+  ctx->smem_bytes = desc_smem_off(G) * 4u + G.L * 512u;
+  if (ctx->smem_bytes > smem_limit) {
+    g_load_error = "per-tile working set of " + std::to_string(ctx->smem_bytes) +
+                   " bytes (with descriptor buffers) exceeds the shared-memory limit";
+    delete ctx;
+    return RTLSIM_E_NOMEM;
+  }
   if (ctx->opt.chunk_cycles) ctx->Tc = ctx->opt.chunk_cycles;
   if (ctx->host_only) {
     *out = ctx;
@@ -191,7 +214,11 @@ extern "C" int rtlsim_load(const rtlsim_ir *ir, const rtlsim_options *opt, rtlsi
     for (uint32_t t = 0; t < (ri.cls == CLS_U32 ? nwords(ri.width) : 1u); t++)
       regmap[ri.word + t] = RegWord{ri.cls, ri.row + t};
   cudaError_t e = cudaSuccess;
-  if (e == cudaSuccess) e = up((void **)&ctx->d_desc, G.desc.data(), G.desc.size() * sizeof(Desc));
+  // the evaluator prefetches descriptor chunks of 16 past the end: pad
+  std::vector<Desc> padded(G.desc);
+  padded.resize(G.desc.size() + 16, Desc{});
+  if (e == cudaSuccess) e = up((void **)&ctx->d_desc, padded.data(), padded.size() * sizeof(Desc));
+  if (e == cudaSuccess) e = up((void **)&ctx->d_inmap, G.in_map.data(), G.in_map.size() * 4);
   if (e == cudaSuccess) e = up((void **)&ctx->d_step, G.step_ptr.data(), G.step_ptr.size() * 4);
   if (e == cudaSuccess) e = up((void **)&ctx->d_consts, G.const_pool.data(), G.const_pool.size() * 4);
   if (e == cudaSuccess) e = up((void **)&ctx->d_mask, G.in_mask.data(), G.in_mask.size() * 4);
@@ -266,8 +293,15 @@ static int bind_common(rtlsim_ctx *ctx, uint64_t N, uint64_t T) {
     if ((rc = alloc_arena(ctx, &ctx->state[b], G.rows)) != RTLSIM_OK) return rc;
   if ((rc = alloc_arena(ctx, &ctx->xnet, G.xrows)) != RTLSIM_OK) return rc;
   const size_t NP = ctx->N_pad, Tc = ctx->Tc;
+  ctx->in_stride.s[CLS_BIT] = (uint64_t)G.in_rows[CLS_BIT] * (NP / 32);
+  ctx->in_stride.s[CLS_U8] = (uint64_t)G.in_rows[CLS_U8] * NP;
+  ctx->in_stride.s[CLS_U16] = (uint64_t)G.in_rows[CLS_U16] * NP;
+  ctx->in_stride.s[CLS_U32] = (uint64_t)G.in_rows[CLS_U32] * NP;
   for (int b = 0; b < 2; b++) {
-    CK(dalloc(ctx, (void **)&ctx->d_in[b], std::max<size_t>(Tc * G.IW * NP * 4, 16), true));
+    CK(dalloc(ctx, (void **)&ctx->d_in[b].bit, std::max<size_t>(Tc * ctx->in_stride.s[CLS_BIT] * 4, 16), true));
+    CK(dalloc(ctx, (void **)&ctx->d_in[b].u8, std::max<size_t>(Tc * ctx->in_stride.s[CLS_U8], 16), true));
+    CK(dalloc(ctx, (void **)&ctx->d_in[b].u16, std::max<size_t>(Tc * ctx->in_stride.s[CLS_U16] * 2, 16), true));
+    CK(dalloc(ctx, (void **)&ctx->d_in[b].u32, std::max<size_t>(Tc * ctx->in_stride.s[CLS_U32] * 4, 16), true));
     CK(dalloc(ctx, (void **)&ctx->d_out[b], std::max<size_t>(Tc * G.OW * NP * 4, 16), true));
     CK(dalloc(ctx, (void **)&ctx->d_dig[b], Tc * NP * 8, true));
     ctx->ev_used[b] = false;
@@ -348,10 +382,37 @@ static EvalParams eval_params(rtlsim_ctx *ctx, int b, uint64_t cycle0, uint32_t 
   p.state[1] = ctx->state[1];
   p.xnet = ctx->xnet;
   p.in = ctx->d_in[b];
+  for (int k = 0; k < 4; k++) p.in_stride[k] = ctx->in_stride.s[k];
+  p.desc_smem_off = desc_smem_off(G);
   p.out = ctx->d_out[b];
   p.consts = ctx->d_consts;
   p.digest = digest ? ctx->d_dig[b] : nullptr;
   return p;
+}
+
+static cudaError_t get_event(rtlsim_ctx *ctx, cudaEvent_t *e) {
+  if (!ctx->event_pool.empty()) {
+    *e = ctx->event_pool.back();
+    ctx->event_pool.pop_back();
+    return cudaSuccess;
+  }
+  return cudaEventCreate(e);
+}
+
+// fold completed timing events into the totals (blocking on them)
+static int fold_timing(rtlsim_ctx *ctx) {
+  for (auto &t : ctx->timed_pending) {
+    CK(cudaEventSynchronize(t.b));
+    float ms = 0;
+    CK(cudaEventElapsedTime(&ms, t.a, t.b));
+    ctx->eval_ms += ms;
+    ctx->eval_launches++;
+    ctx->eval_stim_cycles += t.stim_cycles;
+    ctx->event_pool.push_back(t.a);
+    ctx->event_pool.push_back(t.b);
+  }
+  ctx->timed_pending.clear();
+  return RTLSIM_OK;
 }
 
 // simulate chunk (cycle0, nc) from d_in[b] into d_out[b] / d_dig[b] on ctx->st
@@ -359,10 +420,21 @@ static int launch_chunk(rtlsim_ctx *ctx, int b, uint64_t cycle0, uint32_t nc, bo
   Program &G = ctx->prog;
   if (digest) CK(cudaMemsetAsync(ctx->d_dig[b], 0, (size_t)nc * ctx->N_pad * 8, ctx->st));
   if (G.n_steps == 0) return RTLSIM_OK;
+  const bool timing = (ctx->opt.flags & RTLSIM_F_TIMING) != 0;
+  rtlsim_ctx::Timed tm{nullptr, nullptr, (uint64_t)nc * ctx->N};
+  if (timing) {
+    CK(get_event(ctx, &tm.a));
+    CK(get_event(ctx, &tm.b));
+    CK(cudaEventRecord(tm.a, ctx->st));
+  }
   if (!(ctx->opt.flags & RTLSIM_F_GRAPH)) {
     EvalParams p = eval_params(ctx, b, cycle0, nc, digest);
     CK(launch_eval(p, ctx->smem_bytes, ctx->st));
     ctx->launches++;
+    if (timing) {
+      CK(cudaEventRecord(tm.b, ctx->st));
+      ctx->timed_pending.push_back(tm);
+    }
     return RTLSIM_OK;
   }
   // graph mode: Tc x P per-(cycle, partition) nodes, captured once per
@@ -380,7 +452,10 @@ static int launch_chunk(rtlsim_ctx *ctx, int b, uint64_t cycle0, uint32_t nc, bo
         EvalParams p = eval_params(ctx, b, (cycle0 & 1ull) + c, 1, digest);
         p.step_begin = G.part_steps[q];
         p.step_end = G.part_steps[q + 1];
-        p.in = ctx->d_in[b] + (size_t)c * G.IW * ctx->N_pad;
+        p.in.bit = ctx->d_in[b].bit + (size_t)c * ctx->in_stride.s[CLS_BIT];
+        p.in.u8 = ctx->d_in[b].u8 + (size_t)c * ctx->in_stride.s[CLS_U8];
+        p.in.u16 = ctx->d_in[b].u16 + (size_t)c * ctx->in_stride.s[CLS_U16];
+        p.in.u32 = ctx->d_in[b].u32 + (size_t)c * ctx->in_stride.s[CLS_U32];
         p.out = ctx->d_out[b] + (size_t)c * G.OW * ctx->N_pad;
         if (digest) p.digest = ctx->d_dig[b] + (size_t)c * ctx->N_pad;
         cudaError_t e = launch_eval(p, ctx->smem_bytes, cap);
@@ -401,6 +476,10 @@ static int launch_chunk(rtlsim_ctx *ctx, int b, uint64_t cycle0, uint32_t nc, bo
   }
   CK(cudaGraphLaunch(it->second, ctx->st));
   ctx->launches += (uint64_t)nc * (G.part_steps.size() - 1);
+  if (timing) {
+    CK(cudaEventRecord(tm.b, ctx->st));
+    ctx->timed_pending.push_back(tm);
+  }
   return RTLSIM_OK;
 }
 
@@ -487,7 +566,8 @@ static int run_impl(rtlsim_ctx *ctx, uint64_t cycles, const Dest &dst, bool dige
         src = ctx->d_raw[b];
         pitch = (uint64_t)nc * IW;
       }
-      CK(launch_stim_transpose(src, pitch, N, NP, nc, IW, ctx->d_mask, ctx->d_in[b], ctx->st_h2d));
+      CK(launch_stim_transpose(src, pitch, N, NP, nc, IW, ctx->d_mask, ctx->d_inmap, ctx->d_in[b], ctx->in_stride,
+                               ctx->st_h2d));
       ctx->launches++;
     }
     CK(cudaEventRecord(ctx->ev_in_ready[b], ctx->st_h2d));
@@ -647,8 +727,13 @@ extern "C" int rtlsim_reset(rtlsim_ctx *ctx) {
 }
 
 // ---------------------------------------------------------------- misc --
-extern "C" int rtlsim_stats(const rtlsim_ctx *ctx, rtlsim_stats_t *st) {
-  if (!ctx || !st) return RTLSIM_E_ARG;
+extern "C" int rtlsim_stats(const rtlsim_ctx *cctx, rtlsim_stats_t *st) {
+  if (!cctx || !st) return RTLSIM_E_ARG;
+  rtlsim_ctx *ctx = const_cast<rtlsim_ctx *>(cctx);
+  if (!ctx->failed && !ctx->timed_pending.empty()) {
+    int rc = fold_timing(ctx);
+    if (rc) return rc;
+  }
   const Program &G = ctx->prog;
   memset(st, 0, sizeof *st);
   st->n_ops = G.n_ops;
@@ -671,6 +756,9 @@ extern "C" int rtlsim_stats(const rtlsim_ctx *ctx, rtlsim_stats_t *st) {
   st->tile_stimuli = 32;
   st->iw = G.IW; st->ow = G.OW; st->rw = G.RW;
   st->device_bytes = ctx->device_bytes;
+  st->eval_ms = ctx->eval_ms;
+  st->eval_launches = ctx->eval_launches;
+  st->eval_stim_cycles = ctx->eval_stim_cycles;
   return RTLSIM_OK;
 }
 
@@ -688,6 +776,11 @@ extern "C" void rtlsim_free(rtlsim_ctx *ctx) {
     if (ctx->st_h2d) cudaStreamSynchronize(ctx->st_h2d);
     if (ctx->st_d2h) cudaStreamSynchronize(ctx->st_d2h);
     free_binding(ctx);
+    for (auto &t : ctx->timed_pending) {
+      cudaEventDestroy(t.a);
+      cudaEventDestroy(t.b);
+    }
+    for (cudaEvent_t e : ctx->event_pool) cudaEventDestroy(e);
     for (void *p : ctx->dev_allocs) cudaFree(p);
     for (int b = 0; b < 2; b++) {
       if (ctx->ev_in_ready[b]) cudaEventDestroy(ctx->ev_in_ready[b]);
