@@ -27,6 +27,9 @@
 
 namespace rtlsim {
 
+// external values whose uses are more than this many steps apart are reloaded
+constexpr int32_t kReloadGap = 3;
+
 static int arity(uint32_t opc) {
   switch (opc) {
     case RTLSIM_OP_COPY: case RTLSIM_OP_SEXT: case RTLSIM_OP_NOT: case RTLSIM_OP_NEG:
@@ -49,11 +52,11 @@ namespace {
 struct Value {
   uint32_t sig;        // IR signal (or the register's q for synthesized copies)
   uint32_t width;
-  int32_t def_step;    // step that writes the slot
+  int32_t def_step;    // step that writes the slot (-1: immediate)
   int32_t last_use;    // last step that reads it (-1: dead)
-  uint32_t slot;       // smem word offset
-  bool bcast;          // constant: one copy of the words for all 32 stimuli
-  uint32_t words() const { return slot_words(width, bcast); }
+  uint32_t slot;       // smem word offset (the value itself for LC_IMM)
+  uint32_t layout;     // LC_*
+  uint32_t words() const { return slot_words(layout, width); }
 };
 
 // First-fit allocator over shared-memory words.
@@ -337,15 +340,15 @@ int compile_program(const rtlsim_ir *ir, uint32_t op_lanes, uint32_t smem_limit_
     for (uint32_t o = 0; o < ir->n_outputs; o++) used[G.output_sig[o]] = 1;
     for (uint32_t i = 0; i < G.n_ops; i++) {
       uint32_t d = G.ops[i].dst;
-      if (!used[d]) dump_words = std::max(dump_words, slot_words(G.width[d], false));
+      if (!used[d]) dump_words = std::max(dump_words, slot_words(value_layout(G.width[d], false), G.width[d]));
     }
   }
 
-  struct StepDesc {
-    Desc d;
-    uint32_t cost;
+  struct StepLists {
+    std::vector<std::pair<Desc, uint32_t>> lane;   // descriptor, cost
+    std::vector<BitDesc> bits;
   };
-  std::vector<std::vector<StepDesc>> all_steps;   // global step list
+  std::vector<StepLists> all_steps;   // global step list
   uint32_t peak = dump_words;
   G.part_steps.push_back(0);
   double bytes_state = 0, bytes_part = 0;
@@ -356,14 +359,13 @@ int compile_program(const rtlsim_ir *ir, uint32_t op_lanes, uint32_t smem_limit_
     std::vector<Value> vals;
     std::vector<uint32_t> touched;
     auto vid = [&](uint32_t s) -> int32_t { return vid_of[s]; };
-    auto new_val = [&](uint32_t s, uint32_t w, int32_t def_step) -> int32_t {
-      vals.push_back(Value{s, w, def_step, -1, 0, false});
+    auto new_val = [&](uint32_t s, uint32_t w, int32_t def_step, uint32_t layout) -> int32_t {
+      vals.push_back(Value{s, w, def_step, -1, 0, layout});
       return (int32_t)vals.size() - 1;
     };
-    // 1. levels of the partition's own ops
-    std::vector<int32_t> step_of_op;   // parallel to ops_p
-    step_of_op.reserve(ops_p.size());
+    // 1. levels of the partition's own ops (ASAP)
     std::unordered_map<uint32_t, int32_t> op_step;   // op index -> step
+    op_step.reserve(ops_p.size());
     for (uint32_t i : ops_p) {
       const rtlsim_op &o = G.ops[i];
       uint32_t src[3] = {o.a, o.b, o.c};
@@ -378,8 +380,9 @@ int compile_program(const rtlsim_ir *ir, uint32_t op_lanes, uint32_t smem_limit_
     // shared-memory working set): an op whose result feeds later ops of this
     // partition runs one step before its earliest consumer (ALAP, so loads
     // and producers move next to their use); an op whose result only leaves
-    // the partition (register D, output, cross-partition net) or is dead
-    // keeps its earliest step so its operand cone is not dragged late.
+    // the partition (register D, output, cross-partition net) or is dead runs
+    // right after its latest local operand, or, with none, round-robin over
+    // the partition's steps (no bunching at step 1).
     {
       std::unordered_map<uint32_t, int32_t> first_use;   // op -> earliest consumer step
       first_use.reserve(ops_p.size());
@@ -398,9 +401,6 @@ int compile_program(const rtlsim_ir *ir, uint32_t op_lanes, uint32_t smem_limit_
           }
         }
       }
-      // second pass, forward: ops without local consumers run right after
-      // their latest local operand; those with only external operands are
-      // spread round-robin over the partition's steps (no bunching at step 1)
       int32_t depth = 1;
       for (uint32_t i : ops_p) depth = std::max(depth, op_step[i]);
       uint32_t rr = 0;
@@ -417,28 +417,31 @@ int compile_program(const rtlsim_ir *ir, uint32_t op_lanes, uint32_t smem_limit_
       }
     }
     for (uint32_t i : ops_p) {
-      int32_t v = new_val(G.ops[i].dst, G.width[G.ops[i].dst], op_step[i]);
-      vid_of[G.ops[i].dst] = v;
-      touched.push_back(G.ops[i].dst);
+      const uint32_t d = G.ops[i].dst;
+      vid_of[d] = new_val(d, G.width[d], op_step[i], value_layout(G.width[d], false));
+      touched.push_back(d);
     }
-    // 2. external operands (registers, inputs, constants, other partitions'
-    //    nets): loaded into a slot one step before use. Uses further apart
-    //    than `reload_gap` steps get separate loads (a reload hits L1/L2) so
-    //    the value does not occupy shared memory in between.
     auto is_local = [&](uint32_t s) { return G.kind[s] == RTLSIM_COMB && G.ops[def[s]].part == p; };
+    auto is_imm = [&](uint32_t s) { return G.kind[s] == RTLSIM_CONST && G.width[s] <= 16; };
+    // 2. external operands (registers, inputs, constants > 16 bits, other
+    //    partitions' nets): loaded into a slot one step before use. Uses
+    //    further apart than kReloadGap steps get separate loads (a reload hits
+    //    L1/L2) so the value does not occupy shared memory in between.
+    //    Constants <= 16 bits are immediates in the descriptors.
     std::unordered_map<uint32_t, std::vector<int32_t>> ext_uses;   // signal -> op use steps
     for (uint32_t i : ops_p) {
       const rtlsim_op &o = G.ops[i];
       uint32_t src[3] = {o.a, o.b, o.c};
       for (int k = 0; k < arity(o.opcode); k++)
-        if (!is_local(src[k])) ext_uses[src[k]].push_back(op_step[i]);
+        if (!is_local(src[k]) && !is_imm(src[k])) ext_uses[src[k]].push_back(op_step[i]);
     }
-    // sinks: register next state, outputs, cross-partition nets; width
-    // conversions (w_d != w_q) are synthesized COPY ops
+    // sinks: register next state, outputs, cross-partition nets. A sink
+    // whose source has another width (register q <= d mod 2^w_q) or is a
+    // constant reads a synthesized COPY.
     struct Sink {
-      uint16_t op;       // OP_ST_REG / OP_ST_OUT / OP_ST_X
+      uint32_t code;     // CODE_ST_REG / CODE_ST_OUT / CODE_ST_X
       uint32_t src_sig;  // signal whose value is stored
-      int32_t src_val;   // value id (after conversion), -2-k: synthesized copy k
+      int32_t src_val;   // value id; -2-k: synthesized copy k
       uint32_t idx;      // register or output index, or xnet signal
     };
     std::vector<Sink> sinks;
@@ -447,22 +450,28 @@ int compile_program(const rtlsim_ir *ir, uint32_t op_lanes, uint32_t smem_limit_
       int32_t val, step;
     };
     std::vector<Synth> synth;
-    for (uint32_t r : reg_sinks[p]) {
-      uint32_t d = G.reg_d[r], wq = G.width[G.reg_q[r]];
-      sinks.push_back(Sink{OP_ST_REG, d, -1, r});
-      if (G.width[d] != wq) {
-        synth.push_back(Synth{d, wq, -1, is_local(d) ? op_step[def[d]] + 1 : -1});
+    auto add_sink = [&](uint32_t code, uint32_t s, uint32_t w_target, uint32_t idx) {
+      sinks.push_back(Sink{code, s, -1, idx});
+      if (G.width[s] != w_target || G.kind[s] == RTLSIM_CONST) {
+        synth.push_back(Synth{s, w_target, -1, is_local(s) ? op_step[def[s]] + 1 : -1});
         sinks.back().src_val = -2 - (int32_t)(synth.size() - 1);
       }
-      if (!is_local(d)) ext_uses[d];   // ensure a load exists
-    }
-    for (uint32_t o : out_sinks[p]) {
-      uint32_t s = G.output_sig[o];
-      sinks.push_back(Sink{OP_ST_OUT, s, -1, o});
-      if (!is_local(s)) ext_uses[s];
-    }
+      if (!is_local(s) && !is_imm(s)) ext_uses[s];   // ensure a load exists
+    };
+    for (uint32_t r : reg_sinks[p]) add_sink(CODE_ST_REG, G.reg_d[r], G.width[G.reg_q[r]], r);
+    for (uint32_t o : out_sinks[p]) add_sink(CODE_ST_OUT, G.output_sig[o], G.width[G.output_sig[o]], o);
     for (uint32_t i : ops_p)
-      if (is_xnet[G.ops[i].dst]) sinks.push_back(Sink{OP_ST_X, G.ops[i].dst, -1, G.ops[i].dst});
+      if (is_xnet[G.ops[i].dst]) add_sink(CODE_ST_X, G.ops[i].dst, G.width[G.ops[i].dst], G.ops[i].dst);
+    // immediates: one pseudo-value per constant, always available, no slot
+    std::unordered_map<uint32_t, int32_t> imm_val;
+    auto imm_of = [&](uint32_t s) -> int32_t {
+      auto it = imm_val.find(s);
+      if (it != imm_val.end()) return it->second;
+      int32_t v = new_val(s, G.width[s], -1, LC_IMM);
+      vals[v].slot = G.const_words[(uint32_t)const_of[s]] & (G.width[s] == 32 ? 0xFFFFFFFFu : ((1u << G.width[s]) - 1u));
+      imm_val[s] = v;
+      return v;
+    };
     // load groups
     struct Load {
       uint32_t sig;
@@ -489,30 +498,34 @@ int compile_program(const rtlsim_ir *ir, uint32_t op_lanes, uint32_t smem_limit_
           if (gs.empty() || st - gs.back().last > (int32_t)kReloadGap) gs.push_back(Group{st, st, -1});
           else gs.back().last = st;
         }
-        for (Group &g : gs) {
-          g.val = new_val(s, G.width[s], g.first - 1);
-          vals[g.val].last_use = g.last;
-          vals[g.val].bcast = G.kind[s] == RTLSIM_CONST && G.width[s] > 1;
-          loads.push_back(Load{s, g.val, g.first - 1, &g == &gs.front()});
+        for (size_t g = 0; g < gs.size(); g++) {
+          gs[g].val = new_val(s, G.width[s], gs[g].first - 1, value_layout(G.width[s], G.kind[s] == RTLSIM_CONST));
+          vals[gs[g].val].last_use = gs[g].last;
+          loads.push_back(Load{s, gs[g].val, gs[g].first - 1, g == 0});
         }
         groups[s] = std::move(gs);
-        touched.push_back(s);
       }
     }
-    // value holding signal s at step st (local comb or the covering load)
+    // value holding signal s at step st (local comb, immediate, or the covering load)
     auto val_at = [&](uint32_t s, int32_t st) -> int32_t {
       if (is_local(s)) return vid(s);
+      if (is_imm(s)) return imm_of(s);
       const std::vector<Group> &gs = groups.at(s);
       for (const Group &g : gs)
         if (st >= g.first - 1 && st <= g.last) return g.val;
       return gs.front().val;
     };
+    auto flex_src = [&](uint32_t s) -> int32_t {   // first value of s in this partition
+      if (is_local(s)) return vid(s);
+      if (is_imm(s)) return imm_of(s);
+      return groups.at(s).front().val;
+    };
     // flexible consumers of an external value (sinks, conversion copies) read
     // the first load group, one step after the load
     for (auto &sy : synth) {
-      int32_t src = is_local(sy.src_sig) ? vid(sy.src_sig) : groups.at(sy.src_sig).front().val;
-      if (sy.step < 0) sy.step = vals[src].def_step + 1;
-      sy.val = new_val(sy.src_sig, sy.w, sy.step);
+      int32_t src = flex_src(sy.src_sig);
+      if (sy.step < 0) sy.step = std::max(vals[src].def_step, 0) + 1;
+      sy.val = new_val(sy.src_sig, sy.w, sy.step, value_layout(sy.w, false));
       vals[src].last_use = std::max(vals[src].last_use, sy.step);
     }
     // 3. uses by ops
@@ -531,19 +544,20 @@ int compile_program(const rtlsim_ir *ir, uint32_t op_lanes, uint32_t smem_limit_
     std::vector<int32_t> sink_step(sinks.size());
     for (size_t k = 0; k < sinks.size(); k++) {
       Sink &sk = sinks[k];
-      int32_t v = sk.src_val <= -2 ? synth[-2 - sk.src_val].val
-                  : (is_local(sk.src_sig) ? vid(sk.src_sig) : groups.at(sk.src_sig).front().val);
+      int32_t v = sk.src_val <= -2 ? synth[-2 - sk.src_val].val : flex_src(sk.src_sig);
       sk.src_val = v;
-      sink_step[k] = vals[v].def_step + 1;
+      sink_step[k] = std::max(vals[v].def_step, 0) + 1;
       vals[v].last_use = std::max(vals[v].last_use, sink_step[k]);
     }
     // 5. number of steps
     int32_t nsteps = 0;
     for (auto &v : vals) nsteps = std::max(nsteps, std::max(v.def_step, v.last_use) + 1);
-    // 6. slot allocation by liveness (dead values go to the dump region)
+    // 6. slot allocation by liveness (dead values go to the dump region,
+    //    immediates take no slot)
     {
       std::vector<std::vector<int32_t>> born(nsteps), dies(nsteps);
       for (size_t v = 0; v < vals.size(); v++) {
+        if (vals[v].layout == LC_IMM) continue;
         if (vals[v].last_use < 0) {
           vals[v].slot = 0;   // dump
           continue;
@@ -552,25 +566,6 @@ int compile_program(const rtlsim_ir *ir, uint32_t op_lanes, uint32_t smem_limit_
         dies[vals[v].last_use].push_back((int32_t)v);
       }
       SlotAlloc sa(dump_words);
-      if (getenv("RTLSIM_DEBUG_LIVE")) {
-        // live words per step by kind: reg/input/const/xnet loads vs comb values
-        std::vector<std::array<double, 6>> live(nsteps);
-        for (auto &v : vals) {
-          if (v.last_use < 0) continue;
-          int kd = v.def_step == 0 && false ? 0 : (G.kind[v.sig] == RTLSIM_COMB ? (is_local(v.sig) ? 4 : 3) : G.kind[v.sig]);
-          for (int32_t t = v.def_step; t <= v.last_use; t++) live[t][kd] += v.words();
-        }
-        int32_t best = 0;
-        double bw = 0;
-        for (int32_t t = 0; t < nsteps; t++) {
-          double tot = 0;
-          for (double x : live[t]) tot += x;
-          if (tot > bw) { bw = tot; best = t; }
-        }
-        fprintf(stderr, "part %u steps %d peak step %d words %.0f: in %.0f reg %.0f comb_local %.0f xnet %.0f const %.0f\n",
-                p, nsteps, best, bw, live[best][RTLSIM_INPUT], live[best][RTLSIM_REG], live[best][4], live[best][3],
-                live[best][RTLSIM_CONST]);
-      }
       for (int32_t s = 0; s < nsteps; s++) {
         // largest first keeps wide values contiguous and packs better
         std::sort(born[s].begin(), born[s].end(),
@@ -581,134 +576,183 @@ int compile_program(const rtlsim_ir *ir, uint32_t op_lanes, uint32_t smem_limit_
       peak = std::max(peak, sa.peak);
     }
     // 7. descriptors per step
-    std::vector<std::vector<StepDesc>> steps(nsteps);
-    // operand address: broadcast (constant) slots carry kConstSlot
-    auto operand = [&](int32_t v) -> uint32_t { return vals[v].slot | (vals[v].bcast ? kConstSlot : 0u); };
+    std::vector<StepLists> steps(nsteps);
     for (const Load &ld : loads) {
-      uint32_t s = ld.sig, w = G.width[s];
+      const uint32_t s = ld.sig, w = G.width[s];
       Desc d{};
-      d.wd = (uint16_t)w;
-      d.d = vals[ld.val].slot;   // LD_CONST writes the broadcast layout
-      uint32_t op;
+      d.y = vals[ld.val].slot;
+      uint32_t code;
       if (G.kind[s] == RTLSIM_REG) {
-        const RegInfo &ri = G.regs[reg_of[s]];
-        op = OP_LD_REG; d.a = ri.row;
+        code = CODE_LD_REG;
+        d.z = G.regs[reg_of[s]].row;
         if (ld.first) bytes_state += lane_bytes(w);
       } else if (G.kind[s] == RTLSIM_INPUT) {
-        op = OP_LD_IN; d.a = input_row[s];
+        code = CODE_LD_IN;
+        d.z = input_row[s];
         if (ld.first) bytes_state += lane_bytes(w);
       } else if (G.kind[s] == RTLSIM_CONST) {
-        op = OP_LD_CONST; d.a = (uint32_t)const_of[s];
+        code = CODE_LD_CONST;
+        d.z = (uint32_t)const_of[s];
       } else {
-        op = OP_LD_X; d.a = xrow.at(s);
+        code = CODE_LD_X;
+        d.z = xrow.at(s);
         if (ld.first) {
           bytes_state += lane_bytes(w);
           bytes_part += lane_bytes(w);
         }
       }
-      d.w0 = op | ((uint32_t)width_class(w) << 17);
-      steps[ld.step].push_back(StepDesc{d, nwords(w)});
+      d.x = code | (width_class(w) << 8) | (nwords(w) << 12) | ((vals[ld.val].layout == LC_BCAST ? 1u : 0u) << 18);
+      G.n_ld++;
+      steps[ld.step].lane.push_back({d, 1 + nwords(w)});
     }
-    // compute descriptor: widths, slot offsets, layout codes and flags
-    auto compute_desc = [&](uint32_t opc, uint32_t wd, int32_t vd, int ar, const int32_t *src,
-                            uint32_t imm) -> Desc {
-      Desc d{};
-      d.wd = (uint16_t)wd;
-      d.d = vals[vd].slot;
-      uint32_t w0 = opc | (layout_code(wd, false) << 17);
-      bool wide = wd > 32;
-      const uint32_t sh[3] = {8, 11, 14};
-      uint16_t *ws[3] = {&d.wa, &d.wb, &d.wc};
-      uint32_t *os[3] = {&d.a, &d.b, &d.c};
+    // compute op -> bit-sliced, narrow or wide descriptor
+    auto emit_compute = [&](uint32_t opc, int32_t vd, int ar, const int32_t *src, uint32_t imm, int32_t step) {
+      const Value &D = vals[vd];
+      bool allbit = D.width == 1, narrow = D.width <= 32;
       for (int k = 0; k < ar; k++) {
         const Value &v = vals[src[k]];
-        *ws[k] = (uint16_t)v.width;
-        *os[k] = operand(src[k]);
-        w0 |= layout_code(v.width, v.bcast) << sh[k];
-        wide = wide || v.width > 32;
+        allbit = allbit && v.width == 1;
+        narrow = narrow && v.width <= 32 && v.layout != LC_BCAST;
       }
-      if (ar >= 2) w0 |= DF_HAS_B;
-      if (ar >= 3) w0 |= DF_HAS_C;
-      if (wide) w0 |= DF_WIDE;
-      d.w0 = w0;
-      d.aux = imm;
-      return d;
+      uint32_t wmax = D.width;
+      for (int k = 0; k < std::min(ar, 2); k++) wmax = std::max(wmax, vals[src[k]].width);
+      G.word_ops += nwords(wmax);
+      if (allbit) {
+        BitDesc b{};
+        uint32_t f[3] = {0, 0, 0}, immf = 0;
+        for (int k = 0; k < ar; k++) {
+          f[k] = vals[src[k]].slot;
+          if (vals[src[k]].layout == LC_IMM) immf |= 1u << k;
+        }
+        b.x = bit_lut(opc) | (immf << 8);
+        b.y = D.slot | (f[0] << 16);
+        b.z = f[1] | (f[2] << 16);
+        steps[step].bits.push_back(b);
+        G.n_bitops++;
+        return;
+      }
+      if (narrow) {
+        Desc d{};
+        uint32_t lay[3] = {0, 0, 0}, off[3] = {0, 0, 0}, wsrc[3] = {1, 1, 1};
+        for (int k = 0; k < ar; k++) {
+          lay[k] = vals[src[k]].layout;
+          off[k] = vals[src[k]].slot;
+          wsrc[k] = vals[src[k]].width;
+        }
+        d.x = opc | (lay[0] << 8) | (lay[1] << 11) | (lay[2] << 14) | (D.layout << 17) | (D.width << 20) |
+              (wsrc[0] << 26);
+        d.y = D.slot | (off[0] << 16);
+        d.z = off[1] | (off[2] << 16);
+        d.w = wsrc[1] | (imm << 6) | ((ar >= 2 ? 1u : 0u) << 11) | ((ar >= 3 ? 1u : 0u) << 12);
+        G.n_narrow++;
+        uint32_t cost = (opc == RTLSIM_OP_DIVU || opc == RTLSIM_OP_MODU) ? 6 : 2;
+        steps[step].lane.push_back({d, cost});
+        return;
+      }
+      WideRec r{};
+      r.op = opc;
+      r.wd = (uint16_t)D.width;
+      r.d = D.slot;
+      uint16_t *ws[3] = {&r.wa, &r.wb, &r.wc};
+      uint32_t *os[3] = {&r.a, &r.b, &r.c};
+      for (int k = 0; k < ar; k++) {
+        *ws[k] = (uint16_t)vals[src[k]].width;
+        *os[k] = vals[src[k]].slot;
+        r.lays |= vals[src[k]].layout << (8 * k);
+      }
+      r.imm = imm;
+      Desc d{};
+      d.x = CODE_WIDE;
+      d.y = (uint32_t)G.wide.size();
+      G.wide.push_back(r);
+      G.n_wide++;
+      steps[step].lane.push_back({d, 4 + 2 * nwords(wmax)});
     };
     for (size_t j = 0; j < ops_p.size(); j++) {
       const uint32_t i = ops_p[j];
       const rtlsim_op &o = G.ops[i];
-      const int ar = arity(o.opcode);
-      Desc d = compute_desc(o.opcode, G.width[o.dst], vid(o.dst), ar, op_vals[j].data(),
-                            o.opcode == RTLSIM_OP_SLICE ? o.imm : 0u);
-      uint32_t wmax = std::max<uint32_t>(d.wd, std::max<uint32_t>(d.wa, d.wb));
-      uint32_t cost = nwords(wmax);
-      G.word_ops += cost;
-      if (o.opcode == RTLSIM_OP_MUL || o.opcode == RTLSIM_OP_DIVU || o.opcode == RTLSIM_OP_MODU) cost += 4;
-      if (d.w0 & DF_WIDE) cost += 2;
-      steps[op_step[i]].push_back(StepDesc{d, cost});
+      emit_compute(o.opcode, vid(o.dst), arity(o.opcode), op_vals[j].data(),
+                   o.opcode == RTLSIM_OP_SLICE ? o.imm : 0u, op_step[i]);
     }
     for (const Synth &sy : synth) {
-      const int32_t src = is_local(sy.src_sig) ? vid(sy.src_sig) : groups.at(sy.src_sig).front().val;
-      Desc d = compute_desc(RTLSIM_OP_COPY, sy.w, sy.val, 1, &src, 0u);
-      steps[sy.step].push_back(StepDesc{d, nwords(std::max(sy.w, (uint32_t)d.wa))});
+      const int32_t src = flex_src(sy.src_sig);
+      emit_compute(RTLSIM_OP_COPY, sy.val, 1, &src, 0u, sy.step);
     }
     for (size_t k = 0; k < sinks.size(); k++) {
       const Sink &sk = sinks[k];
+      const Value &v = vals[sk.src_val];
       Desc d{};
-      d.a = operand(sk.src_val);
-      uint32_t op = sk.op;
-      if (sk.op == OP_ST_REG) {
+      d.y = v.slot;
+      const uint32_t w = v.width;
+      if (sk.code == CODE_ST_REG) {
         const RegInfo &ri = G.regs[sk.idx];
-        d.wd = (uint16_t)ri.width; d.d = ri.row; d.aux = ri.word;
+        d.z = ri.row;
+        d.w = ri.word;
         bytes_state += lane_bytes(ri.width);
-      } else if (sk.op == OP_ST_OUT) {
-        d.wd = G.width[G.output_sig[sk.idx]]; d.d = out_word[sk.idx];
-        bytes_state += 4.0 * nwords(d.wd);
+      } else if (sk.code == CODE_ST_OUT) {
+        d.z = out_word[sk.idx];
+        bytes_state += 4.0 * nwords(w);
       } else {
-        d.wd = G.width[sk.idx]; d.d = xrow.at(sk.idx);
-        bytes_state += lane_bytes(d.wd);
-        bytes_part += lane_bytes(d.wd);
+        d.z = xrow.at(sk.idx);
+        bytes_state += lane_bytes(w);
+        bytes_part += lane_bytes(w);
       }
-      d.w0 = op | ((uint32_t)width_class(d.wd) << 17);
-      steps[sink_step[k]].push_back(StepDesc{d, nwords(d.wd)});
+      d.x = sk.code | (width_class(w) << 8) | (nwords(w) << 12) | (v.layout << 18);
+      G.n_st++;
+      steps[sink_step[k]].lane.push_back({d, 1 + nwords(w)});
     }
     for (auto &st : steps)
-      if (!st.empty()) all_steps.push_back(std::move(st));
+      if (!st.lane.empty() || !st.bits.empty()) all_steps.push_back(std::move(st));
     G.part_steps.push_back((uint32_t)all_steps.size());
     for (uint32_t s : touched) vid_of[s] = -1;
+    for (auto &kv : groups) vid_of[kv.first] = -1;
   }
 
   // -------------------------------------------------------- op lanes --
   size_t total = 0;
-  for (auto &st : all_steps) total += st.size();
+  for (auto &st : all_steps) total += st.lane.size() + st.bits.size() / 8;
   uint32_t L = op_lanes;
   if (L == 0) {
     double avg = all_steps.empty() ? 1.0 : (double)total / (double)all_steps.size();
     L = (uint32_t)std::max(1.0, std::min(16.0, avg / 8.0));
   }
-  L = std::max<uint32_t>(1, std::min<uint32_t>(32, L));
+  L = std::max<uint32_t>(1, std::min<uint32_t>(16, L));
   G.L = L;
   G.n_steps = (uint32_t)all_steps.size();
-  G.step_ptr.reserve((size_t)G.n_steps * (L + 1));
+  G.step_ptr.reserve((size_t)G.n_steps * L + 1);
   G.desc.reserve(total);
+  G.bit_ptr.reserve(G.n_steps + 1);
   for (auto &st : all_steps) {
+    G.bit_ptr.push_back((uint32_t)G.bitdesc.size());
+    G.bitdesc.insert(G.bitdesc.end(), st.bits.begin(), st.bits.end());
     // longest-processing-time-first onto the least loaded lane
-    std::stable_sort(st.begin(), st.end(), [](const StepDesc &x, const StepDesc &y) { return x.cost > y.cost; });
+    std::stable_sort(st.lane.begin(), st.lane.end(),
+                     [](const std::pair<Desc, uint32_t> &x, const std::pair<Desc, uint32_t> &y) {
+                       return x.second > y.second;
+                     });
     std::vector<std::vector<Desc>> lanes(L);
     std::vector<uint64_t> load(L, 0);
-    for (auto &sd : st) {
+    for (auto &sd : st.lane) {
       uint32_t best = (uint32_t)(std::min_element(load.begin(), load.end()) - load.begin());
-      lanes[best].push_back(sd.d);
-      load[best] += sd.cost;
+      lanes[best].push_back(sd.first);
+      load[best] += sd.second;
     }
     for (uint32_t l = 0; l < L; l++) {
       G.step_ptr.push_back((uint32_t)G.desc.size());
+      // loads first (their latency overlaps the step's compute; they are
+      // awaited once at the step barrier), then compute ops grouped by code
+      // (fewer divergent dispatch paths), stores last
+      auto rank = [](const Desc &d) -> uint32_t {
+        const uint32_t c = d.x & 0xFFu;
+        return (c >= CODE_LD_REG && c <= CODE_LD_CONST) ? c - CODE_LD_REG : 16u + c;
+      };
       std::stable_sort(lanes[l].begin(), lanes[l].end(),
-                       [](const Desc &x, const Desc &y) { return (x.w0 & 0xFFu) < (y.w0 & 0xFFu); });
+                       [&](const Desc &x, const Desc &y) { return rank(x) < rank(y); });
       G.desc.insert(G.desc.end(), lanes[l].begin(), lanes[l].end());
     }
   }
   G.step_ptr.push_back((uint32_t)G.desc.size());
+  G.bit_ptr.push_back((uint32_t)G.bitdesc.size());
   G.smem_words = std::max<uint32_t>(peak, 1);
   if (smem_limit_words && G.smem_words > smem_limit_words)
     return fail(err, RTLSIM_E_NOMEM,
@@ -724,6 +768,41 @@ int compile_program(const rtlsim_ir *ir, uint32_t op_lanes, uint32_t smem_limit_
   G.b_state = bytes_state;
   G.b_part = bytes_part;
   return RTLSIM_OK;
+}
+
+// Truth table of an op on 1-bit operands / 1-bit result (DESIGN.md §3 table
+// restricted to width 1): bit k = f(a = k & 1, b = (k >> 1) & 1, c = k >> 2).
+uint32_t bit_lut(uint32_t opc) {
+  uint32_t lut = 0;
+  for (uint32_t k = 0; k < 8; k++) {
+    const uint32_t a = k & 1u, b = (k >> 1) & 1u, c = (k >> 2) & 1u;
+    uint32_t r = 0;
+    switch (opc) {
+      case RTLSIM_OP_COPY: case RTLSIM_OP_SEXT: case RTLSIM_OP_NEG: case RTLSIM_OP_SLICE:
+      case RTLSIM_OP_REDAND: case RTLSIM_OP_REDOR: case RTLSIM_OP_REDXOR: case RTLSIM_OP_SHRA:
+        r = a; break;                                   // SHRA: b >= 1 fills with the sign = a
+      case RTLSIM_OP_NOT: r = a ^ 1u; break;
+      case RTLSIM_OP_AND: case RTLSIM_OP_MUL: case RTLSIM_OP_DIVU: r = a & b; break;   // a/1 = a, a/0 = 0
+      case RTLSIM_OP_OR: r = a | b; break;
+      case RTLSIM_OP_XOR: case RTLSIM_OP_ADD: case RTLSIM_OP_SUB: case RTLSIM_OP_NE: r = a ^ b; break;
+      case RTLSIM_OP_MODU: r = 0; break;               // a % 1 = 0, a % 0 = 0
+      case RTLSIM_OP_EQ: r = (a ^ b) ^ 1u; break;
+      case RTLSIM_OP_LTU: r = (a ^ 1u) & b; break;
+      case RTLSIM_OP_LEU: r = (a ^ 1u) | b; break;
+      case RTLSIM_OP_GTU: r = a & (b ^ 1u); break;
+      case RTLSIM_OP_GEU: r = a | (b ^ 1u); break;
+      case RTLSIM_OP_LTS: r = a & (b ^ 1u); break;     // 1-bit signed: 1 means -1
+      case RTLSIM_OP_LES: r = a | (b ^ 1u); break;
+      case RTLSIM_OP_GTS: r = (a ^ 1u) & b; break;
+      case RTLSIM_OP_GES: r = (a ^ 1u) | b; break;
+      case RTLSIM_OP_SHL: case RTLSIM_OP_SHRL: r = a & (b ^ 1u); break;   // shift by 1 >= width
+      case RTLSIM_OP_MUX: r = a ? b : c; break;
+      case RTLSIM_OP_CONCAT: r = b; break;             // ({a, b}) mod 2
+      default: r = 0; break;
+    }
+    lut |= (r & 1u) << k;
+  }
+  return lut;
 }
 
 }  // namespace rtlsim

@@ -24,44 +24,18 @@ namespace rtlsim {
 // ------------------------------------------------------------- helpers --
 __device__ __forceinline__ uint32_t nw_of(uint32_t w) { return (w + 31u) >> 5; }
 
-// Slot layouts in shared memory (per 32-stimulus tile, chosen by width):
-//   w == 1      one packed word, bit `lane` = stimulus lane
-//   w in 2..8   32 byte lanes (8 words)
-//   w in 9..16  32 half-word lanes (16 words)
-//   w > 16      one 32-word row per 32-bit word: word i of lane l at off+32i+l
-//   constants (off & kConstSlot): one broadcast copy of the words
-// Values are canonical (bits >= w are zero).
+// Slot layouts in shared memory (per 32-stimulus tile, program.h LC_*):
+//   LC_BIT   one packed word, bit `lane` = stimulus lane (written by ballot)
+//   LC_U8    32 byte lanes (8 words);  LC_U16  32 half-word lanes (16 words)
+//   LC_U32   one 32-word row per 32-bit word: word i of lane l at off+32i+l
+//   LC_IMM   constant <= 16 bits: `off` is the value itself
+//   LC_BCAST constant > 32 bits: one broadcast copy of its words
+// Values are canonical (bits >= width are zero).
 
-// word i of the value at slot `off` (width w), zero- or sign-extended to
-// infinite precision
-__device__ __forceinline__ uint32_t getw(const uint32_t *sm, uint32_t off, uint32_t w, uint32_t i,
-                                         bool sx, uint32_t lane) {
-  if (w == 1) {
-    const uint32_t b = (sm[off] >> lane) & 1u;
-    return sx ? (0u - b) : (i == 0 ? b : 0u);
-  }
-  const uint32_t n = nw_of(w), rem = w & 31u;
-  uint32_t x;
-  if (off & kConstSlot) {
-    x = sm[(off & ~kConstSlot) + (i < n ? i : n - 1)];
-  } else if (w <= 8) {
-    x = reinterpret_cast<const uint8_t *>(sm)[4u * off + lane];
-  } else if (w <= 16) {
-    x = reinterpret_cast<const uint16_t *>(sm)[2u * off + lane];
-  } else {
-    x = sm[off + 32u * (i < n ? i : n - 1) + lane];
-  }
-  if (i < n) {
-    if (sx && i == n - 1 && rem && ((x >> (rem - 1)) & 1u)) x |= ~((1u << rem) - 1u);
-    return x;
-  }
-  return sx ? 0u - ((x >> ((w - 1) & 31u)) & 1u) : 0u;   // x is the top word here
-}
-
-// store word i of a width-wd value (masking the top word); 1-bit values are
+// store word i of a width-wd result (masking the top word); a 1-bit result is
 // packed with a warp ballot and written by lane 0 (all lanes must call)
-__device__ __forceinline__ void putw(uint32_t *sm, uint32_t off, uint32_t wd, uint32_t i, uint32_t x,
-                                     uint32_t lane) {
+__device__ __forceinline__ void putw_l(uint32_t *sm, uint32_t off, uint32_t wd, uint32_t i, uint32_t x,
+                                       uint32_t lane) {
   if (wd == 1) {
     const uint32_t m = __ballot_sync(0xFFFFFFFFu, x & 1u);
     if (lane == 0) sm[off] = m;
@@ -74,14 +48,6 @@ __device__ __forceinline__ void putw(uint32_t *sm, uint32_t off, uint32_t wd, ui
   else sm[off + 32u * i + lane] = x;
 }
 
-// shift amount (self-determined, unsigned), saturated when >= 2^32
-__device__ __forceinline__ uint32_t shamt(const uint32_t *sm, uint32_t off, uint32_t w, uint32_t lane) {
-  uint32_t s = getw(sm, off, w, 0, false, lane);
-  for (uint32_t i = 1; i < nw_of(w); i++)
-    if (getw(sm, off, w, i, false, lane)) s = 0xFFFFFFFFu;
-  return s;
-}
-
 // 4-byte asynchronous global -> shared copy (LDGSTS); completion is awaited
 // once per step, just before the step barrier
 __device__ __forceinline__ void cp_async4(void *smem_dst, const void *gsrc) {
@@ -90,21 +56,21 @@ __device__ __forceinline__ void cp_async4(void *smem_dst, const void *gsrc) {
 }
 __device__ __forceinline__ void cp_async_wait_all() { asm volatile("cp.async.wait_all;" ::: "memory"); }
 
-// copy the tile's segment of a class row (or nd consecutive u32 rows) into
+// copy the tile's segment of a class row (or nw consecutive u32 rows) into
 // slot d, in the slot layout of its width class
-__device__ __forceinline__ void ld_class(uint32_t *sm, uint32_t d, uint32_t cls, uint32_t nd, const Arena &ar,
+__device__ __forceinline__ void ld_class(uint32_t *sm, uint32_t d, uint32_t cls, uint32_t nw, const Arena &ar,
                                          size_t row, uint32_t N, uint32_t tile, uint32_t lane) {
   uint8_t *smb = reinterpret_cast<uint8_t *>(sm);
-  if (cls == CLS_BIT) {
+  if (cls == CLS_U32) {
+    #pragma unroll 1
+    for (uint32_t i = 0; i < nw; i++) cp_async4(sm + d + 32u * i + lane, ar.u32 + (row + i) * N + tile * 32u + lane);
+  } else if (cls == CLS_BIT) {
     if (lane == 0) cp_async4(sm + d, ar.bit + row * (N >> 5) + tile);
   } else if (cls == CLS_U8) {
     if (lane < 8) cp_async4(smb + 4u * d + 4u * lane, ar.u8 + row * N + tile * 32u + 4u * lane);
-  } else if (cls == CLS_U16) {
-    if (lane < 16)
-      cp_async4(smb + 4u * d + 4u * lane,
-                reinterpret_cast<const uint8_t *>(ar.u16 + row * N + tile * 32u) + 4u * lane);
   } else {
-    for (uint32_t i = 0; i < nd; i++) cp_async4(sm + d + 32u * i + lane, ar.u32 + (row + i) * N + tile * 32u + lane);
+    if (lane < 16)
+      cp_async4(smb + 4u * d + 4u * lane, reinterpret_cast<const uint8_t *>(ar.u16 + row * N + tile * 32u) + 4u * lane);
   }
 }
 
@@ -117,68 +83,129 @@ __device__ __forceinline__ unsigned long long mix64(unsigned long long z) {
   return z;
 }
 
+// Narrow fast path (every width <= 32): one 32-bit word per operand.
+__device__ __forceinline__ uint32_t fetch1(const uint32_t *sm, uint32_t off, uint32_t lc, uint32_t lane) {
+  switch (lc) {
+    case LC_U32: return sm[off + lane];
+    case LC_BIT: return (sm[off] >> lane) & 1u;
+    case LC_U16: return reinterpret_cast<const uint16_t *>(sm)[2u * off + lane];
+    case LC_U8: return reinterpret_cast<const uint8_t *>(sm)[4u * off + lane];
+    default: return off;   // LC_IMM
+  }
+}
+
+__device__ __forceinline__ void store1(uint32_t *sm, uint32_t d, uint32_t lc, uint32_t r, uint32_t lane) {
+  switch (lc) {
+    case LC_U32: sm[d + lane] = r; break;
+    case LC_BIT: {
+      const uint32_t m = __ballot_sync(0xFFFFFFFFu, r & 1u);
+      if (lane == 0) sm[d] = m;
+      break;
+    }
+    case LC_U16: reinterpret_cast<uint16_t *>(sm)[2u * d + lane] = (uint16_t)r; break;
+    default: reinterpret_cast<uint8_t *>(sm)[4u * d + lane] = (uint8_t)r; break;
+  }
+}
+
 // --------------------------------------------------------------- N1 --
 // Generic path: any widths (1..1024), word loops over 32-bit words. Kept out
 // of line so the hot loop below stays small in the instruction cache.
-__device__ __noinline__ void exec_wide(uint32_t *sm, const uint4 q0, const uint4 q1, uint32_t lane) {
-  const uint32_t op = q0.x & 0xFFu;
-  const uint32_t wd = q0.y & 0xFFFFu, wa = q0.y >> 16;
-  const uint32_t wb = q0.z & 0xFFFFu, wc = q0.z >> 16;
-  const uint32_t d = q0.w, a = q1.x, b = q1.y, cc = q1.z, imm = q1.w;
+// word i of a wide-path operand: operands of <= 32 bits were fetched once
+// into v (any layout); wider ones are U32 rows or broadcast constants
+__device__ __forceinline__ uint32_t gw(const uint32_t *sm, uint32_t off, uint32_t w, uint32_t lay, uint32_t v,
+                                       uint32_t i, bool sx, uint32_t lane) {
+  const uint32_t n = nw_of(w), rem = w & 31u, top = n - 1u;
+  uint32_t x;
+  if (w <= 32u) {
+    x = v;
+  } else {
+    const uint32_t j = i < n ? i : top;
+    x = lay == LC_BCAST ? sm[off + j] : sm[off + 32u * j + lane];
+  }
+  if (i < n) {
+    if (sx && i == top && rem && ((x >> (rem - 1)) & 1u)) x |= ~((1u << rem) - 1u);
+    return x;
+  }
+  return sx ? 0u - ((x >> ((w - 1) & 31u)) & 1u) : 0u;   // x is the top word here
+}
+
+__device__ __noinline__ void exec_wide(uint32_t *sm, const WideRec *__restrict__ rec, uint32_t lane) {
+  const uint4 q0 = __ldg(reinterpret_cast<const uint4 *>(rec));       // op, wd|wa, wb|wc, imm
+  const uint4 q1 = __ldg(reinterpret_cast<const uint4 *>(rec) + 1);   // d a b c
+  const uint32_t lays = __ldg(reinterpret_cast<const uint32_t *>(rec) + 8);
+  const uint32_t op = q0.x, imm = q0.w;
+  const uint32_t wd = q0.y & 0xFFFFu, wa = q0.y >> 16, wb = q0.z & 0xFFFFu, wc = q0.z >> 16;
+  const uint32_t d = q1.x, a = q1.y, b = q1.z, cc = q1.w;
+  const uint32_t la = lays & 0xFFu, lb = (lays >> 8) & 0xFFu, lc = (lays >> 16) & 0xFFu;
+  const uint32_t va = wa && wa <= 32u ? fetch1(sm, a, la, lane) : 0u;
+  const uint32_t vb = wb && wb <= 32u ? fetch1(sm, b, lb, lane) : 0u;
+  const uint32_t vc = wc && wc <= 32u ? fetch1(sm, cc, lc, lane) : 0u;
   const uint32_t nd = nw_of(wd);
+#define GA(i, sx, ln) gw(sm, a, wa, la, va, (i), (sx), (ln))
+#define GB(i, sx, ln) gw(sm, b, wb, lb, vb, (i), (sx), (ln))
+#define GS(i, sx, ln) gw(sm, src, wsrc, lsrc, vsrc, (i), (sx), (ln))
+#define PUT(i, v, ln) putw_l(sm, d, wd, (i), (v), (ln))
   switch (op) {
           case RTLSIM_OP_COPY:
-            for (uint32_t i = 0; i < nd; i++) putw(sm, d, wd, i, getw(sm, a, wa, i, false, lane), lane);
+            #pragma unroll 1
+            for (uint32_t i = 0; i < nd; i++) PUT(i, GA(i, false, lane), lane);
             break;
           case RTLSIM_OP_SEXT:
-            for (uint32_t i = 0; i < nd; i++) putw(sm, d, wd, i, getw(sm, a, wa, i, true, lane), lane);
+            #pragma unroll 1
+            for (uint32_t i = 0; i < nd; i++) PUT(i, GA(i, true, lane), lane);
             break;
           case RTLSIM_OP_NOT:
-            for (uint32_t i = 0; i < nd; i++) putw(sm, d, wd, i, ~getw(sm, a, wa, i, false, lane), lane);
+            #pragma unroll 1
+            for (uint32_t i = 0; i < nd; i++) PUT(i, ~GA(i, false, lane), lane);
             break;
           case RTLSIM_OP_AND:
+            #pragma unroll 1
             for (uint32_t i = 0; i < nd; i++)
-              putw(sm, d, wd, i, getw(sm, a, wa, i, false, lane) & getw(sm, b, wb, i, false, lane), lane);
+              PUT(i, GA(i, false, lane) & GB(i, false, lane), lane);
             break;
           case RTLSIM_OP_OR:
+            #pragma unroll 1
             for (uint32_t i = 0; i < nd; i++)
-              putw(sm, d, wd, i, getw(sm, a, wa, i, false, lane) | getw(sm, b, wb, i, false, lane), lane);
+              PUT(i, GA(i, false, lane) | GB(i, false, lane), lane);
             break;
           case RTLSIM_OP_XOR:
+            #pragma unroll 1
             for (uint32_t i = 0; i < nd; i++)
-              putw(sm, d, wd, i, getw(sm, a, wa, i, false, lane) ^ getw(sm, b, wb, i, false, lane), lane);
+              PUT(i, GA(i, false, lane) ^ GB(i, false, lane), lane);
             break;
           case RTLSIM_OP_ADD:
           case RTLSIM_OP_SUB: {
             unsigned long long carry = (op == RTLSIM_OP_SUB) ? 1ull : 0ull;
+            #pragma unroll 1
             for (uint32_t i = 0; i < nd; i++) {
-              uint32_t x = getw(sm, a, wa, i, false, lane), y = getw(sm, b, wb, i, false, lane);
+              uint32_t x = GA(i, false, lane), y = GB(i, false, lane);
               if (op == RTLSIM_OP_SUB) y = ~y;
               unsigned long long t = (unsigned long long)x + y + carry;
               carry = t >> 32;
-              putw(sm, d, wd, i, (uint32_t)t, lane);
+              PUT(i, (uint32_t)t, lane);
             }
             break;
           }
           case RTLSIM_OP_NEG: {
             unsigned long long carry = 1ull;
+            #pragma unroll 1
             for (uint32_t i = 0; i < nd; i++) {
-              unsigned long long t = (unsigned long long)(uint32_t)~getw(sm, a, wa, i, false, lane) + carry;
+              unsigned long long t = (unsigned long long)(uint32_t)~GA(i, false, lane) + carry;
               carry = t >> 32;
-              putw(sm, d, wd, i, (uint32_t)t, lane);
+              PUT(i, (uint32_t)t, lane);
             }
             break;
           }
           case RTLSIM_OP_MUL:
           case RTLSIM_OP_DIVU:
           case RTLSIM_OP_MODU: {
-            unsigned long long x = getw(sm, a, wa, 0, false, lane) |
-                                   ((unsigned long long)getw(sm, a, wa, 1, false, lane) << 32);
-            unsigned long long y = getw(sm, b, wb, 0, false, lane) |
-                                   ((unsigned long long)getw(sm, b, wb, 1, false, lane) << 32);
+            unsigned long long x = GA(0, false, lane) |
+                                   ((unsigned long long)GA(1, false, lane) << 32);
+            unsigned long long y = GB(0, false, lane) |
+                                   ((unsigned long long)GB(1, false, lane) << 32);
             unsigned long long r = op == RTLSIM_OP_MUL ? x * y : (y == 0ull ? 0ull : (op == RTLSIM_OP_DIVU ? x / y : x % y));
-            putw(sm, d, wd, 0, (uint32_t)r, lane);
-            if (nd > 1) putw(sm, d, wd, 1, (uint32_t)(r >> 32), lane);
+            PUT(0, (uint32_t)r, lane);
+            if (nd > 1) PUT(1, (uint32_t)(r >> 32), lane);
             break;
           }
           case RTLSIM_OP_EQ: case RTLSIM_OP_NE: case RTLSIM_OP_LTU: case RTLSIM_OP_LEU:
@@ -187,8 +214,9 @@ __device__ __noinline__ void exec_wide(uint32_t *sm, const uint4 q0, const uint4
             const bool sg = op >= RTLSIM_OP_LTS;
             const uint32_t n = nw_of(wa > wb ? wa : wb);
             int cmp = 0;
+            #pragma unroll 1
             for (int i = (int)n - 1; i >= 0 && cmp == 0; i--) {
-              uint32_t x = getw(sm, a, wa, (uint32_t)i, sg, lane), y = getw(sm, b, wb, (uint32_t)i, sg, lane);
+              uint32_t x = GA((uint32_t)i, sg, lane), y = GB((uint32_t)i, sg, lane);
               if (x != y) {
                 if (sg && i == (int)n - 1) cmp = ((int32_t)x < (int32_t)y) ? -1 : 1;
                 else cmp = x < y ? -1 : 1;
@@ -203,19 +231,23 @@ __device__ __noinline__ void exec_wide(uint32_t *sm, const uint4 q0, const uint4
               case RTLSIM_OP_GTU: case RTLSIM_OP_GTS: t = cmp > 0; break;
               default: t = cmp >= 0; break;
             }
-            for (uint32_t i = 0; i < nd; i++) putw(sm, d, wd, i, i == 0 ? t : 0u, lane);
+            #pragma unroll 1
+            for (uint32_t i = 0; i < nd; i++) PUT(i, i == 0 ? t : 0u, lane);
             break;
           }
           case RTLSIM_OP_SHL: {
-            const uint32_t sa = shamt(sm, b, wb, lane);
+            uint32_t sa = GB(0, false, lane);
+            #pragma unroll 1
+            for (uint32_t i = 1; i < nw_of(wb); i++) if (GB(i, false, lane)) sa = 0xFFFFFFFFu;
             const uint32_t ws = sa >> 5, bs = sa & 31u;
+            #pragma unroll 1
             for (uint32_t i = 0; i < nd; i++) {
               uint32_t x = 0;
               if (sa < wd && i >= ws) {
-                x = getw(sm, a, wa, i - ws, false, lane) << bs;
-                if (bs && i > ws) x |= getw(sm, a, wa, i - ws - 1, false, lane) >> (32u - bs);
+                x = GA(i - ws, false, lane) << bs;
+                if (bs && i > ws) x |= GA(i - ws - 1, false, lane) >> (32u - bs);
               }
-              putw(sm, d, wd, i, x, lane);
+              PUT(i, x, lane);
             }
             break;
           }
@@ -223,41 +255,48 @@ __device__ __noinline__ void exec_wide(uint32_t *sm, const uint4 q0, const uint4
           case RTLSIM_OP_SHRA: {
             const bool sx = op == RTLSIM_OP_SHRA;
             const uint32_t W = wd > wa ? wd : wa;
-            uint32_t sa = shamt(sm, b, wb, lane);
+            uint32_t sa = GB(0, false, lane);
+            #pragma unroll 1
+            for (uint32_t i = 1; i < nw_of(wb); i++) if (GB(i, false, lane)) sa = 0xFFFFFFFFu;
             if (sa > W) sa = W;   // beyond the context width: 0 / sign fill
             const uint32_t ws = sa >> 5, bs = sa & 31u;
+            #pragma unroll 1
             for (uint32_t i = 0; i < nd; i++) {
-              uint32_t x = getw(sm, a, wa, i + ws, sx, lane) >> bs;
-              if (bs) x |= getw(sm, a, wa, i + ws + 1, sx, lane) << (32u - bs);
-              putw(sm, d, wd, i, x, lane);
+              uint32_t x = GA(i + ws, sx, lane) >> bs;
+              if (bs) x |= GA(i + ws + 1, sx, lane) << (32u - bs);
+              PUT(i, x, lane);
             }
             break;
           }
           case RTLSIM_OP_MUX: {
             uint32_t sel = 0;
-            for (uint32_t i = 0; i < nw_of(wa); i++) sel |= getw(sm, a, wa, i, false, lane);
-            const uint32_t src = sel ? b : cc, wsrc = sel ? wb : wc;
-            for (uint32_t i = 0; i < nd; i++) putw(sm, d, wd, i, getw(sm, src, wsrc, i, false, lane), lane);
+            #pragma unroll 1
+            for (uint32_t i = 0; i < nw_of(wa); i++) sel |= GA(i, false, lane);
+            const uint32_t src = sel ? b : cc, wsrc = sel ? wb : wc, lsrc = sel ? lb : lc, vsrc = sel ? vb : vc;
+            #pragma unroll 1
+            for (uint32_t i = 0; i < nd; i++) PUT(i, GS(i, false, lane), lane);
             break;
           }
           case RTLSIM_OP_CONCAT: {
             const uint32_t ws = wb >> 5, bs = wb & 31u;
+            #pragma unroll 1
             for (uint32_t i = 0; i < nd; i++) {
-              uint32_t x = getw(sm, b, wb, i, false, lane);
+              uint32_t x = GB(i, false, lane);
               if (i >= ws) {
-                x |= getw(sm, a, wa, i - ws, false, lane) << bs;
-                if (bs && i > ws) x |= getw(sm, a, wa, i - ws - 1, false, lane) >> (32u - bs);
+                x |= GA(i - ws, false, lane) << bs;
+                if (bs && i > ws) x |= GA(i - ws - 1, false, lane) >> (32u - bs);
               }
-              putw(sm, d, wd, i, x, lane);
+              PUT(i, x, lane);
             }
             break;
           }
           case RTLSIM_OP_SLICE: {
             const uint32_t ws = imm >> 5, bs = imm & 31u;
+            #pragma unroll 1
             for (uint32_t i = 0; i < nd; i++) {
-              uint32_t x = getw(sm, a, wa, i + ws, false, lane) >> bs;
-              if (bs) x |= getw(sm, a, wa, i + ws + 1, false, lane) << (32u - bs);
-              putw(sm, d, wd, i, x, lane);
+              uint32_t x = GA(i + ws, false, lane) >> bs;
+              if (bs) x |= GA(i + ws + 1, false, lane) << (32u - bs);
+              PUT(i, x, lane);
             }
             break;
           }
@@ -266,41 +305,24 @@ __device__ __noinline__ void exec_wide(uint32_t *sm, const uint4 q0, const uint4
           case RTLSIM_OP_REDXOR: {
             const uint32_t n = nw_of(wa), rem = wa & 31u;
             uint32_t t = op == RTLSIM_OP_REDAND ? 1u : 0u;
+            #pragma unroll 1
             for (uint32_t i = 0; i < n; i++) {
-              uint32_t x = getw(sm, a, wa, i, false, lane);
+              uint32_t x = GA(i, false, lane);
               if (op == RTLSIM_OP_REDAND) t &= (x == ((i == n - 1 && rem) ? ((1u << rem) - 1u) : 0xFFFFFFFFu));
               else if (op == RTLSIM_OP_REDOR) t |= (x != 0u);
               else t ^= (__popc(x) & 1u);
             }
-            for (uint32_t i = 0; i < nd; i++) putw(sm, d, wd, i, i == 0 ? t : 0u, lane);
+            #pragma unroll 1
+            for (uint32_t i = 0; i < nd; i++) PUT(i, i == 0 ? t : 0u, lane);
             break;
           }
           default:
             break;
   }
-}
-
-// Narrow fast path (every width <= 32): one 32-bit word per operand.
-__device__ __forceinline__ uint32_t fetch1(const uint32_t *sm, uint32_t off, uint32_t lc, uint32_t lane) {
-  const uint32_t o = off & 0xFFFFu;   // strips kConstSlot
-  if (lc == LC_U32) return sm[o + lane];
-  if (lc == LC_BIT) return (sm[o] >> lane) & 1u;
-  if (lc == LC_U8) return reinterpret_cast<const uint8_t *>(sm)[4u * o + lane];
-  if (lc == LC_U16) return reinterpret_cast<const uint16_t *>(sm)[2u * o + lane];
-  return sm[o];   // LC_CONST: broadcast
-}
-
-__device__ __forceinline__ void store1(uint32_t *sm, uint32_t d, uint32_t lc, uint32_t r, uint32_t lane) {
-  if (lc == LC_U32) {
-    sm[d + lane] = r;
-  } else if (lc == LC_BIT) {
-    const uint32_t m = __ballot_sync(0xFFFFFFFFu, r & 1u);
-    if (lane == 0) sm[d] = m;
-  } else if (lc == LC_U8) {
-    reinterpret_cast<uint8_t *>(sm)[4u * d + lane] = (uint8_t)r;
-  } else {
-    reinterpret_cast<uint16_t *>(sm)[2u * d + lane] = (uint16_t)r;
-  }
+#undef GA
+#undef GB
+#undef GS
+#undef PUT
 }
 
 __device__ __forceinline__ int32_t sx32(uint32_t x, uint32_t w) {
@@ -347,18 +369,41 @@ __device__ __forceinline__ uint32_t alu1(uint32_t op, uint32_t x, uint32_t y, ui
   }
 }
 
+// bit-sliced op: 3-input truth table applied to packed words (32 stimuli)
+__device__ __forceinline__ void exec_bit(uint32_t *sm, const uint4 q) {
+  const uint32_t lut = q.x & 0xFFu, immf = q.x >> 8;
+  const uint32_t fa = q.y >> 16, fb = q.z & 0xFFFFu, fc = q.z >> 16;
+  const uint32_t x = (immf & 1u) ? 0u - (fa & 1u) : sm[fa];
+  const uint32_t y = (immf & 2u) ? 0u - (fb & 1u) : sm[fb];
+  const uint32_t z = (immf & 4u) ? 0u - (fc & 1u) : sm[fc];
+  uint32_t r = 0;
+#pragma unroll
+  for (int k = 0; k < 8; k++) {
+    const uint32_t t = ((k & 1) ? x : ~x) & ((k & 2) ? y : ~y) & ((k & 4) ? z : ~z);
+    r |= t & (0u - ((lut >> k) & 1u));
+  }
+  sm[q.y & 0xFFFFu] = r;
+}
+
 // N1: op-stream evaluator.
-__global__ void __launch_bounds__(1024) rtl_eval_kernel(const EvalParams p) {
+__global__ void __launch_bounds__(512, 2) rtl_eval_kernel(const EvalParams p) {
   extern __shared__ uint32_t sm[];
   const uint32_t lane = threadIdx.x & 31u, wl = threadIdx.x >> 5;
   const uint32_t tile = blockIdx.x;
   const uint32_t s = tile * 32u + lane;
   const uint32_t N = p.N_pad, N32 = p.N_pad >> 5;
-  // per-warp descriptor staging buffer: 16 descriptors (512 B), refilled from
+  const uint32_t nthr = blockDim.x;
+  // per-warp descriptor staging buffer: 32 descriptors (512 B), refilled from
   // registers that were prefetched while the previous chunk executed
   uint4 *dbuf = reinterpret_cast<uint4 *>(sm + p.desc_smem_off) + wl * 32u;
   uint4 pf = make_uint4(0, 0, 0, 0);
   uint32_t pf_k = 0xFFFFFFFFu;
+  // bit-sliced ops: one per thread per step, prefetched one step ahead
+  uint4 pfb = make_uint4(0, 0, 0, 0);
+  {
+    const uint32_t b0 = __ldg(p.bit_ptr + p.step_begin), b1 = __ldg(p.bit_ptr + p.step_begin + 1);
+    if (b0 + threadIdx.x < b1) pfb = __ldg(p.bitdesc + b0 + threadIdx.x);
+  }
 
   for (uint32_t c = 0; c < p.n_cycles; c++) {
     const uint32_t par = (uint32_t)((p.cycle0 + c) & 1ull);
@@ -376,71 +421,94 @@ __global__ void __launch_bounds__(1024) rtl_eval_kernel(const EvalParams p) {
       const uint32_t ke = __ldg(p.step_ptr + step * p.L + wl + 1);
       const uint32_t nstep = step + 1 < p.step_end ? step + 1 : p.step_begin;
       const uint32_t nb = __ldg(p.step_ptr + nstep * p.L + wl);
-      for (uint32_t k0 = kb; k0 < ke; k0 += 16u) {
-        if (pf_k != k0) pf = __ldg(p.desc + 2u * k0 + lane);
+      // ---- bit-sliced ops of this step (lane = op)
+      {
+        const uint32_t bb = __ldg(p.bit_ptr + step), be = __ldg(p.bit_ptr + step + 1);
+        const uint32_t nbb = __ldg(p.bit_ptr + nstep), nbe = __ldg(p.bit_ptr + nstep + 1);
+        const uint4 qb = pfb;
+        if (nbb + threadIdx.x < nbe) pfb = __ldg(p.bitdesc + nbb + threadIdx.x);
+        if (bb + threadIdx.x < be) exec_bit(sm, qb);
+        for (uint32_t k = bb + threadIdx.x + nthr; k < be; k += nthr) exec_bit(sm, __ldg(p.bitdesc + k));
+      }
+      // ---- this warp's list of per-stimulus ops
+      for (uint32_t k0 = kb; k0 < ke; k0 += 32u) {
+        if (pf_k != k0) pf = __ldg(p.desc + k0 + lane);
         __syncwarp();
         dbuf[lane] = pf;
         __syncwarp();
-        pf_k = (k0 + 16u < ke) ? k0 + 16u : nb;
-        pf = __ldg(p.desc + 2u * pf_k + lane);   // the array is padded by 16 descriptors
-        const uint32_t nk = min(16u, ke - k0);
+        pf_k = (k0 + 32u < ke) ? k0 + 32u : nb;
+        pf = __ldg(p.desc + pf_k + lane);   // the array is padded by 32 descriptors
+        const uint32_t nk = min(32u, ke - k0);
         for (uint32_t j = 0; j < nk; j++) {
-          const uint4 q0 = dbuf[2u * j];
-          const uint4 q1 = dbuf[2u * j + 1u];
-          const uint32_t w0 = q0.x, op = w0 & 0xFFu;
-          if (op < 32u) {
-            if (w0 & DF_WIDE) {
-              exec_wide(sm, q0, q1, lane);
-            } else {
-              const uint32_t wd = q0.y & 0xFFFFu, wa = q0.y >> 16, wb = q0.z & 0xFFFFu;
-              const uint32_t x = fetch1(sm, q1.x, (w0 >> 8) & 7u, lane);
-              const uint32_t y = (w0 & DF_HAS_B) ? fetch1(sm, q1.y, (w0 >> 11) & 7u, lane) : 0u;
-              const uint32_t z = (w0 & DF_HAS_C) ? fetch1(sm, q1.z, (w0 >> 14) & 7u, lane) : 0u;
-              const uint32_t r = alu1(op, x, y, z, wd, wa, wb, q1.w) & (0xFFFFFFFFu >> (32u - wd));
-              store1(sm, q0.w, (w0 >> 17) & 7u, r, lane);
-            }
+          const uint4 q = dbuf[j];
+          const uint32_t code = q.x & 0xFFu;
+          if (code < 32u) {   // narrow compute op
+            const uint32_t x = fetch1(sm, q.y >> 16, (q.x >> 8) & 7u, lane);
+            const uint32_t y = (q.w & (1u << 11)) ? fetch1(sm, q.z & 0xFFFFu, (q.x >> 11) & 7u, lane) : 0u;
+            const uint32_t z = (q.w & (1u << 12)) ? fetch1(sm, q.z >> 16, (q.x >> 14) & 7u, lane) : 0u;
+            const uint32_t wd = (q.x >> 20) & 63u;
+            const uint32_t r = alu1(code, x, y, z, wd, q.x >> 26, q.w & 63u, (q.w >> 6) & 31u) &
+                               (0xFFFFFFFFu >> (32u - wd));
+            store1(sm, q.y & 0xFFFFu, (q.x >> 17) & 7u, r, lane);
             continue;
           }
-          const uint32_t wd = q0.y & 0xFFFFu, nd = nw_of(wd), cls = (w0 >> 17) & 7u;
-          const uint32_t d = q0.w, a = q1.x;
-          switch (op) {
-            case OP_LD_REG: ld_class(sm, d, cls, nd, cur, a, N, tile, lane); break;
-            case OP_LD_X: ld_class(sm, d, cls, nd, p.xnet, a, N, tile, lane); break;
-            case OP_LD_IN: ld_class(sm, d, cls, nd, inp, a, N, tile, lane); break;
-            case OP_LD_CONST:   // broadcast layout: one copy of the words per tile
-              if (lane == 0) {
-                if (wd == 1) sm[d] = (__ldg(p.consts + a) & 1u) ? 0xFFFFFFFFu : 0u;
-                else
-                  for (uint32_t i = 0; i < nd; i++) sm[d + i] = __ldg(p.consts + a + i);
+          if (code == CODE_WIDE) {
+            exec_wide(sm, p.wide + q.y, lane);
+            continue;
+          }
+          const uint32_t cls = (q.x >> 8) & 3u, nw = (q.x >> 12) & 63u;
+          switch (code) {
+            case CODE_LD_REG: ld_class(sm, q.y, cls, nw, cur, q.z, N, tile, lane); break;
+            case CODE_LD_X: ld_class(sm, q.y, cls, nw, p.xnet, q.z, N, tile, lane); break;
+            case CODE_LD_IN: ld_class(sm, q.y, cls, nw, inp, q.z, N, tile, lane); break;
+            case CODE_LD_CONST:
+              if ((q.x >> 18) & 1u) {   // broadcast copy
+                if (lane < nw) sm[q.y + lane] = __ldg(p.consts + q.z + lane);
+              } else {
+                #pragma unroll 1
+                for (uint32_t i = 0; i < nw; i++) sm[q.y + 32u * i + lane] = __ldg(p.consts + q.z + i);
               }
               break;
-            case OP_ST_REG:
-            case OP_ST_X: {
-              const Arena ar = op == OP_ST_REG ? nxt : p.xnet;
-              const bool dg = p.digest && op == OP_ST_REG;
-              const uint32_t aux = q1.w;
+            case CODE_ST_REG:
+            case CODE_ST_X: {
+              const Arena ar = code == CODE_ST_REG ? nxt : p.xnet;
+              const bool dg = p.digest && code == CODE_ST_REG;
+              const uint32_t row = q.z, aux = q.w, a = q.y;
               if (cls == CLS_BIT) {
-                const uint32_t word = sm[a];   // packed bits (1-bit constants are stored packed too)
-                if (lane == 0) ar.bit[(size_t)d * N32 + tile] = word;
+                const uint32_t word = sm[a];
+                if (lane == 0) ar.bit[(size_t)row * N32 + tile] = word;
                 if (dg) dig ^= mix64(((unsigned long long)(aux + 1u + 0x80000000u) << 32) | ((word >> lane) & 1u));
-              } else {
-                for (uint32_t i = 0; i < nd; i++) {
-                  const uint32_t v = getw(sm, a, wd, i, false, lane);
-                  if (cls == CLS_U8) ar.u8[(size_t)d * N + s] = (uint8_t)v;
-                  else if (cls == CLS_U16) ar.u16[(size_t)d * N + s] = (uint16_t)v;
-                  else ar.u32[(size_t)(d + i) * N + s] = v;
+              } else if (cls == CLS_U32) {
+                #pragma unroll 1
+                for (uint32_t i = 0; i < nw; i++) {
+                  const uint32_t v = sm[a + 32u * i + lane];
+                  ar.u32[(size_t)(row + i) * N + s] = v;
                   if (dg) dig ^= mix64(((unsigned long long)(aux + i + 1u + 0x80000000u) << 32) | v);
+                }
+              } else {
+                // 32 byte / half-word lanes: copy the packed words (8 or 16 lanes)
+                const uint32_t nlw = cls == CLS_U8 ? 8u : 16u;
+                uint8_t *dst = cls == CLS_U8 ? ar.u8 + (size_t)row * N + tile * 32u
+                                             : reinterpret_cast<uint8_t *>(ar.u16 + (size_t)row * N + tile * 32u);
+                if (lane < nlw) reinterpret_cast<uint32_t *>(dst)[lane] = sm[a + lane];
+                if (dg) {
+                  const uint32_t v = cls == CLS_U8 ? reinterpret_cast<const uint8_t *>(sm)[4u * a + lane]
+                                                   : reinterpret_cast<const uint16_t *>(sm)[2u * a + lane];
+                  dig ^= mix64(((unsigned long long)(aux + 1u + 0x80000000u) << 32) | v);
                 }
               }
               break;
             }
-            case OP_ST_OUT:
-              for (uint32_t i = 0; i < nd; i++) {
-                const uint32_t v = getw(sm, a, wd, i, false, lane);
-                out[(size_t)(d + i) * N + s] = v;
-                if (p.digest) dig ^= mix64(((unsigned long long)(d + i + 1u) << 32) | v);
+            case CODE_ST_OUT: {
+              const uint32_t lay = (q.x >> 18) & 7u, a = q.y;
+              #pragma unroll 1
+              for (uint32_t i = 0; i < nw; i++) {
+                const uint32_t v = lay == LC_U32 ? sm[a + 32u * i + lane] : fetch1(sm, a, lay, lane);
+                out[(size_t)(q.z + i) * N + s] = v;
+                if (p.digest) dig ^= mix64(((unsigned long long)(q.z + i + 1u) << 32) | v);
               }
               break;
+            }
             default:
               break;
           }

@@ -4,6 +4,8 @@
 
 #include <cstdint>
 
+#include "program.h"
+
 namespace rtlsim {
 
 // Arena pointers of one state buffer (or of the cross-partition net arena).
@@ -25,8 +27,13 @@ struct RegWord {
   uint32_t cls, row;
 };
 
+struct WideRec;
+
 struct EvalParams {
-  const uint4 *desc;          // 32-byte descriptors = 2 x uint4
+  const uint4 *desc;          // 16-byte descriptors (program.h Desc), padded by 32
+  const uint4 *bitdesc;       // bit-sliced ops (program.h BitDesc)
+  const uint32_t *bit_ptr;    // [n_steps + 1]
+  const WideRec *wide;        // generic-path records
   const uint32_t *step_ptr;   // [n_steps * L + 1]: lane l of step s = [p[sL+l], p[sL+l+1])
   uint32_t step_begin, step_end, L;
   uint32_t n_cycles;          // cycles processed by this launch

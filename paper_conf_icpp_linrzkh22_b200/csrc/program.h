@@ -13,7 +13,9 @@
 //     one 32-stimulus tile); a CTA barrier separates steps;
 //   * combinational values live in shared-memory slots assigned by liveness;
 //     registers, inputs, constants and cross-partition nets are loaded into
-//     slots by LD descriptors and stored by ST descriptors.
+//     slots by LD descriptors and stored by ST descriptors;
+//   * ops whose operands and result are all 1 bit run bit-sliced: one lane per
+//     op, 32 stimuli per packed word, as a 3-input truth table.
 #pragma once
 #include <cstdint>
 #include <string>
@@ -23,65 +25,86 @@
 
 namespace rtlsim {
 
-// internal opcodes beyond the IR's 0..30
-enum : uint16_t {
-  OP_LD_REG = 32,   // slot d <- state_cur[class][row a..] ; wd width
-  OP_LD_X = 33,     // slot d <- xnet[class][row a..]
-  OP_LD_IN = 34,    // slot d <- input class arena of cycle c [class imm][row a..]
-  OP_LD_CONST = 35, // slot d <- const_pool[a..] (broadcast)
-  OP_ST_REG = 40,   // state_next[class][row d..] <- slot a ; aux = register word index
-  OP_ST_X = 41,     // xnet[class][row d..] <- slot a
-  OP_ST_OUT = 42,   // out_chunk[c][word d..] <- slot a
+// state / xnet / input arena classes (lane bytes b(w): 1/8, 1, 2, 4 per word)
+enum : uint32_t { CLS_BIT = 0, CLS_U8 = 1, CLS_U16 = 2, CLS_U32 = 3 };
+
+// shared-memory slot layouts of a value (per 32-stimulus tile)
+enum : uint32_t {
+  LC_U32 = 0,    // one 32-word row per 32-bit word: word i of lane l at off + 32 i + l
+  LC_BIT = 1,    // one packed word: bit l = stimulus lane l
+  LC_U16 = 2,    // 32 half-word lanes (16 words)
+  LC_U8 = 3,     // 32 byte lanes (8 words)
+  LC_IMM = 4,    // constant <= 16 bits: the value itself is the operand field
+  LC_BCAST = 5,  // constant > 32 bits: one broadcast copy of its words
 };
 
-// state / xnet arena classes (lane bytes b(w): 1/8, 1, 2, 4 per word)
-enum : uint16_t { CLS_BIT = 0, CLS_U8 = 1, CLS_U16 = 2, CLS_U32 = 3 };
-
-// operand slot flag: constant values are stored once per tile (broadcast)
-constexpr uint32_t kConstSlot = 0x80000000u;
-// external values whose uses are more than this many steps apart are reloaded
-constexpr uint32_t kReloadGap = 3;
+// descriptor codes (x & 0xFF): 0..31 narrow compute op (the IR opcode)
+enum : uint32_t {
+  CODE_WIDE = 64,       // y = index of a WideRec
+  CODE_LD_REG = 80,     // slot y <- state_cur[cls][row z .. + nw)
+  CODE_LD_X = 81,       // slot y <- xnet[cls][row z ..]
+  CODE_LD_IN = 82,      // slot y <- input arena of cycle c [cls][row z ..]
+  CODE_LD_CONST = 83,   // slot y <- const pool[z .. + nw) (per-lane U32 or broadcast)
+  CODE_ST_REG = 96,     // state_next[cls][row z ..] <- slot y ; w = register word index
+  CODE_ST_X = 97,       // xnet[cls][row z ..] <- slot y
+  CODE_ST_OUT = 98,     // out_chunk[c][word z ..] <- slot y
+};
 
 inline uint32_t nwords(uint32_t w) { return (w + 31u) / 32u; }
-inline uint16_t width_class(uint32_t w) {
+inline uint32_t width_class(uint32_t w) {
   return w == 1 ? CLS_BIT : w <= 8 ? CLS_U8 : w <= 16 ? CLS_U16 : CLS_U32;
-}
-// shared-memory words one value occupies per 32-stimulus tile: packed bits,
-// byte lanes (2..8 bits), half-word lanes (9..16), word lanes (>16, one
-// 32-word row per 32-bit word); constants keep one broadcast copy
-inline uint32_t slot_words(uint32_t w, bool bcast) {
-  if (w == 1) return 1u;
-  if (bcast) return nwords(w);
-  if (w <= 8) return 8u;
-  if (w <= 16) return 16u;
-  return 32u * nwords(w);
 }
 inline double lane_bytes(uint32_t w) {
   return w == 1 ? 0.125 : w <= 8 ? 1.0 : w <= 16 ? 2.0 : 4.0 * nwords(w);
 }
-
-// slot layout codes (operand / destination addressing in shared memory)
-enum : uint32_t { LC_BIT = 0, LC_U8 = 1, LC_U16 = 2, LC_U32 = 3, LC_CONST = 4 };
-inline uint32_t layout_code(uint32_t w, bool bcast) {
-  return bcast ? LC_CONST : w == 1 ? LC_BIT : w <= 8 ? LC_U8 : w <= 16 ? LC_U16 : LC_U32;
+// layout of a signal's value in shared memory
+inline uint32_t value_layout(uint32_t w, bool is_const) {
+  if (is_const) return w <= 16 ? LC_IMM : (w <= 32 ? LC_U32 : LC_BCAST);
+  return w == 1 ? LC_BIT : w <= 8 ? LC_U8 : w <= 16 ? LC_U16 : LC_U32;
 }
-// descriptor flags (word 0)
-constexpr uint32_t DF_WIDE = 1u << 20;   // some width > 32: generic word-loop path
-constexpr uint32_t DF_HAS_B = 1u << 21;
-constexpr uint32_t DF_HAS_C = 1u << 22;
+inline uint32_t slot_words(uint32_t layout, uint32_t w) {
+  switch (layout) {
+    case LC_BIT: return 1u;
+    case LC_U8: return 8u;
+    case LC_U16: return 16u;
+    case LC_IMM: return 0u;
+    case LC_BCAST: return nwords(w);
+    default: return 32u * nwords(w);
+  }
+}
 
-// 32-byte descriptor, read by the kernel as two uint4:
-//   w0 = op | la << 8 | lb << 11 | lc << 14 | ld << 17 | flags   (compute ops)
-//   w0 = op | class << 17                                          (LD / ST)
-//   wd, wa, wb, wc widths; d, a, b, c slot offsets (or arena rows for LD/ST);
-//   aux = SLICE lo, or the register word index of ST_REG (digest)
+// 16-byte descriptor (one uint4), see kernels.cu for the decoding:
+//   narrow compute (code = IR opcode < 32, every width <= 32):
+//     x = op | la << 8 | lb << 11 | lc << 14 | ld << 17 | wd << 20 | wa << 26
+//     y = d | a << 16 ; z = b | c << 16 ; w = wb | imm << 6
+//   CODE_WIDE: y = WideRec index
+//   LD:  x = code | cls << 8 | nw << 12 | bcast << 18 ; y = slot ; z = row
+//   ST:  x = code | cls << 8 | nw << 12 | src layout << 18 ; y = slot ; z = row ; w = aux
 struct Desc {
-  uint32_t w0;
-  uint16_t wd, wa, wb, wc;
-  uint32_t d, a, b, c;
-  uint32_t aux;
+  uint32_t x, y, z, w;
 };
-static_assert(sizeof(Desc) == 32, "descriptor must be 32 bytes");
+static_assert(sizeof(Desc) == 16, "descriptor must be 16 bytes");
+
+// bit-sliced op (every operand and the result 1 bit): one lane evaluates a
+// 3-input truth table on packed words.  x = lut | imm_a << 8 | imm_b << 9 |
+// imm_c << 10 ; y = d | a << 16 ; z = b | c << 16 (an immediate operand field
+// holds the constant 0 / 1)
+struct BitDesc {
+  uint32_t x, y, z, w;
+};
+static_assert(sizeof(BitDesc) == 16, "bit descriptor must be 16 bytes");
+
+// generic (any width) op record for the out-of-line wide path; three uint4:
+// {op, wd | wa << 16, wb | wc << 16, imm} {d, a, b, c} {la | lb << 8 | lc << 16, -, -, -}
+struct WideRec {
+  uint32_t op;
+  uint16_t wd, wa, wb, wc;
+  uint32_t imm;           // SLICE lo
+  uint32_t d, a, b, c;    // slot offsets (or immediate values for LC_IMM)
+  uint32_t lays;
+  uint32_t pad[3];
+};
+static_assert(sizeof(WideRec) == 48, "wide record layout");
 
 struct RegInfo {
   uint32_t sig, width, cls, row, word;   // row in its class arena; word = first RW index
@@ -106,17 +129,24 @@ struct Program {
   // ---- schedule
   uint32_t L = 1;                       // op-lanes (warps) per tile
   uint32_t n_steps = 0;
-  std::vector<Desc> desc;
+  std::vector<Desc> desc;               // lane lists, step-major
   std::vector<uint32_t> step_ptr;       // [n_steps * L + 1]: lane l of step s = [p[s*L+l], p[s*L+l+1])
+  std::vector<BitDesc> bitdesc;         // bit-sliced ops, step-major
+  std::vector<uint32_t> bit_ptr;        // [n_steps + 1]
+  std::vector<WideRec> wide;            // records referenced by CODE_WIDE
   std::vector<uint32_t> part_steps;     // exec-order partition boundaries in steps (size P+1)
-  uint32_t smem_words = 0;              // shared words per tile
+  uint32_t smem_words = 0;              // shared words per tile (slots)
   // ---- stats
-  uint64_t word_ops = 0;
+  uint64_t word_ops = 0, n_bitops = 0, n_wide = 0, n_narrow = 0, n_ld = 0, n_st = 0;
   double b_floor = 0, b_state = 0, b_part = 0;
 };
 
 // Returns RTLSIM_OK or a negative status with *err set.
-int compile_program(const rtlsim_ir *ir, uint32_t op_lanes, uint32_t smem_limit_words,
-                    Program *out, std::string *err);
+int compile_program(const rtlsim_ir *ir, uint32_t op_lanes, uint32_t smem_limit_words, Program *out,
+                    std::string *err);
+
+// 3-input truth table (bit k = f(a = k&1, b = k>>1&1, c = k>>2&1)) of an IR
+// opcode on 1-bit operands and a 1-bit result.
+uint32_t bit_lut(uint32_t opcode);
 
 }  // namespace rtlsim

@@ -66,7 +66,9 @@ struct rtlsim_ctx {
   std::vector<void *> bind_allocs;    // freed at re-bind
   std::vector<void *> host_allocs;    // pinned, freed at re-bind
   // static device data
-  uint4 *d_desc = nullptr;
+  uint4 *d_desc = nullptr, *d_bitdesc = nullptr;
+  uint32_t *d_bitptr = nullptr;
+  WideRec *d_wide = nullptr;
   uint32_t *d_step = nullptr, *d_consts = nullptr, *d_mask = nullptr, *d_reginit = nullptr;
   RegWord *d_regmap = nullptr;
   // binding
@@ -216,8 +218,11 @@ extern "C" int rtlsim_load(const rtlsim_ir *ir, const rtlsim_options *opt, rtlsi
   cudaError_t e = cudaSuccess;
   // the evaluator prefetches descriptor chunks of 16 past the end: pad
   std::vector<Desc> padded(G.desc);
-  padded.resize(G.desc.size() + 16, Desc{});
+  padded.resize(G.desc.size() + 32, Desc{});   // chunk prefetch reads up to 32 past any start
   if (e == cudaSuccess) e = up((void **)&ctx->d_desc, padded.data(), padded.size() * sizeof(Desc));
+  if (e == cudaSuccess) e = up((void **)&ctx->d_bitdesc, G.bitdesc.data(), G.bitdesc.size() * sizeof(BitDesc));
+  if (e == cudaSuccess) e = up((void **)&ctx->d_bitptr, G.bit_ptr.data(), G.bit_ptr.size() * 4);
+  if (e == cudaSuccess) e = up((void **)&ctx->d_wide, G.wide.data(), G.wide.size() * sizeof(WideRec));
   if (e == cudaSuccess) e = up((void **)&ctx->d_inmap, G.in_map.data(), G.in_map.size() * 4);
   if (e == cudaSuccess) e = up((void **)&ctx->d_step, G.step_ptr.data(), G.step_ptr.size() * 4);
   if (e == cudaSuccess) e = up((void **)&ctx->d_consts, G.const_pool.data(), G.const_pool.size() * 4);
@@ -369,6 +374,9 @@ static EvalParams eval_params(rtlsim_ctx *ctx, int b, uint64_t cycle0, uint32_t 
   Program &G = ctx->prog;
   EvalParams p{};
   p.desc = ctx->d_desc;
+  p.bitdesc = ctx->d_bitdesc;
+  p.bit_ptr = ctx->d_bitptr;
+  p.wide = ctx->d_wide;
   p.step_ptr = ctx->d_step;
   p.step_begin = 0;
   p.step_end = G.n_steps;
