@@ -53,9 +53,10 @@ static void setbit(big_t *x, unsigned i, int v) {
     x->w[i / 32] &= ~(1u << (i % 32));
 }
 
-/* zero every bit at position >= bits */
-static void mask_to(big_t *x, unsigned bits) {
-  for (unsigned i = 0; i < BIGW; i++) {
+/* zero every bit at position >= bits among the first `words` words (the
+ * words above are already zero) */
+static void mask_range(big_t *x, unsigned bits, unsigned words) {
+  for (unsigned i = 0; i < words && i < BIGW; i++) {
     unsigned lo = 32 * i;
     if (lo >= bits)
       x->w[i] = 0;
@@ -64,15 +65,20 @@ static void mask_to(big_t *x, unsigned bits) {
   }
 }
 
+/* zero every bit at position >= bits */
+static void mask_to(big_t *x, unsigned bits) { mask_range(x, bits, BIGW); }
+
 /* x := src (w_src bits) extended to `bits` bits (zero- or sign-extension),
- * or truncated when bits < w_src. */
+ * or truncated when bits < w_src. Only the first max(nw(w_src), nw(bits))
+ * words can be non-zero, so only those are masked. */
 static void ext(big_t *x, const uint32_t *src, unsigned w_src, unsigned bits, int sign) {
   memset(x, 0, sizeof *x);
-  for (unsigned i = 0; i < nw(w_src); i++) x->w[i] = src[i];
-  mask_to(x, w_src);
+  const unsigned n = nw(w_src), nb = nw(bits) > n ? nw(bits) : n;
+  for (unsigned i = 0; i < n; i++) x->w[i] = src[i];
+  mask_range(x, w_src, n);
   if (sign && bits > w_src && getbit(x, w_src - 1))
     for (unsigned i = w_src; i < bits; i++) setbit(x, i, 1);
-  mask_to(x, bits);
+  mask_range(x, bits, nb);
 }
 
 static int is_zero(const big_t *x) {

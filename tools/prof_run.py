@@ -8,7 +8,8 @@ from paper_conf_icpp_linrzkh22_b200 import rtlsim as R
 cid = int(sys.argv[1]); Tc = int(sys.argv[2]); nl = int(sys.argv[3]) if len(sys.argv) > 3 else 2
 NS = {1: 1024, 2: 4096, 3: 16384, 4: 65536}
 ir = designs.tiny_dut() if cid == 1 else shaped.generate(cid)
-N = NS[cid]
+import os
+N = int(os.environ.get('PROF_N', NS[cid]))
 s = torch.cuda.Stream(); torch.cuda.set_stream(s)
 sim = R.Simulator(ir, chunk_cycles=Tc, stream=s.cuda_stream)
 d_stim = stim.stimulus_torch(ir, stim.STIM_SEED_BASE + cid, 0, N, 0, Tc * nl)
