@@ -29,6 +29,12 @@ namespace rtlsim {
 
 // external values whose uses are more than this many steps apart are reloaded
 constexpr int32_t kReloadGap = 3;
+// loads are issued this many steps before their first use (cp.async groups,
+// awaited with a per-step wait depth just before the step barrier)
+static int32_t load_ahead() {
+  static const int32_t d = getenv("RTLSIM_LOAD_AHEAD") ? atoi(getenv("RTLSIM_LOAD_AHEAD")) : 2;
+  return std::max(1, std::min(d, 4));
+}
 
 static int arity(uint32_t opc) {
   switch (opc) {
@@ -54,6 +60,7 @@ struct Value {
   uint32_t width;
   int32_t def_step;    // step that writes the slot (-1: immediate)
   int32_t last_use;    // last step that reads it (-1: dead)
+  int32_t first_use;   // first step that reads it (loads: completion deadline)
   uint32_t slot;       // smem word offset (the value itself for LC_IMM)
   uint32_t layout;     // LC_*
   uint32_t words() const { return slot_words(layout, width); }
@@ -347,6 +354,7 @@ int compile_program(const rtlsim_ir *ir, uint32_t op_lanes, uint32_t smem_limit_
   struct StepLists {
     std::vector<std::pair<Desc, uint32_t>> lane;   // descriptor, cost
     std::vector<BitDesc> bits;
+    uint32_t wait = 0;                             // cp.async groups allowed pending at the step end
   };
   std::vector<StepLists> all_steps;   // global step list
   uint32_t peak = dump_words;
@@ -360,7 +368,7 @@ int compile_program(const rtlsim_ir *ir, uint32_t op_lanes, uint32_t smem_limit_
     std::vector<uint32_t> touched;
     auto vid = [&](uint32_t s) -> int32_t { return vid_of[s]; };
     auto new_val = [&](uint32_t s, uint32_t w, int32_t def_step, uint32_t layout) -> int32_t {
-      vals.push_back(Value{s, w, def_step, -1, 0, layout});
+      vals.push_back(Value{s, w, def_step, -1, 1 << 30, 0, layout});
       return (int32_t)vals.size() - 1;
     };
     // 1. levels of the partition's own ops (ASAP)
@@ -499,9 +507,10 @@ int compile_program(const rtlsim_ir *ir, uint32_t op_lanes, uint32_t smem_limit_
           else gs.back().last = st;
         }
         for (size_t g = 0; g < gs.size(); g++) {
-          gs[g].val = new_val(s, G.width[s], gs[g].first - 1, value_layout(G.width[s], G.kind[s] == RTLSIM_CONST));
+          const int32_t issue = std::max(0, gs[g].first - load_ahead());
+          gs[g].val = new_val(s, G.width[s], issue, value_layout(G.width[s], G.kind[s] == RTLSIM_CONST));
           vals[gs[g].val].last_use = gs[g].last;
-          loads.push_back(Load{s, gs[g].val, gs[g].first - 1, g == 0});
+          loads.push_back(Load{s, gs[g].val, issue, g == 0});
         }
         groups[s] = std::move(gs);
       }
@@ -527,6 +536,7 @@ int compile_program(const rtlsim_ir *ir, uint32_t op_lanes, uint32_t smem_limit_
       if (sy.step < 0) sy.step = std::max(vals[src].def_step, 0) + 1;
       sy.val = new_val(sy.src_sig, sy.w, sy.step, value_layout(sy.w, false));
       vals[src].last_use = std::max(vals[src].last_use, sy.step);
+      vals[src].first_use = std::min(vals[src].first_use, sy.step);
     }
     // 3. uses by ops
     std::vector<std::array<int32_t, 3>> op_vals(ops_p.size());
@@ -538,6 +548,7 @@ int compile_program(const rtlsim_ir *ir, uint32_t op_lanes, uint32_t smem_limit_
         int32_t v = val_at(src[k], op_step[i]);
         op_vals[j][k] = v;
         vals[v].last_use = std::max(vals[v].last_use, op_step[i]);
+        vals[v].first_use = std::min(vals[v].first_use, op_step[i]);
       }
     }
     // 4. sink steps: one after the stored value is written
@@ -548,6 +559,7 @@ int compile_program(const rtlsim_ir *ir, uint32_t op_lanes, uint32_t smem_limit_
       sk.src_val = v;
       sink_step[k] = std::max(vals[v].def_step, 0) + 1;
       vals[v].last_use = std::max(vals[v].last_use, sink_step[k]);
+      vals[v].first_use = std::min(vals[v].first_use, sink_step[k]);
     }
     // 5. number of steps
     int32_t nsteps = 0;
@@ -701,8 +713,22 @@ int compile_program(const rtlsim_ir *ir, uint32_t op_lanes, uint32_t smem_limit_
       G.n_st++;
       steps[sink_step[k]].lane.push_back({d, 1 + nwords(w)});
     }
-    for (auto &st : steps)
-      if (!st.lane.empty() || !st.bits.empty()) all_steps.push_back(std::move(st));
+    // wait depth: at the end of step e at most w_e of the most recent
+    // per-step cp.async groups may be pending; a load issued at step i and
+    // first read at step f needs w_{f-1} <= f-1-i. Drain at the last step.
+    {
+      const uint32_t deflt = (uint32_t)load_ahead() - 1u;
+      for (auto &st : steps) st.wait = deflt;
+      for (const Load &ld : loads) {
+        const int32_t f = vals[ld.val].first_use;
+        if (f <= 0 || f >= (1 << 30)) continue;
+        const int32_t e = f - 1;
+        steps[e].wait = std::min<uint32_t>(steps[e].wait, (uint32_t)std::max(0, e - ld.step));
+      }
+      if (!steps.empty()) steps.back().wait = 0;
+    }
+    // empty steps are kept (their barrier / wait depth is part of the schedule)
+    for (auto &st : steps) all_steps.push_back(std::move(st));
     G.part_steps.push_back((uint32_t)all_steps.size());
     for (uint32_t s : touched) vid_of[s] = -1;
     for (auto &kv : groups) vid_of[kv.first] = -1;
@@ -753,6 +779,8 @@ int compile_program(const rtlsim_ir *ir, uint32_t op_lanes, uint32_t smem_limit_
   }
   G.step_ptr.push_back((uint32_t)G.desc.size());
   G.bit_ptr.push_back((uint32_t)G.bitdesc.size());
+  G.step_wait.reserve(all_steps.size());
+  for (auto &st : all_steps) G.step_wait.push_back(st.wait);
   G.smem_words = std::max<uint32_t>(peak, 1);
   if (smem_limit_words && G.smem_words > smem_limit_words)
     return fail(err, RTLSIM_E_NOMEM,

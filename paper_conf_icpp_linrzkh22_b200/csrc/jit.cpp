@@ -1,0 +1,913 @@
+// jit.cpp — PTX generation for specialized partition kernels, in-process
+// compilation with nvPTXCompiler, loading with the CUDA runtime library API.
+//
+// Semantics are exactly those of the interpreter (kernels.cu / DESIGN.md §3):
+// the generator walks the same compiled schedule (steps, per-warp op lists,
+// shared-memory slots and layouts) and emits, per op, the straight-line PTX
+// the interpreter would have executed after decoding — offsets, widths,
+// layouts and immediates become constants. Wide shifts by a variable amount
+// call the interpreter's generic path (rtl_exec_wide, from jit_rt.ptx).
+#include "jit.h"
+
+#include <nvPTXCompiler.h>
+
+#include <algorithm>
+#include <atomic>
+#include <chrono>
+#include <cstdarg>
+#include <cstdio>
+#include <cstdlib>
+#include <cstring>
+#include <fstream>
+#include <mutex>
+#include <sstream>
+#include <thread>
+
+namespace rtlsim {
+namespace {
+
+std::string fmt(const char *f, ...) {
+  char buf[512];
+  va_list ap;
+  va_start(ap, f);
+  int n = vsnprintf(buf, sizeof buf, f, ap);
+  va_end(ap);
+  if (n < (int)sizeof buf) return std::string(buf, (size_t)std::max(n, 0));
+  std::string s((size_t)n + 1, '\0');
+  va_start(ap, f);
+  vsnprintf(&s[0], s.size(), f, ap);
+  va_end(ap);
+  s.resize((size_t)n);
+  return s;
+}
+
+// context values passed from the kernel to every step function
+const char *kCtx32[] = {"smb", "lane", "wl", "N"};
+const char *kCtx64[] = {"tb_c0", "tb_c1", "tb_c2", "tb_c3", "tb_n0", "tb_n1", "tb_n2", "tb_n3",
+                        "tb_x0", "tb_x1", "tb_x2", "tb_x3", "tb_i0", "tb_i1", "tb_i2", "tb_i3",
+                        "outb", "dig", "wide", "smg"};
+constexpr int kN32 = 4, kN64 = 20;
+
+struct Em {
+  std::string s;
+  uint32_t nr = 0, nrd = 0, np = 0, nlab = 0;
+  std::string R() { return fmt("%%r%u", nr++); }
+  std::string RD() { return fmt("%%rd%u", nrd++); }
+  std::string P() { return fmt("%%p%u", np++); }
+  std::string L(const char *pfx) { return fmt("$%s%u", pfx, nlab++); }
+  void l(const std::string &x) {
+    s += '\t';
+    s += x;
+    s += ";\n";
+  }
+  void lab(const std::string &x) {
+    s += x;
+    s += ":\n";
+  }
+};
+
+inline uint32_t mask_of(uint32_t w) { return w >= 32 ? 0xFFFFFFFFu : ((1u << w) - 1u); }
+
+// ------------------------------------------------------------- operands --
+// narrow (<= 32-bit) value from a slot of layout `lay` (or an immediate)
+std::string fetch_narrow(Em &e, uint32_t lay, uint32_t off, uint32_t /*w*/) {
+  std::string r = e.R();
+  switch (lay) {
+    case LC_U32: e.l(fmt("ld.shared.u32 %s, [%%rw+%u]", r.c_str(), off * 4)); break;
+    case LC_U16: e.l(fmt("ld.shared.u16 %s, [%%rh+%u]", r.c_str(), off * 4)); break;
+    case LC_U8: e.l(fmt("ld.shared.u8 %s, [%%rb+%u]", r.c_str(), off * 4)); break;
+    case LC_BIT: {
+      std::string t = e.R(), t2 = e.R();
+      e.l(fmt("ld.shared.u32 %s, [%%smb+%u]", t.c_str(), off * 4));
+      e.l(fmt("shr.b32 %s, %s, %%lane", t2.c_str(), t.c_str()));
+      e.l(fmt("and.b32 %s, %s, 1", r.c_str(), t2.c_str()));
+      break;
+    }
+    case LC_BCAST: e.l(fmt("ld.shared.u32 %s, [%%smb+%u]", r.c_str(), off * 4)); break;
+    default: e.l(fmt("mov.u32 %s, %u", r.c_str(), off)); break;   // LC_IMM
+  }
+  return r;
+}
+
+void store_narrow(Em &e, uint32_t lay, uint32_t off, const std::string &r) {
+  switch (lay) {
+    case LC_U32: e.l(fmt("st.shared.u32 [%%rw+%u], %s", off * 4, r.c_str())); break;
+    case LC_U16: e.l(fmt("st.shared.u16 [%%rh+%u], %s", off * 4, r.c_str())); break;
+    case LC_U8: e.l(fmt("st.shared.u8 [%%rb+%u], %s", off * 4, r.c_str())); break;
+    default: {   // LC_BIT: pack the warp's 32 results
+      std::string p = e.P(), m = e.R();
+      e.l(fmt("setp.ne.u32 %s, %s, 0", p.c_str(), r.c_str()));
+      e.l(fmt("vote.sync.ballot.b32 %s, %s, 0xffffffff", m.c_str(), p.c_str()));
+      // every lane holds the same ballot word: an unpredicated store is one
+      // same-address wavefront (and compiles much faster than a predicated one)
+      e.l(fmt("st.shared.u32 [%%smb+%u], %s", off * 4, m.c_str()));
+      break;
+    }
+  }
+}
+
+// sign-extend a canonical w-bit value held in r (w < 32) to 32 bits
+std::string sext32(Em &e, const std::string &r, uint32_t w) {
+  if (w >= 32) return r;
+  std::string t = e.R(), u = e.R();
+  e.l(fmt("shl.b32 %s, %s, %u", t.c_str(), r.c_str(), 32 - w));
+  e.l(fmt("shr.s32 %s, %s, %u", u.c_str(), t.c_str(), 32 - w));
+  return u;
+}
+
+// a wide-op operand: word i of the value zero- or sign-extended
+struct WOp {
+  uint32_t off = 0, w = 0, lay = LC_U32;
+  std::vector<std::string> zw, sw;   // cached zero / sign views per word
+  std::string top_sx;                // sign-extended top word
+  std::string fill;                  // 0 / all ones from the sign
+  std::string narrow;                // fetched value when w <= 32
+};
+
+std::string wword(Em &e, WOp &o, uint32_t i, bool sx) {
+  const uint32_t n = nwords(o.w), rem = o.w & 31u;
+  if (o.zw.size() < n) {
+    o.zw.assign(n, "");
+    o.sw.assign(n, "");
+  }
+  auto raw = [&](uint32_t j) -> std::string {
+    if (!o.zw[j].empty()) return o.zw[j];
+    std::string r;
+    if (o.w <= 32) {
+      if (o.narrow.empty()) o.narrow = fetch_narrow(e, o.lay, o.off, o.w);
+      r = o.narrow;
+    } else {
+      r = e.R();
+      if (o.lay == LC_BCAST) e.l(fmt("ld.shared.u32 %s, [%%smb+%u]", r.c_str(), (o.off + j) * 4));
+      else e.l(fmt("ld.shared.u32 %s, [%%rw+%u]", r.c_str(), (o.off + 32 * j) * 4));
+    }
+    o.zw[j] = r;
+    return r;
+  };
+  if (i < n) {
+    if (!sx || i != n - 1 || rem == 0) return raw(i);
+    if (o.top_sx.empty()) o.top_sx = sext32(e, raw(n - 1), rem);
+    return o.top_sx;
+  }
+  if (!sx) return "0";
+  if (o.fill.empty()) {
+    std::string top = (rem == 0) ? raw(n - 1) : (o.top_sx.empty() ? (o.top_sx = sext32(e, raw(n - 1), rem)) : o.top_sx);
+    o.fill = e.R();
+    e.l(fmt("shr.s32 %s, %s, 31", o.fill.c_str(), top.c_str()));
+  }
+  return o.fill;
+}
+
+// store word i of a wide result (masking the top word)
+void wstore(Em &e, uint32_t off, uint32_t wd, uint32_t i, const std::string &v) {
+  const uint32_t n = nwords(wd), rem = wd & 31u;
+  std::string x = v;
+  if (v == "0") {
+    x = e.R();
+    e.l(fmt("mov.u32 %s, 0", x.c_str()));
+  }
+  if (wd <= 32) {   // a narrow result of a wide op
+    std::string m = x;
+    if (wd < 32) {
+      m = e.R();
+      e.l(fmt("and.b32 %s, %s, %u", m.c_str(), x.c_str(), mask_of(wd)));
+    }
+    store_narrow(e, value_layout(wd, false), off, m);
+    return;
+  }
+  if (i == n - 1 && rem) {
+    std::string m = e.R();
+    e.l(fmt("and.b32 %s, %s, %u", m.c_str(), x.c_str(), mask_of(rem)));
+    x = m;
+  }
+  e.l(fmt("st.shared.u32 [%%rw+%u], %s", (off + 32 * i) * 4, x.c_str()));
+}
+
+std::string reg_of(Em &e, const std::string &v) {
+  if (v == "0") {
+    std::string r = e.R();
+    e.l(fmt("mov.u32 %s, 0", r.c_str()));
+    return r;
+  }
+  return v;
+}
+
+// -------------------------------------------------------- narrow ops --
+void emit_narrow(Em &e, const Desc &q) {
+  const uint32_t op = q.x & 0xFFu;
+  const uint32_t la = (q.x >> 8) & 7u, lb = (q.x >> 11) & 7u, lc = (q.x >> 14) & 7u, ld = (q.x >> 17) & 7u;
+  const uint32_t wd = (q.x >> 20) & 63u, wa = q.x >> 26, wb = q.w & 63u, imm = (q.w >> 6) & 31u;
+  const bool hb = (q.w >> 11) & 1u, hc = (q.w >> 12) & 1u;
+  const uint32_t d = q.y & 0xFFFFu, a = q.y >> 16, b = q.z & 0xFFFFu, c = q.z >> 16;
+  std::string x = fetch_narrow(e, la, a, wa);
+  std::string y = hb ? fetch_narrow(e, lb, b, wb) : std::string();
+  std::string z = hc ? fetch_narrow(e, lc, c, 32) : std::string();
+  std::string r = e.R();
+  bool canon = false;   // result already < 2^wd
+  // predicate-free forms (set.* gives 0 / all ones): ptxas compiles them far
+  // faster than setp/selp chains and the SASS is the same length
+  auto cmp = [&](const char *cc, const std::string &u, const std::string &v) {
+    std::string m = e.R();
+    const char *ty = strstr(cc, ".s32") ? "s32" : "u32";
+    std::string c2(cc);
+    c2 = c2.substr(0, c2.find('.'));
+    e.l(fmt("set.%s.u32.%s %s, %s, %s", c2.c_str(), ty, m.c_str(), u.c_str(), v.c_str()));
+    e.l(fmt("and.b32 %s, %s, 1", r.c_str(), m.c_str()));
+    canon = true;
+  };
+  switch (op) {
+    case RTLSIM_OP_COPY: e.l(fmt("mov.u32 %s, %s", r.c_str(), x.c_str())); break;
+    case RTLSIM_OP_SEXT: e.l(fmt("mov.u32 %s, %s", r.c_str(), sext32(e, x, wa).c_str())); break;
+    case RTLSIM_OP_NOT: e.l(fmt("not.b32 %s, %s", r.c_str(), x.c_str())); break;
+    case RTLSIM_OP_AND: e.l(fmt("and.b32 %s, %s, %s", r.c_str(), x.c_str(), y.c_str())); break;
+    case RTLSIM_OP_OR: e.l(fmt("or.b32 %s, %s, %s", r.c_str(), x.c_str(), y.c_str())); break;
+    case RTLSIM_OP_XOR: e.l(fmt("xor.b32 %s, %s, %s", r.c_str(), x.c_str(), y.c_str())); break;
+    case RTLSIM_OP_ADD: e.l(fmt("add.u32 %s, %s, %s", r.c_str(), x.c_str(), y.c_str())); break;
+    case RTLSIM_OP_SUB: e.l(fmt("sub.u32 %s, %s, %s", r.c_str(), x.c_str(), y.c_str())); break;
+    case RTLSIM_OP_NEG: e.l(fmt("neg.s32 %s, %s", r.c_str(), x.c_str())); break;
+    case RTLSIM_OP_MUL: e.l(fmt("mul.lo.u32 %s, %s, %s", r.c_str(), x.c_str(), y.c_str())); break;
+    case RTLSIM_OP_DIVU:
+    case RTLSIM_OP_MODU: {   // b == 0 gives 0
+      std::string m = e.R(), t = e.R();
+      e.l(fmt("set.ne.u32.u32 %s, %s, 0", m.c_str(), y.c_str()));
+      e.l(fmt("%s.u32 %s, %s, %s", op == RTLSIM_OP_DIVU ? "div" : "rem", t.c_str(), x.c_str(), y.c_str()));
+      e.l(fmt("and.b32 %s, %s, %s", r.c_str(), t.c_str(), m.c_str()));
+      break;
+    }
+    case RTLSIM_OP_EQ: cmp("eq.u32", x, y); break;
+    case RTLSIM_OP_NE: cmp("ne.u32", x, y); break;
+    case RTLSIM_OP_LTU: cmp("lt.u32", x, y); break;
+    case RTLSIM_OP_LEU: cmp("le.u32", x, y); break;
+    case RTLSIM_OP_GTU: cmp("gt.u32", x, y); break;
+    case RTLSIM_OP_GEU: cmp("ge.u32", x, y); break;
+    case RTLSIM_OP_LTS: cmp("lt.s32", sext32(e, x, wa), sext32(e, y, wb)); break;
+    case RTLSIM_OP_LES: cmp("le.s32", sext32(e, x, wa), sext32(e, y, wb)); break;
+    case RTLSIM_OP_GTS: cmp("gt.s32", sext32(e, x, wa), sext32(e, y, wb)); break;
+    case RTLSIM_OP_GES: cmp("ge.s32", sext32(e, x, wa), sext32(e, y, wb)); break;
+    case RTLSIM_OP_SHL: {   // b >= wd gives 0
+      std::string m = e.R(), t = e.R();
+      e.l(fmt("set.lt.u32.u32 %s, %s, %u", m.c_str(), y.c_str(), wd));
+      e.l(fmt("shl.b32 %s, %s, %s", t.c_str(), x.c_str(), y.c_str()));
+      e.l(fmt("and.b32 %s, %s, %s", r.c_str(), t.c_str(), m.c_str()));
+      break;
+    }
+    case RTLSIM_OP_SHRL: e.l(fmt("shr.u32 %s, %s, %s", r.c_str(), x.c_str(), y.c_str())); break;   // clamps at 32
+    case RTLSIM_OP_SHRA: e.l(fmt("shr.s32 %s, %s, %s", r.c_str(), sext32(e, x, wa).c_str(), y.c_str())); break;
+    case RTLSIM_OP_MUX: {   // m = all ones when sel != 0; r = (y & m) | (z & ~m)
+      std::string m = e.R();
+      e.l(fmt("set.ne.u32.u32 %s, %s, 0", m.c_str(), x.c_str()));
+      e.l(fmt("lop3.b32 %s, %s, %s, %s, 0xca", r.c_str(), m.c_str(), y.c_str(), z.c_str()));
+      break;
+    }
+    case RTLSIM_OP_CONCAT:
+      if (wb >= 32) {
+        e.l(fmt("mov.u32 %s, %s", r.c_str(), y.c_str()));
+      } else {
+        std::string t = e.R();
+        e.l(fmt("shl.b32 %s, %s, %u", t.c_str(), x.c_str(), wb));
+        e.l(fmt("or.b32 %s, %s, %s", r.c_str(), t.c_str(), y.c_str()));
+      }
+      break;
+    case RTLSIM_OP_SLICE: e.l(fmt("shr.u32 %s, %s, %u", r.c_str(), x.c_str(), imm)); break;
+    case RTLSIM_OP_REDAND: cmp("eq.u32", x, fmt("%u", mask_of(wa))); break;
+    case RTLSIM_OP_REDOR: cmp("ne.u32", x, "0"); break;
+    default: {   // REDXOR
+      std::string t = e.R();
+      e.l(fmt("popc.b32 %s, %s", t.c_str(), x.c_str()));
+      e.l(fmt("and.b32 %s, %s, 1", r.c_str(), t.c_str()));
+      canon = true;
+      break;
+    }
+  }
+  std::string res = r;
+  if (!canon && wd < 32) {
+    res = e.R();
+    e.l(fmt("and.b32 %s, %s, %u", res.c_str(), r.c_str(), mask_of(wd)));
+  }
+  store_narrow(e, ld, d, res);
+}
+
+// ---------------------------------------------------------- wide ops --
+void emit_generic_call(Em &e, uint32_t idx) {
+  std::string rec = e.RD();
+  e.l(fmt("add.u64 %s, %%wide, %u", rec.c_str(), idx * (uint32_t)sizeof(WideRec)));
+  e.s += "\t{\n\t.param .b64 wp0;\n\t.param .b64 wp1;\n\t.param .b32 wp2;\n";
+  e.l("st.param.b64 [wp0], %smg");
+  e.l(fmt("st.param.b64 [wp1], %s", rec.c_str()));
+  e.l("st.param.b32 [wp2], %lane");
+  e.l("call.uni rtl_exec_wide, (wp0, wp1, wp2)");
+  e.s += "\t}\n";
+}
+
+void emit_wide(Em &e, const WideRec &w, uint32_t idx) {
+  const uint32_t op = w.op, wd = w.wd, nd = nwords(wd);
+  WOp A, B, C;
+  A.off = w.a; A.w = w.wa; A.lay = w.lays & 0xFFu;
+  B.off = w.b; B.w = w.wb; B.lay = (w.lays >> 8) & 0xFFu;
+  C.off = w.c; C.w = w.wc; C.lay = (w.lays >> 16) & 0xFFu;
+  auto bin = [&](const char *ins) {
+    for (uint32_t i = 0; i < nd; i++) {
+      std::string xa = reg_of(e, wword(e, A, i, false)), xb = reg_of(e, wword(e, B, i, false)), r = e.R();
+      e.l(fmt("%s %s, %s, %s", ins, r.c_str(), xa.c_str(), xb.c_str()));
+      wstore(e, w.d, wd, i, r);
+    }
+  };
+  switch (op) {
+    case RTLSIM_OP_COPY:
+    case RTLSIM_OP_SEXT:
+      for (uint32_t i = 0; i < nd; i++) wstore(e, w.d, wd, i, wword(e, A, i, op == RTLSIM_OP_SEXT));
+      return;
+    case RTLSIM_OP_NOT:
+      for (uint32_t i = 0; i < nd; i++) {
+        std::string xa = reg_of(e, wword(e, A, i, false)), r = e.R();
+        e.l(fmt("not.b32 %s, %s", r.c_str(), xa.c_str()));
+        wstore(e, w.d, wd, i, r);
+      }
+      return;
+    case RTLSIM_OP_AND: bin("and.b32"); return;
+    case RTLSIM_OP_OR: bin("or.b32"); return;
+    case RTLSIM_OP_XOR: bin("xor.b32"); return;
+    case RTLSIM_OP_ADD:
+    case RTLSIM_OP_SUB:
+    case RTLSIM_OP_NEG: {
+      std::vector<std::string> xs(nd), ys(nd), rs(nd);
+      for (uint32_t i = 0; i < nd; i++) {
+        if (op == RTLSIM_OP_NEG) {
+          xs[i] = "0";
+          ys[i] = reg_of(e, wword(e, A, i, false));
+        } else {
+          xs[i] = reg_of(e, wword(e, A, i, false));
+          ys[i] = reg_of(e, wword(e, B, i, false));
+        }
+        rs[i] = e.R();
+      }
+      const char *base = op == RTLSIM_OP_ADD ? "add" : "sub";
+      for (uint32_t i = 0; i < nd; i++) {
+        const char *cc = nd == 1 ? "" : (i == 0 ? ".cc" : (i + 1 < nd ? ".cc" : ""));
+        const char *car = (i == 0) ? "" : "c";
+        e.l(fmt("%s%s%s.u32 %s, %s, %s", base, car, cc, rs[i].c_str(), xs[i].c_str(), ys[i].c_str()));
+      }
+      for (uint32_t i = 0; i < nd; i++) wstore(e, w.d, wd, i, rs[i]);
+      return;
+    }
+    case RTLSIM_OP_MUL:
+    case RTLSIM_OP_DIVU:
+    case RTLSIM_OP_MODU: {
+      std::string a64 = e.RD(), b64 = e.RD(), r64 = e.RD();
+      std::string a0 = reg_of(e, wword(e, A, 0, false)), a1 = reg_of(e, wword(e, A, 1, false));
+      std::string b0 = reg_of(e, wword(e, B, 0, false)), b1 = reg_of(e, wword(e, B, 1, false));
+      e.l(fmt("mov.b64 %s, {%s, %s}", a64.c_str(), a0.c_str(), a1.c_str()));
+      e.l(fmt("mov.b64 %s, {%s, %s}", b64.c_str(), b0.c_str(), b1.c_str()));
+      if (op == RTLSIM_OP_MUL) {
+        e.l(fmt("mul.lo.u64 %s, %s, %s", r64.c_str(), a64.c_str(), b64.c_str()));
+      } else {   // b == 0 gives 0
+        std::string m = e.R(), m64 = e.RD(), t = e.RD();
+        e.l(fmt("set.ne.u32.u64 %s, %s, 0", m.c_str(), b64.c_str()));
+        e.l(fmt("mov.b64 %s, {%s, %s}", m64.c_str(), m.c_str(), m.c_str()));
+        e.l(fmt("%s.u64 %s, %s, %s", op == RTLSIM_OP_DIVU ? "div" : "rem", t.c_str(), a64.c_str(), b64.c_str()));
+        e.l(fmt("and.b64 %s, %s, %s", r64.c_str(), t.c_str(), m64.c_str()));
+      }
+      std::string lo = e.R(), hi = e.R();
+      e.l(fmt("mov.b64 {%s, %s}, %s", lo.c_str(), hi.c_str(), r64.c_str()));
+      wstore(e, w.d, wd, 0, lo);
+      if (nd > 1) wstore(e, w.d, wd, 1, hi);
+      return;
+    }
+    case RTLSIM_OP_EQ: case RTLSIM_OP_NE: case RTLSIM_OP_LTU: case RTLSIM_OP_LEU: case RTLSIM_OP_GTU:
+    case RTLSIM_OP_GEU: case RTLSIM_OP_LTS: case RTLSIM_OP_LES: case RTLSIM_OP_GTS: case RTLSIM_OP_GES: {
+      const bool sg = op >= RTLSIM_OP_LTS;
+      const uint32_t n = nwords(std::max<uint32_t>(w.wa, w.wb));
+      // lexicographic compare from the least significant word up, as masks:
+      // LT_i = lt_i | (eq_i & LT_{i-1}), EQ_i = eq_i & EQ_{i-1}
+      std::string LT, EQ;
+      for (uint32_t i = 0; i < n; i++) {
+        std::string xa = reg_of(e, wword(e, A, i, sg)), xb = reg_of(e, wword(e, B, i, sg));
+        std::string lt = e.R(), eq = e.R();
+        const bool top_signed = sg && i == n - 1;
+        e.l(fmt("set.lt.u32.%s %s, %s, %s", top_signed ? "s32" : "u32", lt.c_str(), xa.c_str(), xb.c_str()));
+        e.l(fmt("set.eq.u32.u32 %s, %s, %s", eq.c_str(), xa.c_str(), xb.c_str()));
+        if (i == 0) {
+          LT = lt;
+          EQ = eq;
+        } else {
+          std::string LT2 = e.R(), EQ2 = e.R();
+          e.l(fmt("lop3.b32 %s, %s, %s, %s, 0xf8", LT2.c_str(), lt.c_str(), eq.c_str(), LT.c_str()));
+          e.l(fmt("and.b32 %s, %s, %s", EQ2.c_str(), eq.c_str(), EQ.c_str()));
+          LT = LT2;
+          EQ = EQ2;
+        }
+      }
+      std::string res = e.R();
+      switch (op) {
+        case RTLSIM_OP_EQ: e.l(fmt("mov.u32 %s, %s", res.c_str(), EQ.c_str())); break;
+        case RTLSIM_OP_NE: e.l(fmt("not.b32 %s, %s", res.c_str(), EQ.c_str())); break;
+        case RTLSIM_OP_LTU: case RTLSIM_OP_LTS: e.l(fmt("mov.u32 %s, %s", res.c_str(), LT.c_str())); break;
+        case RTLSIM_OP_LEU: case RTLSIM_OP_LES: e.l(fmt("or.b32 %s, %s, %s", res.c_str(), LT.c_str(), EQ.c_str())); break;
+        case RTLSIM_OP_GTU: case RTLSIM_OP_GTS: e.l(fmt("lop3.b32 %s, %s, %s, 0, 0x03", res.c_str(), LT.c_str(), EQ.c_str())); break;
+        default: e.l(fmt("not.b32 %s, %s", res.c_str(), LT.c_str())); break;
+      }
+      std::string r = e.R();
+      e.l(fmt("and.b32 %s, %s, 1", r.c_str(), res.c_str()));
+      for (uint32_t i = 0; i < nd; i++) wstore(e, w.d, wd, i, i == 0 ? r : std::string("0"));
+      return;
+    }
+    case RTLSIM_OP_MUX: {
+      std::string acc;
+      for (uint32_t i = 0; i < nwords(w.wa); i++) {
+        std::string xa = reg_of(e, wword(e, A, i, false));
+        if (acc.empty()) {
+          acc = xa;
+        } else {
+          std::string t = e.R();
+          e.l(fmt("or.b32 %s, %s, %s", t.c_str(), acc.c_str(), xa.c_str()));
+          acc = t;
+        }
+      }
+      std::string m = e.R();
+      e.l(fmt("set.ne.u32.u32 %s, %s, 0", m.c_str(), acc.c_str()));
+      for (uint32_t i = 0; i < nd; i++) {
+        std::string tb = reg_of(e, wword(e, B, i, false)), tc = reg_of(e, wword(e, C, i, false)), r = e.R();
+        e.l(fmt("lop3.b32 %s, %s, %s, %s, 0xca", r.c_str(), m.c_str(), tb.c_str(), tc.c_str()));
+        wstore(e, w.d, wd, i, r);
+      }
+      return;
+    }
+    case RTLSIM_OP_CONCAT: {   // (a << wb) | b
+      const uint32_t ws = w.wb >> 5, bs = w.wb & 31u;
+      for (uint32_t i = 0; i < nd; i++) {
+        std::string v = reg_of(e, wword(e, B, i, false));
+        if (i >= ws) {
+          std::string lo = reg_of(e, wword(e, A, i - ws, false)), t = e.R();
+          if (bs == 0) {
+            e.l(fmt("or.b32 %s, %s, %s", t.c_str(), v.c_str(), lo.c_str()));
+          } else {
+            std::string hi_part = e.R();
+            e.l(fmt("shl.b32 %s, %s, %u", hi_part.c_str(), lo.c_str(), bs));
+            std::string t2 = e.R();
+            e.l(fmt("or.b32 %s, %s, %s", t2.c_str(), v.c_str(), hi_part.c_str()));
+            if (i > ws) {
+              std::string prev = reg_of(e, wword(e, A, i - ws - 1, false)), sh = e.R();
+              e.l(fmt("shr.u32 %s, %s, %u", sh.c_str(), prev.c_str(), 32 - bs));
+              e.l(fmt("or.b32 %s, %s, %s", t.c_str(), t2.c_str(), sh.c_str()));
+            } else {
+              e.l(fmt("mov.u32 %s, %s", t.c_str(), t2.c_str()));
+            }
+          }
+          v = t;
+        }
+        wstore(e, w.d, wd, i, v);
+      }
+      return;
+    }
+    case RTLSIM_OP_SLICE: {
+      const uint32_t ws = w.imm >> 5, bs = w.imm & 31u;
+      for (uint32_t i = 0; i < nd; i++) {
+        std::string lo = reg_of(e, wword(e, A, i + ws, false));
+        if (bs == 0) {
+          wstore(e, w.d, wd, i, lo);
+        } else {
+          std::string hi = reg_of(e, wword(e, A, i + ws + 1, false)), r = e.R();
+          e.l(fmt("shf.r.clamp.b32 %s, %s, %s, %u", r.c_str(), lo.c_str(), hi.c_str(), bs));
+          wstore(e, w.d, wd, i, r);
+        }
+      }
+      return;
+    }
+    case RTLSIM_OP_REDAND:
+    case RTLSIM_OP_REDOR:
+    case RTLSIM_OP_REDXOR: {
+      const uint32_t n = nwords(w.wa), rem = w.wa & 31u;
+      std::string acc;
+      for (uint32_t i = 0; i < n; i++) {
+        std::string xa = reg_of(e, wword(e, A, i, false)), t = e.R();
+        if (op == RTLSIM_OP_REDAND) {   // compare against the all-ones word of this position
+          std::string m = e.R();
+          e.l(fmt("set.eq.u32.u32 %s, %s, %u", m.c_str(), xa.c_str(), (i == n - 1 && rem) ? mask_of(rem) : 0xFFFFFFFFu));
+          e.l(fmt("and.b32 %s, %s, 1", t.c_str(), m.c_str()));
+          if (!acc.empty()) {
+            std::string u = e.R();
+            e.l(fmt("and.b32 %s, %s, %s", u.c_str(), acc.c_str(), t.c_str()));
+            t = u;
+          }
+        } else if (op == RTLSIM_OP_REDOR) {
+          if (acc.empty()) {
+            e.l(fmt("mov.u32 %s, %s", t.c_str(), xa.c_str()));
+          } else {
+            e.l(fmt("or.b32 %s, %s, %s", t.c_str(), acc.c_str(), xa.c_str()));
+          }
+        } else {
+          e.l(fmt("popc.b32 %s, %s", t.c_str(), xa.c_str()));
+          if (!acc.empty()) {
+            std::string u = e.R();
+            e.l(fmt("add.u32 %s, %s, %s", u.c_str(), acc.c_str(), t.c_str()));
+            t = u;
+          }
+        }
+        acc = t;
+      }
+      std::string r = e.R();
+      if (op == RTLSIM_OP_REDAND) {
+        e.l(fmt("mov.u32 %s, %s", r.c_str(), acc.c_str()));
+      } else if (op == RTLSIM_OP_REDOR) {
+        std::string m = e.R();
+        e.l(fmt("set.ne.u32.u32 %s, %s, 0", m.c_str(), acc.c_str()));
+        e.l(fmt("and.b32 %s, %s, 1", r.c_str(), m.c_str()));
+      } else {
+        e.l(fmt("and.b32 %s, %s, 1", r.c_str(), acc.c_str()));
+      }
+      for (uint32_t i = 0; i < nd; i++) wstore(e, w.d, wd, i, i == 0 ? r : std::string("0"));
+      return;
+    }
+    default:   // SHL / SHRL / SHRA by a variable amount: generic path
+      emit_generic_call(e, idx);
+      return;
+  }
+}
+
+// ----------------------------------------------------------- loads / stores --
+const char *kArenaTag[4] = {"c", "n", "x", "i"};   // cur, nxt, xnet, in
+
+void emit_ld(Em &e, uint32_t arena, uint32_t cls, uint32_t row, uint32_t slot, uint32_t nw) {
+  const char *A = kArenaTag[arena];
+  std::string addr = e.RD();
+  switch (cls) {
+    case CLS_U32:
+      for (uint32_t i = 0; i < nw; i++) {
+        std::string ai = i == 0 ? addr : e.RD();
+        e.l(fmt("mad.wide.u32 %s, %%N4, %u, %%tb_%s3", ai.c_str(), row + i, A));
+        e.l(fmt("cp.async.ca.shared.global [%%rw+%u], [%s], 4", (slot + 32 * i) * 4, ai.c_str()));
+      }
+      break;
+    case CLS_U16:
+      e.l(fmt("mad.wide.u32 %s, %%N2, %u, %%tb_%s2", addr.c_str(), row, A));
+      e.l(fmt("@%%pl16 cp.async.ca.shared.global [%%rw+%u], [%s], 4", slot * 4, addr.c_str()));
+      break;
+    case CLS_U8:
+      e.l(fmt("mad.wide.u32 %s, %%N, %u, %%tb_%s1", addr.c_str(), row, A));
+      e.l(fmt("@%%pl8 cp.async.ca.shared.global [%%rw+%u], [%s], 4", slot * 4, addr.c_str()));
+      break;
+    default:
+      e.l(fmt("mad.wide.u32 %s, %%Nb, %u, %%tb_%s0", addr.c_str(), row, A));
+      e.l(fmt("@%%pl0 cp.async.ca.shared.global [%%smb+%u], [%s], 4", slot * 4, addr.c_str()));
+      break;
+  }
+}
+
+void emit_dig(Em &e, uint32_t key, const std::string &v) {
+  std::string skip = e.L("nd");
+  e.l(fmt("@!%%pdig bra.uni %s", skip.c_str()));
+  e.s += "\t{\n\t.param .b64 dp0;\n\t.param .b32 dp1;\n\t.param .b32 dp2;\n";
+  e.l("st.param.b64 [dp0], %dig");
+  e.l(fmt("st.param.b32 [dp1], %u", key));
+  e.l(fmt("st.param.b32 [dp2], %s", v.c_str()));
+  e.l("call.uni rtl_dig, (dp0, dp1, dp2)");
+  e.s += "\t}\n";
+  e.lab(skip);
+}
+
+void emit_st(Em &e, uint32_t code, uint32_t cls, uint32_t nw, uint32_t lay, uint32_t slot, uint32_t row,
+             uint32_t aux) {
+  const bool dg = code == CODE_ST_REG;
+  if (code == CODE_ST_OUT) {
+    for (uint32_t i = 0; i < nw; i++) {
+      std::string v;
+      if (lay == LC_U32) {
+        v = e.R();
+        e.l(fmt("ld.shared.u32 %s, [%%rw+%u]", v.c_str(), (slot + 32 * i) * 4));
+      } else {
+        v = fetch_narrow(e, lay, slot, 32);
+      }
+      std::string addr = e.RD();
+      e.l(fmt("mad.wide.u32 %s, %%N4, %u, %%outb", addr.c_str(), row + i));
+      e.l(fmt("st.global.u32 [%s], %s", addr.c_str(), v.c_str()));
+      emit_dig(e, row + i + 1, v);
+    }
+    return;
+  }
+  const char *A = code == CODE_ST_REG ? "n" : "x";
+  std::string addr = e.RD();
+  switch (cls) {
+    case CLS_U32:
+      for (uint32_t i = 0; i < nw; i++) {
+        std::string v = e.R(), ai = e.RD();
+        e.l(fmt("ld.shared.u32 %s, [%%rw+%u]", v.c_str(), (slot + 32 * i) * 4));
+        e.l(fmt("mad.wide.u32 %s, %%N4, %u, %%tb_%s3", ai.c_str(), row + i, A));
+        e.l(fmt("st.global.u32 [%s], %s", ai.c_str(), v.c_str()));
+        if (dg) emit_dig(e, aux + i + 1u + 0x80000000u, v);
+      }
+      return;
+    case CLS_U16:
+    case CLS_U8: {
+      // 32 byte / half-word lanes: 8 or 16 lanes copy the packed words
+      std::string t = e.R();
+      const char *pl = cls == CLS_U8 ? "%pl8" : "%pl16";
+      e.l(fmt("@%s ld.shared.u32 %s, [%%rw+%u]", pl, t.c_str(), slot * 4));
+      if (cls == CLS_U8) e.l(fmt("mad.wide.u32 %s, %%N, %u, %%tb_%s1", addr.c_str(), row, A));
+      else e.l(fmt("mad.wide.u32 %s, %%N2, %u, %%tb_%s2", addr.c_str(), row, A));
+      e.l(fmt("@%s st.global.u32 [%s], %s", pl, addr.c_str(), t.c_str()));
+      if (dg) emit_dig(e, aux + 1u + 0x80000000u, fetch_narrow(e, lay, slot, 16));
+      return;
+    }
+    default: {
+      std::string t = e.R();
+      e.l(fmt("ld.shared.u32 %s, [%%smb+%u]", t.c_str(), slot * 4));
+      e.l(fmt("mad.wide.u32 %s, %%Nb, %u, %%tb_%s0", addr.c_str(), row, A));
+      e.l(fmt("@%%pl0 st.global.u32 [%s], %s", addr.c_str(), t.c_str()));
+      if (dg) {
+        std::string b = e.R(), b2 = e.R();
+        e.l(fmt("shr.b32 %s, %s, %%lane", b.c_str(), t.c_str()));
+        e.l(fmt("and.b32 %s, %s, 1", b2.c_str(), b.c_str()));
+        emit_dig(e, aux + 1u + 0x80000000u, b2);
+      }
+      return;
+    }
+  }
+}
+
+void emit_ld_const(Em &e, const Program &G, uint32_t slot, uint32_t pool, uint32_t nw, bool bcast) {
+  for (uint32_t i = 0; i < nw; i++) {
+    std::string v = e.R();
+    e.l(fmt("mov.u32 %s, %u", v.c_str(), G.const_pool[pool + i]));
+    if (bcast) e.l(fmt("st.shared.u32 [%%smb+%u], %s", (slot + i) * 4, v.c_str()));
+    else e.l(fmt("st.shared.u32 [%%rw+%u], %s", (slot + 32 * i) * 4, v.c_str()));
+  }
+}
+
+// convert program.h truth-table order (bit k = f(a=k&1, b=k>>1&1, c=k>>2)) to
+// PTX lop3 order (bit j = f(a=j>>2&1, b=j>>1&1, c=j&1))
+uint32_t lop3_lut(uint32_t lut) {
+  uint32_t r = 0;
+  for (uint32_t j = 0; j < 8; j++) {
+    const uint32_t a = (j >> 2) & 1u, b = (j >> 1) & 1u, c = j & 1u;
+    r |= ((lut >> (a | (b << 1) | (c << 2))) & 1u) << j;
+  }
+  return r;
+}
+
+void emit_bit(Em &e, const BitDesc &q) {
+  const uint32_t lut = q.x & 0xFFu, immf = q.x >> 8;
+  const uint32_t f[3] = {q.y >> 16, q.z & 0xFFFFu, q.z >> 16};
+  std::string v[3];
+  for (int k = 0; k < 3; k++) {
+    v[k] = e.R();
+    if (immf & (1u << k)) e.l(fmt("mov.u32 %s, %u", v[k].c_str(), (f[k] & 1u) ? 0xFFFFFFFFu : 0u));
+    else e.l(fmt("ld.shared.u32 %s, [%%smb+%u]", v[k].c_str(), f[k] * 4));
+  }
+  std::string r = e.R();
+  e.l(fmt("lop3.b32 %s, %s, %s, %s, 0x%02x", r.c_str(), v[0].c_str(), v[1].c_str(), v[2].c_str(), lop3_lut(lut)));
+  e.l(fmt("st.shared.u32 [%%smb+%u], %s", (q.y & 0xFFFFu) * 4, r.c_str()));
+}
+
+void emit_desc(Em &e, const Program &G, const Desc &q) {
+  const uint32_t code = q.x & 0xFFu;
+  if (code < 32u) {
+    emit_narrow(e, q);
+    return;
+  }
+  if (code == CODE_WIDE) {
+    emit_wide(e, G.wide[q.y], q.y);
+    return;
+  }
+  const uint32_t cls = (q.x >> 8) & 3u, nw = (q.x >> 12) & 63u;
+  switch (code) {
+    case CODE_LD_REG: emit_ld(e, 0, cls, q.z, q.y, nw); break;
+    case CODE_LD_X: emit_ld(e, 2, cls, q.z, q.y, nw); break;
+    case CODE_LD_IN: emit_ld(e, 3, cls, q.z, q.y, nw); break;
+    case CODE_LD_CONST: emit_ld_const(e, G, q.y, q.z, nw, ((q.x >> 18) & 1u) != 0); break;
+    case CODE_ST_REG: case CODE_ST_X: case CODE_ST_OUT:
+      emit_st(e, code, cls, nw, (q.x >> 18) & 7u, q.y, q.z, q.w);
+      break;
+    default: break;
+  }
+}
+
+std::string func_proto(const std::string &name) {
+  std::string s = ".func " + name + "(";
+  for (int i = 0; i < kN32; i++) s += fmt("%s.param .b32 a_%s", i ? ", " : "", kCtx32[i]);
+  for (int i = 0; i < kN64; i++) s += fmt(", .param .b64 a_%s", kCtx64[i]);
+  return s + ")";
+}
+
+// one step function: steps [s0, s1)
+std::string step_function(const Program &G, const std::string &name, uint32_t s0, uint32_t s1) {
+  Em e;
+  for (uint32_t s = s0; s < s1; s++) {
+    // per-warp lists: bit ops round-robin over warps, then the warp's descriptors
+    std::vector<std::string> cases(G.L);
+    for (uint32_t w = 0; w < G.L; w++) {
+      Em c;
+      c.nr = e.nr; c.nrd = e.nrd; c.np = e.np; c.nlab = e.nlab;
+      for (uint32_t k = G.bit_ptr[s] + w; k < G.bit_ptr[s + 1]; k += G.L) emit_bit(c, G.bitdesc[k]);
+      for (uint32_t k = G.step_ptr[s * G.L + w]; k < G.step_ptr[s * G.L + w + 1]; k++) emit_desc(c, G, G.desc[k]);
+      e.nr = c.nr; e.nrd = c.nrd; e.np = c.np; e.nlab = c.nlab;
+      cases[w] = std::move(c.s);
+    }
+    std::string end = e.L("E");
+    if (G.L > 1) {
+      std::string tbl = e.L("T");
+      std::vector<std::string> labs(G.L);
+      std::string targets;
+      for (uint32_t w = 0; w < G.L; w++) {
+        labs[w] = e.L("W");
+        targets += (w ? ", " : "") + labs[w];
+      }
+      e.s += tbl + ": .branchtargets " + targets + ";\n";
+      e.l(fmt("brx.idx %%wl, %s", tbl.c_str()));
+      for (uint32_t w = 0; w < G.L; w++) {
+        e.lab(labs[w]);
+        e.s += cases[w];
+        e.l(fmt("bra.uni %s", end.c_str()));
+      }
+    } else {
+      e.s += cases[0];
+    }
+    e.lab(end);
+    e.l("cp.async.commit_group");
+    e.l(fmt("cp.async.wait_group %u", G.step_wait[s]));
+    e.l("bar.sync 0");
+  }
+  std::string out = func_proto(name) + "\n{\n";
+  out += fmt("\t.reg .b32 %%r<%u>;\n\t.reg .b64 %%rd<%u>;\n\t.reg .pred %%p<%u>;\n", e.nr + 1, e.nrd + 1, e.np + 1);
+  out += "\t.reg .b32 %smb, %lane, %wl, %N, %rw, %rh, %rb, %N4, %N2, %Nb;\n\t.reg .b64 ";
+  for (int i = 0; i < kN64; i++) out += fmt("%s%%%s", i ? ", " : "", kCtx64[i]);
+  out += ";\n\t.reg .pred %pl0, %pl8, %pl16, %pdig;\n";
+  for (int i = 0; i < kN32; i++) out += fmt("\tld.param.u32 %%%s, [a_%s];\n", kCtx32[i], kCtx32[i]);
+  for (int i = 0; i < kN64; i++) out += fmt("\tld.param.u64 %%%s, [a_%s];\n", kCtx64[i], kCtx64[i]);
+  out += "\tmad.lo.u32 %rw, %lane, 4, %smb;\n\tmad.lo.u32 %rh, %lane, 2, %smb;\n\tadd.u32 %rb, %lane, %smb;\n"
+         "\tshl.b32 %N4, %N, 2;\n\tshl.b32 %N2, %N, 1;\n\tshr.u32 %Nb, %N, 3;\n"
+         "\tsetp.eq.u32 %pl0, %lane, 0;\n\tsetp.lt.u32 %pl8, %lane, 8;\n\tsetp.lt.u32 %pl16, %lane, 16;\n"
+         "\tsetp.ne.u64 %pdig, %dig, 0;\n";
+  out += e.s;
+  out += "\tret;\n}\n";
+  return out;
+}
+
+}  // namespace
+
+std::string jit_partition_ptx(const Program &G, uint32_t q, const std::string &rt_ptx) {
+  const uint32_t s0 = G.part_steps[q], s1 = G.part_steps[q + 1];
+  std::string mod;
+  mod.reserve(1 << 20);
+  mod += ".version 8.8\n.target sm_100a\n.address_size 64\n\n";
+  mod += rt_ptx;
+  mod += "\n.extern .shared .align 16 .b8 dyn_smem[];\n\n";
+  // step groups of bounded size (ptxas time is superlinear in function size)
+  std::vector<std::pair<uint32_t, uint32_t>> groups;
+  static const uint64_t kGroupOps = getenv("RTLSIM_JIT_GROUP") ? strtoull(getenv("RTLSIM_JIT_GROUP"), nullptr, 10) : 400;
+  uint32_t g0 = s0;
+  uint64_t acc = 0;
+  for (uint32_t s = s0; s < s1; s++) {
+    acc += (G.step_ptr[(s + 1) * G.L] - G.step_ptr[s * G.L]) + (G.bit_ptr[s + 1] - G.bit_ptr[s]);
+    if (acc >= kGroupOps || s + 1 == s1) {
+      groups.push_back({g0, s + 1});
+      g0 = s + 1;
+      acc = 0;
+    }
+  }
+  for (size_t g = 0; g < groups.size(); g++)
+    mod += step_function(G, fmt("rtl_steps_%zu", g), groups[g].first, groups[g].second) + "\n";
+  // the kernel: per-thread context, then the step functions in order
+  mod += fmt(".visible .entry rtl_jit_part(.param .align 8 .b8 prm[%zu])\n.maxntid %u, 1, 1\n{\n",
+             sizeof(JitParams), 32u * G.L);
+  mod += "\t.reg .b32 %tidx, %tile, %s, %smb, %lane, %wl, %N;\n\t.reg .b64 %t64, %b64, %digb;\n\t.reg .pred %pz;\n\t.reg .b64 ";
+  for (int i = 0; i < kN64; i++) mod += fmt("%s%%%s", i ? ", " : "", kCtx64[i]);
+  mod += ";\n";
+  mod += "\tmov.u32 %tidx, %tid.x;\n\tand.b32 %lane, %tidx, 31;\n\tshr.u32 %wl, %tidx, 5;\n\tmov.u32 %tile, %ctaid.x;\n"
+         "\tmad.lo.u32 %s, %tile, 32, %lane;\n";
+  mod += fmt("\tld.param.u32 %%N, [prm+%zu];\n", offsetof(JitParams, N));
+  const size_t aoff[4] = {offsetof(JitParams, cur), offsetof(JitParams, nxt), offsetof(JitParams, xnet),
+                          offsetof(JitParams, in)};
+  const char *tag[4] = {"c", "n", "x", "i"};
+  for (int A = 0; A < 4; A++) {
+    // bit rows: + tile*4 ; u8: + tile*32 + lane*4 ; u16: + tile*64 + lane*4 ; u32: + tile*128 + lane*4
+    const uint32_t tmul[4] = {4, 32, 64, 128};
+    for (int k = 0; k < 4; k++) {
+      mod += fmt("\tld.param.u64 %%b64, [prm+%zu];\n", aoff[A] + 8 * k);
+      mod += fmt("\tmul.wide.u32 %%t64, %%tile, %u;\n\tadd.u64 %%tb_%s%d, %%b64, %%t64;\n", tmul[k], tag[A], k);
+      if (k > 0) mod += fmt("\tmul.wide.u32 %%t64, %%lane, 4;\n\tadd.u64 %%tb_%s%d, %%tb_%s%d, %%t64;\n", tag[A], k, tag[A], k);
+    }
+  }
+  mod += fmt("\tld.param.u64 %%b64, [prm+%zu];\n\tmul.wide.u32 %%t64, %%s, 4;\n\tadd.u64 %%outb, %%b64, %%t64;\n",
+             offsetof(JitParams, out));
+  mod += fmt("\tld.param.u64 %%digb, [prm+%zu];\n\tmul.wide.u32 %%t64, %%s, 8;\n\tadd.u64 %%t64, %%digb, %%t64;\n"
+             "\tsetp.eq.u64 %%pz, %%digb, 0;\n\tselp.b64 %%dig, 0, %%t64, %%pz;\n",
+             offsetof(JitParams, digest));
+  mod += fmt("\tld.param.u64 %%wide, [prm+%zu];\n", offsetof(JitParams, wide));
+  mod += "\tmov.u32 %smb, dyn_smem;\n\tcvta.shared.u64 %smg, dyn_smem;\n";
+  for (size_t g = 0; g < groups.size(); g++) {
+    mod += "\t{\n";
+    std::string args;
+    int pi = 0;
+    for (int i = 0; i < kN32; i++, pi++) {
+      mod += fmt("\t.param .b32 q%d;\n\tst.param.b32 [q%d], %%%s;\n", pi, pi, kCtx32[i]);
+      args += fmt("%sq%d", pi ? ", " : "", pi);
+    }
+    for (int i = 0; i < kN64; i++, pi++) {
+      mod += fmt("\t.param .b64 q%d;\n\tst.param.b64 [q%d], %%%s;\n", pi, pi, kCtx64[i]);
+      args += fmt(", q%d", pi);
+    }
+    mod += fmt("\tcall.uni rtl_steps_%zu, (%s);\n\t}\n", g, args.c_str());
+  }
+  mod += "\tret;\n}\n";
+  return mod;
+}
+
+static int compile_ptx(const std::string &ptx, std::vector<char> *cubin, std::string *err) {
+  nvPTXCompilerHandle h = nullptr;
+  if (nvPTXCompilerCreate(&h, ptx.size(), ptx.c_str()) != NVPTXCOMPILE_SUCCESS) {
+    *err = "nvPTXCompilerCreate failed";
+    return -1;
+  }
+  const char *opts[] = {"--gpu-name=sm_100a", "-O3"};
+  nvPTXCompileResult rc = nvPTXCompilerCompile(h, 2, opts);
+  if (rc != NVPTXCOMPILE_SUCCESS) {
+    size_t n = 0;
+    nvPTXCompilerGetErrorLogSize(h, &n);
+    std::string log(n, '\0');
+    if (n) nvPTXCompilerGetErrorLog(h, &log[0]);
+    *err = "ptx compile failed: " + log.substr(0, 2000);
+    nvPTXCompilerDestroy(&h);
+    return -1;
+  }
+  size_t n = 0;
+  nvPTXCompilerGetCompiledProgramSize(h, &n);
+  cubin->resize(n);
+  nvPTXCompilerGetCompiledProgram(h, cubin->data());
+  nvPTXCompilerDestroy(&h);
+  return 0;
+}
+
+int jit_build(const Program &G, const std::string &rt_ptx_path, uint32_t smem_bytes, int device, JitKernels *out,
+              std::string *err) {
+  std::ifstream f(rt_ptx_path);
+  if (!f) {
+    *err = "cannot read " + rt_ptx_path;
+    return RTLSIM_E_ARG;
+  }
+  std::stringstream ss;
+  ss << f.rdbuf();
+  // strip the header lines (.version/.target/.address_size) of the runtime PTX
+  std::string rt, line;
+  std::istringstream is(ss.str());
+  while (std::getline(is, line)) {
+    if (line.rfind(".version", 0) == 0 || line.rfind(".target", 0) == 0 || line.rfind(".address_size", 0) == 0) continue;
+    rt += line + "\n";
+  }
+  const uint32_t NP = (uint32_t)G.part_steps.size() - 1;
+  out->kern.assign(NP, nullptr);
+  out->libs.assign(NP, nullptr);
+  std::vector<std::vector<char>> cubins(NP);
+  std::vector<std::string> errs(NP);
+  std::atomic<uint32_t> next{0};
+  std::atomic<size_t> ptx_bytes{0};
+  auto t0 = std::chrono::steady_clock::now();
+  unsigned nth = std::max(1u, std::thread::hardware_concurrency());
+  std::vector<std::thread> th;
+  for (unsigned t = 0; t < std::min<unsigned>(nth, NP ? NP : 1); t++) {
+    th.emplace_back([&]() {
+      for (uint32_t q; (q = next++) < NP;) {
+        if (G.part_steps[q] == G.part_steps[q + 1]) continue;
+        std::string ptx = jit_partition_ptx(G, q, rt);
+        ptx_bytes += ptx.size();
+        if (compile_ptx(ptx, &cubins[q], &errs[q]) != 0 && getenv("RTLSIM_JIT_DUMP")) {
+          std::ofstream o(fmt("/tmp/rtlsim_jit_fail_%u.ptx", q));
+          o << ptx;
+        }
+      }
+    });
+  }
+  for (auto &t : th) t.join();
+  auto t1 = std::chrono::steady_clock::now();
+  out->compile_s = std::chrono::duration<double>(t1 - t0).count();
+  out->ptx_bytes = ptx_bytes;
+  for (uint32_t q = 0; q < NP; q++)
+    if (!errs[q].empty()) {
+      *err = fmt("partition %u: ", q) + errs[q];
+      return RTLSIM_E_ARG;
+    }
+  for (uint32_t q = 0; q < NP; q++) {
+    if (cubins[q].empty()) continue;
+    out->cubin_bytes += cubins[q].size();
+    if (device < 0) continue;
+    cudaError_t e = cudaLibraryLoadData(&out->libs[q], cubins[q].data(), nullptr, nullptr, 0, nullptr, nullptr, 0);
+    if (e == cudaSuccess) e = cudaLibraryGetKernel(&out->kern[q], out->libs[q], "rtl_jit_part");
+    if (e == cudaSuccess)
+      e = cudaKernelSetAttributeForDevice(out->kern[q], cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                          (int)std::max<uint32_t>(smem_bytes, 1024), device);
+    if (e != cudaSuccess) {
+      *err = std::string("loading JIT kernel: ") + cudaGetErrorString(e);
+      cudaGetLastError();
+      return RTLSIM_E_CUDA;
+    }
+  }
+  return RTLSIM_OK;
+}
+
+void jit_free(JitKernels *k) {
+  for (cudaLibrary_t l : k->libs)
+    if (l) cudaLibraryUnload(l);
+  k->libs.clear();
+  k->kern.clear();
+}
+
+}  // namespace rtlsim

@@ -1,0 +1,48 @@
+// jit.h — specialized per-partition kernels (RTLSIM_F_JIT).
+//
+// The interpreter (kernels.cu) is issue-bound: decoding, dispatch and layout
+// branches cost ~100 SASS instructions per op. PAPER.md's own flow transpiles
+// the design into straight-line CUDA per partition; SURVEY
+// §8(f) row 4 keeps that idea as the fallback "if the interpreter stalls on
+// issue". Here the compiled schedule (the same steps, slots and layouts the
+// interpreter walks) is translated into PTX — one kernel per partition, steps
+// split into device functions so ptxas time stays linear — compiled in-process
+// with nvPTXCompiler on all host cores and loaded with cudaLibraryLoadData.
+#pragma once
+#include <cuda_runtime.h>
+
+#include <cstdint>
+#include <string>
+#include <vector>
+
+#include "program.h"
+
+namespace rtlsim {
+
+// Kernel parameter block of a JIT partition kernel (one cycle per launch).
+struct JitParams {
+  uint64_t cur[4], nxt[4], xnet[4], in[4];   // arena bases per class (bit, u8, u16, u32)
+  uint64_t out;                              // out rows of this cycle: [OW][N_pad] u32
+  uint64_t digest;                           // digest row of this cycle [N_pad] u64, or 0
+  uint64_t wide;                             // WideRec array (generic path)
+  uint32_t N;                                // N_pad
+  uint32_t pad;
+};
+static_assert(sizeof(JitParams) == 160, "JitParams layout is hard-coded in the PTX generator");
+
+struct JitKernels {
+  std::vector<cudaLibrary_t> libs;
+  std::vector<cudaKernel_t> kern;   // per exec-order partition (nullptr: empty partition)
+  double gen_s = 0, compile_s = 0;
+  size_t ptx_bytes = 0, cubin_bytes = 0;
+};
+
+// PTX text of exec-order partition q (steps part_steps[q]..part_steps[q+1]).
+std::string jit_partition_ptx(const Program &G, uint32_t q, const std::string &rt_ptx);
+// Generate + compile (nvPTXCompiler, all host cores) + load every partition.
+// device < 0: generate and compile only (host-only contexts, CPU tests).
+int jit_build(const Program &G, const std::string &rt_ptx_path, uint32_t smem_bytes, int device, JitKernels *out,
+              std::string *err);
+void jit_free(JitKernels *k);
+
+}  // namespace rtlsim

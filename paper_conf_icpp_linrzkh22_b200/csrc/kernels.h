@@ -33,6 +33,7 @@ struct EvalParams {
   const uint4 *desc;          // 16-byte descriptors (program.h Desc), padded by 32
   const uint4 *bitdesc;       // bit-sliced ops (program.h BitDesc)
   const uint32_t *bit_ptr;    // [n_steps + 1]
+  const uint32_t *step_wait;  // [n_steps] cp.async wait depth at the step end
   const WideRec *wide;        // generic-path records
   const uint32_t *step_ptr;   // [n_steps * L + 1]: lane l of step s = [p[sL+l], p[sL+l+1])
   uint32_t step_begin, step_end, L;

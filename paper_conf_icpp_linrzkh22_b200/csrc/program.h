@@ -133,6 +133,7 @@ struct Program {
   std::vector<uint32_t> step_ptr;       // [n_steps * L + 1]: lane l of step s = [p[s*L+l], p[s*L+l+1])
   std::vector<BitDesc> bitdesc;         // bit-sliced ops, step-major
   std::vector<uint32_t> bit_ptr;        // [n_steps + 1]
+  std::vector<uint32_t> step_wait;      // [n_steps] cp.async groups allowed pending at the step end
   std::vector<WideRec> wide;            // records referenced by CODE_WIDE
   std::vector<uint32_t> part_steps;     // exec-order partition boundaries in steps (size P+1)
   uint32_t smem_words = 0;              // shared words per tile (slots)

@@ -22,6 +22,9 @@
 #include <vector>
 
 #include "../../include/rtlsim.h"
+#include <dlfcn.h>
+
+#include "jit.h"
 #include "kernels.h"
 #include "program.h"
 
@@ -67,7 +70,7 @@ struct rtlsim_ctx {
   std::vector<void *> host_allocs;    // pinned, freed at re-bind
   // static device data
   uint4 *d_desc = nullptr, *d_bitdesc = nullptr;
-  uint32_t *d_bitptr = nullptr;
+  uint32_t *d_bitptr = nullptr, *d_stepwait = nullptr;
   WideRec *d_wide = nullptr;
   uint32_t *d_step = nullptr, *d_consts = nullptr, *d_mask = nullptr, *d_reginit = nullptr;
   RegWord *d_regmap = nullptr;
@@ -100,6 +103,8 @@ struct rtlsim_ctx {
   std::vector<cudaEvent_t> event_pool;
   double eval_ms = 0;
   uint64_t eval_launches = 0, eval_stim_cycles = 0;
+  JitKernels jit;        // RTLSIM_F_JIT
+  uint32_t jit_smem = 0;
 };
 
 #define CK(call)                                                                       \
@@ -201,7 +206,27 @@ extern "C" int rtlsim_load(const rtlsim_ir *ir, const rtlsim_options *opt, rtlsi
     return RTLSIM_E_NOMEM;
   }
   if (ctx->opt.chunk_cycles) ctx->Tc = ctx->opt.chunk_cycles;
+  auto jit_setup = [&](int device) -> int {
+    Dl_info info;
+    std::string dir = ".";
+    if (dladdr((void *)&rtlsim_load, &info) && info.dli_fname) {
+      dir = info.dli_fname;
+      dir = dir.substr(0, dir.find_last_of('/'));
+    }
+    ctx->jit_smem = std::max<uint32_t>(G.smem_words * 4u, 16u);
+    std::string jerr;
+    int jr = jit_build(G, dir + "/jit_rt.ptx", ctx->jit_smem, device, &ctx->jit, &jerr);
+    if (jr != RTLSIM_OK) g_load_error = "JIT: " + jerr;
+    return jr;
+  };
   if (ctx->host_only) {
+    if (ctx->opt.flags & RTLSIM_F_JIT) {
+      int jr = jit_setup(-1);   // generate + compile (no device needed)
+      if (jr != RTLSIM_OK) {
+        delete ctx;
+        return jr;
+      }
+    }
     *out = ctx;
     return RTLSIM_OK;
   }
@@ -222,6 +247,7 @@ extern "C" int rtlsim_load(const rtlsim_ir *ir, const rtlsim_options *opt, rtlsi
   if (e == cudaSuccess) e = up((void **)&ctx->d_desc, padded.data(), padded.size() * sizeof(Desc));
   if (e == cudaSuccess) e = up((void **)&ctx->d_bitdesc, G.bitdesc.data(), G.bitdesc.size() * sizeof(BitDesc));
   if (e == cudaSuccess) e = up((void **)&ctx->d_bitptr, G.bit_ptr.data(), G.bit_ptr.size() * 4);
+  if (e == cudaSuccess) e = up((void **)&ctx->d_stepwait, G.step_wait.data(), G.step_wait.size() * 4);
   if (e == cudaSuccess) e = up((void **)&ctx->d_wide, G.wide.data(), G.wide.size() * sizeof(WideRec));
   if (e == cudaSuccess) e = up((void **)&ctx->d_inmap, G.in_map.data(), G.in_map.size() * 4);
   if (e == cudaSuccess) e = up((void **)&ctx->d_step, G.step_ptr.data(), G.step_ptr.size() * 4);
@@ -252,6 +278,13 @@ extern "C" int rtlsim_load(const rtlsim_ir *ir, const rtlsim_options *opt, rtlsi
     cudaGetLastError();
     rtlsim_free(ctx);
     return e == cudaErrorMemoryAllocation ? RTLSIM_E_NOMEM : RTLSIM_E_CUDA;
+  }
+  if (ctx->opt.flags & RTLSIM_F_JIT) {
+    int jr = jit_setup(ctx->device);
+    if (jr != RTLSIM_OK) {
+      rtlsim_free(ctx);
+      return jr;
+    }
   }
   ctx->static_bytes = ctx->device_bytes;
   *out = ctx;
@@ -376,6 +409,7 @@ static EvalParams eval_params(rtlsim_ctx *ctx, int b, uint64_t cycle0, uint32_t 
   p.desc = ctx->d_desc;
   p.bitdesc = ctx->d_bitdesc;
   p.bit_ptr = ctx->d_bitptr;
+  p.step_wait = ctx->d_stepwait;
   p.wide = ctx->d_wide;
   p.step_ptr = ctx->d_step;
   p.step_begin = 0;
@@ -435,7 +469,7 @@ static int launch_chunk(rtlsim_ctx *ctx, int b, uint64_t cycle0, uint32_t nc, bo
     CK(get_event(ctx, &tm.b));
     CK(cudaEventRecord(tm.a, ctx->st));
   }
-  if (!(ctx->opt.flags & RTLSIM_F_GRAPH)) {
+  if (!(ctx->opt.flags & (RTLSIM_F_GRAPH | RTLSIM_F_JIT))) {
     EvalParams p = eval_params(ctx, b, cycle0, nc, digest);
     CK(launch_eval(p, ctx->smem_bytes, ctx->st));
     ctx->launches++;
@@ -445,8 +479,9 @@ static int launch_chunk(rtlsim_ctx *ctx, int b, uint64_t cycle0, uint32_t nc, bo
     }
     return RTLSIM_OK;
   }
-  // graph mode: Tc x P per-(cycle, partition) nodes, captured once per
-  // (buffer, parity, nc, digest) and replayed
+  const bool jit = (ctx->opt.flags & RTLSIM_F_JIT) != 0;
+  // graph mode (and JIT mode): Tc x P per-(cycle, partition) nodes, captured
+  // once per (buffer, parity, nc, digest) and replayed
   const uint64_t key = ((uint64_t)nc << 8) | ((uint64_t)b << 2) | ((cycle0 & 1ull) << 1) | (digest ? 1u : 0u);
   auto it = ctx->graphs.find(key);
   if (it == ctx->graphs.end()) {
@@ -457,6 +492,34 @@ static int launch_chunk(rtlsim_ctx *ctx, int b, uint64_t cycle0, uint32_t nc, bo
     for (uint32_t c = 0; c < nc; c++) {
       for (uint32_t q = 0; q < NP; q++) {
         if (G.part_steps[q] == G.part_steps[q + 1]) continue;
+        if (jit) {
+          if (!ctx->jit.kern[q]) continue;
+          const uint32_t par = (uint32_t)(((cycle0 & 1ull) + c) & 1ull);
+          JitParams jp{};
+          const Arena *ar[3] = {&ctx->state[par], &ctx->state[par ^ 1u], &ctx->xnet};
+          uint64_t *dst[3] = {jp.cur, jp.nxt, jp.xnet};
+          for (int t = 0; t < 3; t++) {
+            dst[t][0] = (uint64_t)ar[t]->bit; dst[t][1] = (uint64_t)ar[t]->u8;
+            dst[t][2] = (uint64_t)ar[t]->u16; dst[t][3] = (uint64_t)ar[t]->u32;
+          }
+          jp.in[0] = (uint64_t)(ctx->d_in[b].bit + (size_t)c * ctx->in_stride.s[CLS_BIT]);
+          jp.in[1] = (uint64_t)(ctx->d_in[b].u8 + (size_t)c * ctx->in_stride.s[CLS_U8]);
+          jp.in[2] = (uint64_t)(ctx->d_in[b].u16 + (size_t)c * ctx->in_stride.s[CLS_U16]);
+          jp.in[3] = (uint64_t)(ctx->d_in[b].u32 + (size_t)c * ctx->in_stride.s[CLS_U32]);
+          jp.out = (uint64_t)(ctx->d_out[b] + (size_t)c * G.OW * ctx->N_pad);
+          jp.digest = digest ? (uint64_t)(ctx->d_dig[b] + (size_t)c * ctx->N_pad) : 0;
+          jp.wide = (uint64_t)ctx->d_wide;
+          jp.N = ctx->N_pad;
+          void *args[] = {&jp};
+          cudaError_t e = cudaLaunchKernel((const void *)ctx->jit.kern[q], dim3(ctx->N_pad / 32u), dim3(32u * G.L),
+                                           args, ctx->jit_smem, cap);
+          if (e != cudaSuccess) {
+            cudaGraph_t g;
+            cudaStreamEndCapture(cap, &g);
+            return cuda_fail(ctx, e, "JIT graph capture", __LINE__);
+          }
+          continue;
+        }
         EvalParams p = eval_params(ctx, b, (cycle0 & 1ull) + c, 1, digest);
         p.step_begin = G.part_steps[q];
         p.step_end = G.part_steps[q + 1];
@@ -784,6 +847,7 @@ extern "C" void rtlsim_free(rtlsim_ctx *ctx) {
     if (ctx->st_h2d) cudaStreamSynchronize(ctx->st_h2d);
     if (ctx->st_d2h) cudaStreamSynchronize(ctx->st_d2h);
     free_binding(ctx);
+    jit_free(&ctx->jit);
     for (auto &t : ctx->timed_pending) {
       cudaEventDestroy(t.a);
       cudaEventDestroy(t.b);

@@ -88,6 +88,34 @@ def test_shaped_reduced(R, oracle_lib, cid, scale, N, T):
                 f"config{cid}@{scale}")
 
 
+@pytest.mark.parametrize("seed,parts", [(0, 1), (1, 3), (2, 5)])
+def test_jit_sequential_dag(R, oracle_lib, seed, parts):
+    """The JIT backend (specialized PTX per partition) on wide, partitioned designs."""
+    ir = designs.random_dag(500 + seed, n_ops=300, n_regs=24, n_partitions=parts,
+                            input_widths=(7, 33, 1, 64, 100), max_width=1024)
+    st = stim.stimulus(ir, 11 + seed, np.arange(96), 0, 40, mask=False)
+    assert_same(gpu_run(R, ir, st, chunk_cycles=7, flags=R.F_JIT),
+                oracle_lib.simulate(ir, st, digest=True, threads=8), f"jit seq{seed}")
+
+
+@pytest.mark.parametrize("seed", range(4))
+def test_jit_comb_dag_exhaustive(R, oracle_lib, seed):
+    ir = designs.random_dag(seed, n_ops=60 + 25 * seed, input_widths=(3, 5, 1, 4, 3))
+    st = designs.exhaustive_stimulus(ir)
+    assert_same(gpu_run(R, ir, st, flags=R.F_JIT), oracle_lib.simulate(ir, st, digest=True, threads=8),
+                f"jit dag{seed}")
+
+
+def test_jit_tiny_and_shaped(R, oracle_lib):
+    ir = designs.tiny_dut()
+    st = stim.tiny_stimulus(stim.STIM_SEED_BASE + 1, np.arange(1024), 100, mode="B")
+    assert_same(gpu_run(R, ir, st, flags=R.F_JIT), oracle_lib.simulate(ir, st, digest=True, threads=8), "jit tiny")
+    ir = shaped.generate(3, scale=0.25)
+    st = stim.stimulus(ir, stim.STIM_SEED_BASE + 3, np.arange(160), 0, 24)
+    assert_same(gpu_run(R, ir, st, chunk_cycles=16, flags=R.F_JIT),
+                oracle_lib.simulate(ir, st, digest=True, threads=16), "jit config3@0.25")
+
+
 def test_modes_agree(R, oracle_lib):
     """Graph mode, no-pipeline mode, op-lane counts and chunk sizes change only the schedule."""
     ir = designs.random_dag(600, n_ops=250, n_regs=16, n_partitions=4, input_widths=(9, 40, 1))

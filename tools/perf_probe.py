@@ -18,7 +18,9 @@ for cid in cfgs:
     Tc = 8 if cid == 4 else 32
     T = Tc * 4
     t0 = time.time()
-    sim = R.Simulator(ir, chunk_cycles=Tc, flags=R.F_TIMING, stream=torch.cuda.current_stream().cuda_stream)
+    import os
+    jit = R.F_JIT if os.environ.get('JIT') else 0
+    sim = R.Simulator(ir, chunk_cycles=Tc, flags=R.F_TIMING | jit, stream=torch.cuda.current_stream().cuda_stream)
     tl = time.time() - t0
     st = sim.stats()
     d_stim = stim.stimulus_torch(ir, stim.STIM_SEED_BASE + cid, 0, N, 0, T)

@@ -11,7 +11,8 @@ ir = designs.tiny_dut() if cid == 1 else shaped.generate(cid)
 import os
 N = int(os.environ.get('PROF_N', NS[cid]))
 s = torch.cuda.Stream(); torch.cuda.set_stream(s)
-sim = R.Simulator(ir, chunk_cycles=Tc, stream=s.cuda_stream)
+flags = R.F_JIT if os.environ.get('JIT') else 0
+sim = R.Simulator(ir, chunk_cycles=Tc, stream=s.cuda_stream, flags=flags)
 d_stim = stim.stimulus_torch(ir, stim.STIM_SEED_BASE + cid, 0, N, 0, Tc * nl)
 out = torch.empty((N, Tc, ir.OW), dtype=torch.int32, device='cuda')
 sim.bind_device(d_stim, N, Tc * nl)
