@@ -818,7 +818,9 @@ static int compile_ptx(const std::string &ptx, std::vector<char> *cubin, std::st
     *err = "nvPTXCompilerCreate failed";
     return -1;
   }
-  const char *opts[] = {"--gpu-name=sm_100a", "-O3"};
+  // --Ofast-compile=mid: ~3x faster than -O3 on this straight-line code for
+  // ~2% more SASS (measured on the riscv-mini-shaped design)
+  const char *opts[] = {"--gpu-name=sm_100a", "--Ofast-compile=mid"};
   nvPTXCompileResult rc = nvPTXCompilerCompile(h, 2, opts);
   if (rc != NVPTXCOMPILE_SUCCESS) {
     size_t n = 0;

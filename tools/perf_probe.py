@@ -20,7 +20,7 @@ for cid in cfgs:
     t0 = time.time()
     import os
     jit = R.F_JIT if os.environ.get('JIT') else 0
-    sim = R.Simulator(ir, chunk_cycles=Tc, flags=R.F_TIMING | jit, stream=torch.cuda.current_stream().cuda_stream)
+    sim = R.Simulator(ir, chunk_cycles=Tc, flags=R.F_TIMING | jit, op_lanes=int(os.environ.get('LANES', '0')), stream=torch.cuda.current_stream().cuda_stream)
     tl = time.time() - t0
     st = sim.stats()
     d_stim = stim.stimulus_torch(ir, stim.STIM_SEED_BASE + cid, 0, N, 0, T)
