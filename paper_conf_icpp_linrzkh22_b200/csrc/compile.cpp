@@ -112,6 +112,35 @@ struct SlotAlloc {
 
 }  // namespace
 
+// Specialized interpreter handler for a narrow op (kernels.cu fast_narrow), or
+// 0 for the generic path: handler = 1 + 3 * kind + {U32, U16, U8}.
+static uint32_t fast_handler(uint32_t opc, int ar, const uint32_t *lay, uint32_t ld, const uint32_t *ws,
+                             uint32_t wd) {
+  auto xi = [](uint32_t l) -> int { return l == LC_U32 ? 0 : l == LC_U16 ? 1 : l == LC_U8 ? 2 : -1; };
+  const int X = xi(ld);
+  switch (opc) {
+    case RTLSIM_OP_AND: case RTLSIM_OP_OR: case RTLSIM_OP_XOR: case RTLSIM_OP_ADD: case RTLSIM_OP_SUB:
+    case RTLSIM_OP_MUL:
+      if (X < 0 || lay[0] != ld) return 0;
+      if (lay[1] == ld) return 1 + X;                 // binary X,X->X
+      if (lay[1] == LC_IMM) return 4 + X;             // binary X,IMM->X
+      return 0;
+    case RTLSIM_OP_COPY: case RTLSIM_OP_NOT: case RTLSIM_OP_NEG: case RTLSIM_OP_SLICE:
+      return (X >= 0 && lay[0] == ld) ? 7 + X : 0;    // unary X->X
+    case RTLSIM_OP_SEXT:
+      return (X >= 0 && lay[0] == ld && ws[0] <= 32) ? 7 + X : 0;
+    case RTLSIM_OP_MUX:   // then/else as wide as the result: no extension needed
+      return (X >= 0 && lay[0] == LC_BIT && lay[1] == ld && lay[2] == ld && ws[1] <= wd && ws[2] <= wd) ? 10 + X : 0;
+    case RTLSIM_OP_EQ: case RTLSIM_OP_NE: case RTLSIM_OP_LTU: case RTLSIM_OP_LEU: case RTLSIM_OP_GTU:
+    case RTLSIM_OP_GEU: {
+      const int A = xi(lay[0]);
+      return (ld == LC_BIT && A >= 0 && lay[1] == lay[0] && ar == 2) ? 13 + A : 0;
+    }
+    default:
+      return 0;
+  }
+}
+
 int compile_program(const rtlsim_ir *ir, uint32_t op_lanes, uint32_t smem_limit_words, Program *P,
                     std::string *err) {
   if (!ir || !P) return fail(err, RTLSIM_E_ARG, "NULL ir");
@@ -655,7 +684,8 @@ int compile_program(const rtlsim_ir *ir, uint32_t op_lanes, uint32_t smem_limit_
               (wsrc[0] << 26);
         d.y = D.slot | (off[0] << 16);
         d.z = off[1] | (off[2] << 16);
-        d.w = wsrc[1] | (imm << 6) | ((ar >= 2 ? 1u : 0u) << 11) | ((ar >= 3 ? 1u : 0u) << 12);
+        d.w = wsrc[1] | (imm << 6) | ((ar >= 2 ? 1u : 0u) << 11) | ((ar >= 3 ? 1u : 0u) << 12) |
+              (fast_handler(opc, ar, lay, D.layout, wsrc, D.width) << 13);
         G.n_narrow++;
         uint32_t cost = (opc == RTLSIM_OP_DIVU || opc == RTLSIM_OP_MODU) ? 6 : 2;
         steps[step].lane.push_back({d, cost});

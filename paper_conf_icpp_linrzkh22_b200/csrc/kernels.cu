@@ -66,6 +66,92 @@ __device__ __forceinline__ uint32_t alu1(uint32_t op, uint32_t x, uint32_t y, ui
   }
 }
 
+// ---- specialized narrow handlers (program.h HID_*): operand layouts are
+// fixed per handler, so fetch / store compile to one shared-memory access
+template <int X>
+__device__ __forceinline__ uint32_t ldx(const uint32_t *sm, uint32_t off, uint32_t lane) {
+  if constexpr (X == LC_U32) return sm[off + lane];
+  else if constexpr (X == LC_U16) return reinterpret_cast<const uint16_t *>(sm)[2u * off + lane];
+  else return reinterpret_cast<const uint8_t *>(sm)[4u * off + lane];
+}
+template <int X>
+__device__ __forceinline__ void stx(uint32_t *sm, uint32_t off, uint32_t lane, uint32_t r) {
+  if constexpr (X == LC_U32) sm[off + lane] = r;
+  else if constexpr (X == LC_U16) reinterpret_cast<uint16_t *>(sm)[2u * off + lane] = (uint16_t)r;
+  else reinterpret_cast<uint8_t *>(sm)[4u * off + lane] = (uint8_t)r;
+}
+
+__device__ __forceinline__ uint32_t bin_op(uint32_t op, uint32_t x, uint32_t y) {
+  switch (op) {
+    case RTLSIM_OP_AND: return x & y;
+    case RTLSIM_OP_OR: return x | y;
+    case RTLSIM_OP_XOR: return x ^ y;
+    case RTLSIM_OP_ADD: return x + y;
+    case RTLSIM_OP_SUB: return x - y;
+    default: return x * y;   // MUL
+  }
+}
+
+// kind: 0 binary X,X->X ; 1 binary X,IMM->X ; 2 unary X->X ; 3 MUX BIT,X,X->X ;
+// 4 unsigned compare X,X->BIT
+template <int X, int KIND>
+__device__ __forceinline__ void fast_h(uint32_t *sm, const uint4 q, uint32_t op, uint32_t lane) {
+  const uint32_t wd = (q.x >> 20) & 63u, m = 0xFFFFFFFFu >> (32u - wd);
+  const uint32_t d = q.y & 0xFFFFu, a = q.y >> 16, b = q.z & 0xFFFFu, c = q.z >> 16;
+  if constexpr (KIND == 0 || KIND == 1) {
+    const uint32_t x = ldx<X>(sm, a, lane);
+    const uint32_t y = KIND == 0 ? ldx<X>(sm, b, lane) : b;
+    stx<X>(sm, d, lane, bin_op(op, x, y) & m);
+  } else if constexpr (KIND == 2) {
+    const uint32_t x = ldx<X>(sm, a, lane), wa = q.x >> 26;
+    uint32_t r;
+    switch (op) {
+      case RTLSIM_OP_COPY: r = x; break;
+      case RTLSIM_OP_NOT: r = ~x; break;
+      case RTLSIM_OP_NEG: r = 0u - x; break;
+      case RTLSIM_OP_SLICE: r = x >> ((q.w >> 6) & 31u); break;
+      default: { const uint32_t sb = 1u << (wa - 1u); r = (x ^ sb) - sb; break; }   // SEXT
+    }
+    stx<X>(sm, d, lane, r & m);
+  } else if constexpr (KIND == 3) {
+    const uint32_t sel = (sm[a] >> lane) & 1u;
+    stx<X>(sm, d, lane, ldx<X>(sm, sel ? b : c, lane));
+  } else {
+    const uint32_t x = ldx<X>(sm, a, lane), y = ldx<X>(sm, b, lane);
+    bool t;
+    switch (op) {
+      case RTLSIM_OP_EQ: t = x == y; break;
+      case RTLSIM_OP_NE: t = x != y; break;
+      case RTLSIM_OP_LTU: t = x < y; break;
+      case RTLSIM_OP_LEU: t = x <= y; break;
+      case RTLSIM_OP_GTU: t = x > y; break;
+      default: t = x >= y; break;   // GEU
+    }
+    const uint32_t bits = __ballot_sync(0xFFFFFFFFu, t);
+    if (lane == 0) sm[d] = bits;
+  }
+}
+
+__device__ __forceinline__ void fast_narrow(uint32_t *sm, const uint4 q, uint32_t hid, uint32_t op, uint32_t lane) {
+  switch (hid) {
+    case 1: fast_h<LC_U32, 0>(sm, q, op, lane); break;
+    case 2: fast_h<LC_U16, 0>(sm, q, op, lane); break;
+    case 3: fast_h<LC_U8, 0>(sm, q, op, lane); break;
+    case 4: fast_h<LC_U32, 1>(sm, q, op, lane); break;
+    case 5: fast_h<LC_U16, 1>(sm, q, op, lane); break;
+    case 6: fast_h<LC_U8, 1>(sm, q, op, lane); break;
+    case 7: fast_h<LC_U32, 2>(sm, q, op, lane); break;
+    case 8: fast_h<LC_U16, 2>(sm, q, op, lane); break;
+    case 9: fast_h<LC_U8, 2>(sm, q, op, lane); break;
+    case 10: fast_h<LC_U32, 3>(sm, q, op, lane); break;
+    case 11: fast_h<LC_U16, 3>(sm, q, op, lane); break;
+    case 12: fast_h<LC_U8, 3>(sm, q, op, lane); break;
+    case 13: fast_h<LC_U32, 4>(sm, q, op, lane); break;
+    case 14: fast_h<LC_U16, 4>(sm, q, op, lane); break;
+    default: fast_h<LC_U8, 4>(sm, q, op, lane); break;
+  }
+}
+
 // bit-sliced op: 3-input truth table applied to packed words (32 stimuli)
 __device__ __forceinline__ void exec_bit(uint32_t *sm, const uint4 q) {
   const uint32_t lut = q.x & 0xFFu, immf = q.x >> 8;
@@ -140,6 +226,11 @@ __global__ void __launch_bounds__(512, 2) rtl_eval_kernel(const EvalParams p) {
           const uint4 q = dbuf[j];
           const uint32_t code = q.x & 0xFFu;
           if (code < 32u) {   // narrow compute op
+            const uint32_t hid = (q.w >> 13) & 31u;
+            if (hid) {   // specialized handler: uniform operand layout, one small op switch
+              fast_narrow(sm, q, hid, code, lane);
+              continue;
+            }
             const uint32_t x = fetch1(sm, q.y >> 16, (q.x >> 8) & 7u, lane);
             const uint32_t y = (q.w & (1u << 11)) ? fetch1(sm, q.z & 0xFFFFu, (q.x >> 11) & 7u, lane) : 0u;
             const uint32_t z = (q.w & (1u << 12)) ? fetch1(sm, q.z >> 16, (q.x >> 14) & 7u, lane) : 0u;
