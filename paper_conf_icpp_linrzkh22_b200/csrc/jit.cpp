@@ -688,44 +688,36 @@ std::string func_proto(const std::string &name) {
   return s + ")";
 }
 
-// one step function: steps [s0, s1)
+// one step function: steps [s0, s1). The code is laid out per warp — each
+// warp's ops of all the steps follow each other, with the step barrier
+// (bar.sync 0, counted per CTA, not per PC) inside every warp's stream — so
+// a warp's instruction fetch is sequential across steps instead of jumping
+// over the other warps' code at every step.
 std::string step_function(const Program &G, const std::string &name, uint32_t s0, uint32_t s1) {
   Em e;
-  for (uint32_t s = s0; s < s1; s++) {
-    // per-warp lists: bit ops round-robin over warps, then the warp's descriptors
-    std::vector<std::string> cases(G.L);
+  std::vector<std::string> labs(G.L);
+  std::string tbl = e.L("T"), end = e.L("E");
+  if (G.L > 1) {
+    std::string targets;
     for (uint32_t w = 0; w < G.L; w++) {
-      Em c;
-      c.nr = e.nr; c.nrd = e.nrd; c.np = e.np; c.nlab = e.nlab;
-      for (uint32_t k = G.bit_ptr[s] + w; k < G.bit_ptr[s + 1]; k += G.L) emit_bit(c, G.bitdesc[k]);
-      for (uint32_t k = G.step_ptr[s * G.L + w]; k < G.step_ptr[s * G.L + w + 1]; k++) emit_desc(c, G, G.desc[k]);
-      e.nr = c.nr; e.nrd = c.nrd; e.np = c.np; e.nlab = c.nlab;
-      cases[w] = std::move(c.s);
+      labs[w] = e.L("W");
+      targets += (w ? ", " : "") + labs[w];
     }
-    std::string end = e.L("E");
-    if (G.L > 1) {
-      std::string tbl = e.L("T");
-      std::vector<std::string> labs(G.L);
-      std::string targets;
-      for (uint32_t w = 0; w < G.L; w++) {
-        labs[w] = e.L("W");
-        targets += (w ? ", " : "") + labs[w];
-      }
-      e.s += tbl + ": .branchtargets " + targets + ";\n";
-      e.l(fmt("brx.idx %%wl, %s", tbl.c_str()));
-      for (uint32_t w = 0; w < G.L; w++) {
-        e.lab(labs[w]);
-        e.s += cases[w];
-        e.l(fmt("bra.uni %s", end.c_str()));
-      }
-    } else {
-      e.s += cases[0];
-    }
-    e.lab(end);
-    e.l("cp.async.commit_group");
-    e.l(fmt("cp.async.wait_group %u", G.step_wait[s]));
-    e.l("bar.sync 0");
+    e.s += tbl + ": .branchtargets " + targets + ";\n";
+    e.l(fmt("brx.idx %%wl, %s", tbl.c_str()));
   }
+  for (uint32_t w = 0; w < G.L; w++) {
+    if (G.L > 1) e.lab(labs[w]);
+    for (uint32_t s = s0; s < s1; s++) {
+      for (uint32_t k = G.bit_ptr[s] + w; k < G.bit_ptr[s + 1]; k += G.L) emit_bit(e, G.bitdesc[k]);
+      for (uint32_t k = G.step_ptr[s * G.L + w]; k < G.step_ptr[s * G.L + w + 1]; k++) emit_desc(e, G, G.desc[k]);
+      e.l("cp.async.commit_group");
+      e.l(fmt("cp.async.wait_group %u", G.step_wait[s]));
+      e.l("bar.sync 0");
+    }
+    if (G.L > 1) e.l(fmt("bra.uni %s", end.c_str()));
+  }
+  e.lab(end);
   std::string out = func_proto(name) + "\n{\n";
   out += fmt("\t.reg .b32 %%r<%u>;\n\t.reg .b64 %%rd<%u>;\n\t.reg .pred %%p<%u>;\n", e.nr + 1, e.nrd + 1, e.np + 1);
   out += "\t.reg .b32 %smb, %lane, %wl, %N, %rw, %rh, %rb, %N4, %N2, %Nb;\n\t.reg .b64 ";
