@@ -144,6 +144,9 @@ typedef struct {
   double eval_ms;            /* RTLSIM_F_TIMING: summed evaluator launch time  */
   uint64_t eval_launches;    /* RTLSIM_F_TIMING: timed evaluator launches      */
   uint64_t eval_stim_cycles; /* RTLSIM_F_TIMING: stimulus-cycles they covered  */
+  double jit_compile_s;      /* RTLSIM_F_JIT: PTX generation + compile seconds  */
+  uint64_t jit_cubin_bytes;  /* RTLSIM_F_JIT: SASS bytes of all partition kernels */
+  uint64_t n_bitops, n_narrow, n_wide, n_ld, n_st;   /* op stream composition    */
 } rtlsim_stats_t;
 
 typedef struct rtlsim_ctx rtlsim_ctx;

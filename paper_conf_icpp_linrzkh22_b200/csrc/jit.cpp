@@ -804,7 +804,7 @@ std::string jit_partition_ptx(const Program &G, uint32_t q, const std::string &r
   return mod;
 }
 
-static int compile_ptx(const std::string &ptx, std::vector<char> *cubin, std::string *err) {
+static int compile_ptx(const std::string &ptx, bool o3, std::vector<char> *cubin, std::string *err) {
   nvPTXCompilerHandle h = nullptr;
   if (nvPTXCompilerCreate(&h, ptx.size(), ptx.c_str()) != NVPTXCOMPILE_SUCCESS) {
     *err = "nvPTXCompilerCreate failed";
@@ -812,7 +812,7 @@ static int compile_ptx(const std::string &ptx, std::vector<char> *cubin, std::st
   }
   // --Ofast-compile=mid: ~3x faster than -O3 on this straight-line code for
   // ~2% more SASS (measured on the riscv-mini-shaped design)
-  const char *opts[] = {"--gpu-name=sm_100a", "--Ofast-compile=mid"};
+  const char *opts[] = {"--gpu-name=sm_100a", o3 ? "-O3" : "--Ofast-compile=mid"};
   nvPTXCompileResult rc = nvPTXCompilerCompile(h, 2, opts);
   if (rc != NVPTXCOMPILE_SUCCESS) {
     size_t n = 0;
@@ -848,6 +848,13 @@ int jit_build(const Program &G, const std::string &rt_ptx_path, uint32_t smem_by
     rt += line + "\n";
   }
   const uint32_t NP = (uint32_t)G.part_steps.size() - 1;
+  // ptxas -O3 schedules this code ~1.8x better (config 3) but compiles ~3x
+  // slower than --Ofast-compile=mid: use it unless the design is large
+  // (RTLSIM_JIT_OPT=O3 / mid overrides)
+  const uint64_t nops = G.desc.size() + G.bitdesc.size();
+  const char *lvl = getenv("RTLSIM_JIT_OPT");
+  const bool o3 = lvl ? strcmp(lvl, "O3") == 0 : nops <= 250000;
+  out->o3 = o3;
   out->kern.assign(NP, nullptr);
   out->libs.assign(NP, nullptr);
   std::vector<std::vector<char>> cubins(NP);
@@ -863,7 +870,7 @@ int jit_build(const Program &G, const std::string &rt_ptx_path, uint32_t smem_by
         if (G.part_steps[q] == G.part_steps[q + 1]) continue;
         std::string ptx = jit_partition_ptx(G, q, rt);
         ptx_bytes += ptx.size();
-        if (compile_ptx(ptx, &cubins[q], &errs[q]) != 0 && getenv("RTLSIM_JIT_DUMP")) {
+        if (compile_ptx(ptx, o3, &cubins[q], &errs[q]) != 0 && getenv("RTLSIM_JIT_DUMP")) {
           std::ofstream o(fmt("/tmp/rtlsim_jit_fail_%u.ptx", q));
           o << ptx;
         }

@@ -34,6 +34,7 @@ struct JitKernels {
   std::vector<cudaLibrary_t> libs;
   std::vector<cudaKernel_t> kern;   // per exec-order partition (nullptr: empty partition)
   double gen_s = 0, compile_s = 0;
+  bool o3 = false;
   size_t ptx_bytes = 0, cubin_bytes = 0;
 };
 

@@ -843,6 +843,10 @@ extern "C" int rtlsim_stats(const rtlsim_ctx *cctx, rtlsim_stats_t *st) {
   st->eval_ms = ctx->eval_ms;
   st->eval_launches = ctx->eval_launches;
   st->eval_stim_cycles = ctx->eval_stim_cycles;
+  st->jit_compile_s = ctx->jit.compile_s;
+  st->jit_cubin_bytes = ctx->jit.cubin_bytes;
+  st->n_bitops = G.n_bitops; st->n_narrow = G.n_narrow; st->n_wide = G.n_wide;
+  st->n_ld = G.n_ld; st->n_st = G.n_st;
   return RTLSIM_OK;
 }
 

@@ -68,7 +68,10 @@ class Stats(ctypes.Structure):
                 ("op_lanes", ctypes.c_uint32), ("chunk_cycles", ctypes.c_uint32), ("tile_stimuli", ctypes.c_uint32),
                 ("iw", ctypes.c_uint32), ("ow", ctypes.c_uint32), ("rw", ctypes.c_uint32),
                 ("device_bytes", ctypes.c_uint64), ("eval_ms", ctypes.c_double),
-                ("eval_launches", ctypes.c_uint64), ("eval_stim_cycles", ctypes.c_uint64)]
+                ("eval_launches", ctypes.c_uint64), ("eval_stim_cycles", ctypes.c_uint64),
+                ("jit_compile_s", ctypes.c_double), ("jit_cubin_bytes", ctypes.c_uint64),
+                ("n_bitops", ctypes.c_uint64), ("n_narrow", ctypes.c_uint64), ("n_wide", ctypes.c_uint64),
+                ("n_ld", ctypes.c_uint64), ("n_st", ctypes.c_uint64)]
 
 
 PRODUCER = ctypes.CFUNCTYPE(ctypes.c_int, ctypes.c_void_p, ctypes.c_uint64, ctypes.c_uint64,
