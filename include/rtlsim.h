@@ -123,7 +123,8 @@ typedef struct {
   uint32_t op_lanes;         /* warps per CTA sharing one stimulus tile (0 = auto) */
   uint32_t chunk_cycles;     /* cycles per launch / pipeline chunk (0 = auto) */
   uint32_t flags;            /* RTLSIM_F_*                                    */
-  uint32_t smem_limit;       /* bytes of shared memory per CTA (0 = device max) */
+  uint32_t smem_limit;       /* bytes of shared memory per CTA (0 = device max);
+                                long-lived values beyond it spill to HBM rows */
 } rtlsim_options;
 
 typedef struct {
@@ -147,6 +148,8 @@ typedef struct {
   double jit_compile_s;      /* RTLSIM_F_JIT: PTX generation + compile seconds  */
   uint64_t jit_cubin_bytes;  /* RTLSIM_F_JIT: SASS bytes of all partition kernels */
   uint64_t n_bitops, n_narrow, n_wide, n_ld, n_st;   /* op stream composition    */
+  double b_spill;            /* of b_state: spill stores + reloads of values that
+                                exceed the smem budget (options.smem_limit) */
 } rtlsim_stats_t;
 
 typedef struct rtlsim_ctx rtlsim_ctx;

@@ -29,6 +29,9 @@ namespace rtlsim {
 
 // external values whose uses are more than this many steps apart are reloaded
 constexpr int32_t kReloadGap = 3;
+// uses of a spilled value closer than this to its definition read the slot
+// (a reload must follow the spill store's step barrier and the load-ahead)
+constexpr int32_t kSpillNear = 4;
 // loads are issued this many steps before their first use (cp.async groups,
 // awaited with a per-step wait depth just before the step barrier)
 static int32_t load_ahead() {
@@ -388,7 +391,16 @@ int compile_program(const rtlsim_ir *ir, uint32_t op_lanes, uint32_t smem_limit_
   std::vector<StepLists> all_steps;   // global step list
   uint32_t peak = dump_words;
   G.part_steps.push_back(0);
-  double bytes_state = 0, bytes_part = 0;
+  double bytes_state = 0, bytes_part = 0, bytes_spill = 0;
+  // spill rows start after the cross-partition net rows; partitions reuse them
+  uint32_t xnet_rows[4], max_spill_rows[4] = {0, 0, 0, 0};
+  for (int c = 0; c < 4; c++) xnet_rows[c] = G.xrows[c];
+  // spill target: the limit minus the descriptor staging buffers (128 words
+  // per op-lane warp; the lane count is not known yet, assume the maximum)
+  const uint32_t stage_words = (op_lanes ? std::min<uint32_t>(op_lanes, 16) : 16) * 128u;
+  const uint32_t step_cap = getenv("RTLSIM_STEP_CAP") ? (uint32_t)atoi(getenv("RTLSIM_STEP_CAP")) : 0;
+  const uint32_t slot_budget =
+      smem_limit_words > stage_words ? smem_limit_words - stage_words : (smem_limit_words ? 1u : 0xFFFFFFFFu);
 
   std::vector<int32_t> vid_of(n, -1);   // per partition: signal -> value id (reset per partition)
   for (uint32_t p : porder) {
@@ -400,59 +412,134 @@ int compile_program(const rtlsim_ir *ir, uint32_t op_lanes, uint32_t smem_limit_
       vals.push_back(Value{s, w, def_step, -1, 1 << 30, 0, layout});
       return (int32_t)vals.size() - 1;
     };
-    // 1. levels of the partition's own ops (ASAP)
+    // The per-tile working set is capped at the slot budget by spilling the
+    // longest-lived local values to rows of the cross-partition arena
+    // (stored one step after definition, reloaded before far uses): HBM
+    // bandwidth is traded for occupancy (more CTAs / warps per SM).
+    std::unordered_map<uint32_t, uint32_t> spilled;   // signal -> row in the xnet arena
+    uint32_t spill_rows[4] = {0, 0, 0, 0};
+    auto row_of_x = [&](uint32_t sg) -> uint32_t {
+      auto it = spilled.find(sg);
+      return it != spilled.end() ? it->second : xrow.at(sg);
+    };
+    std::vector<StepLists> steps;
     std::unordered_map<uint32_t, int32_t> op_step;   // op index -> step
-    op_step.reserve(ops_p.size());
-    for (uint32_t i : ops_p) {
-      const rtlsim_op &o = G.ops[i];
-      uint32_t src[3] = {o.a, o.b, o.c};
-      int32_t lv = 1;
-      for (int k = 0; k < arity(o.opcode); k++) {
-        uint32_t s = src[k];
-        if (G.kind[s] == RTLSIM_COMB && G.ops[def[s]].part == p) lv = std::max(lv, op_step[def[s]] + 1);
-      }
-      op_step[i] = lv;
-    }
-    // Placement that keeps values short-lived (what bounds the per-tile
-    // shared-memory working set): an op whose result feeds later ops of this
-    // partition runs one step before its earliest consumer (ALAP, so loads
-    // and producers move next to their use); an op whose result only leaves
-    // the partition (register D, output, cross-partition net) or is dead runs
-    // right after its latest local operand, or, with none, round-robin over
-    // the partition's steps (no bunching at step 1).
-    {
-      std::unordered_map<uint32_t, int32_t> first_use;   // op -> earliest consumer step
-      first_use.reserve(ops_p.size());
-      for (auto it = ops_p.rbegin(); it != ops_p.rend(); ++it) {
-        auto f = first_use.find(*it);
-        if (f != first_use.end()) op_step[*it] = f->second - 1;   // else: keep ASAP
-        const int32_t st = op_step[*it];
-        const rtlsim_op &o = G.ops[*it];
+    // width cap of the list scheduler: 0 (levels as they are) first, then
+    // halved from half the partition's mean level width while the working
+    // set does not fit the budget even with spilling
+    uint32_t cap = step_cap;
+    int cap_tries = 0, stall = 0;
+    uint32_t best_peak = 0xFFFFFFFFu;
+    bool give_up = false;
+    const size_t wide_base = G.wide.size();
+    const auto snap = std::make_tuple(G.word_ops, G.n_bitops, G.n_narrow, G.n_wide, G.n_ld, G.n_st, bytes_state,
+                                      bytes_part, bytes_spill);
+    for (int attempt = 0;; attempt++) {
+      for (uint32_t s2 : touched) vid_of[s2] = -1;
+      touched.clear();
+      vals.clear();
+      G.wide.resize(wide_base);
+      std::tie(G.word_ops, G.n_bitops, G.n_narrow, G.n_wide, G.n_ld, G.n_st, bytes_state, bytes_part, bytes_spill) =
+          snap;
+      // 1. levels of the partition's own ops (ASAP)
+      op_step.clear();
+      op_step.reserve(ops_p.size());
+      for (uint32_t i : ops_p) {
+        const rtlsim_op &o = G.ops[i];
         uint32_t src[3] = {o.a, o.b, o.c};
+        int32_t lv = 1;
         for (int k = 0; k < arity(o.opcode); k++) {
-          uint32_t sg = src[k];
-          if (G.kind[sg] == RTLSIM_COMB && G.ops[def[sg]].part == p) {
-            auto g = first_use.find((uint32_t)def[sg]);
-            if (g == first_use.end()) first_use[(uint32_t)def[sg]] = st;
-            else g->second = std::min(g->second, st);
+          uint32_t s = src[k];
+          if (G.kind[s] == RTLSIM_COMB && G.ops[def[s]].part == p) lv = std::max(lv, op_step[def[s]] + 1);
+        }
+        op_step[i] = lv;
+      }
+      // Placement that keeps values short-lived (what bounds the per-tile
+      // shared-memory working set): an op whose result feeds later ops of this
+      // partition runs one step before its earliest consumer (ALAP, so loads
+      // and producers move next to their use); an op whose result only leaves
+      // the partition (register D, output, cross-partition net) or is dead runs
+      // right after its latest local operand, or, with none, round-robin over
+      // the partition's steps (no bunching at step 1).
+      {
+        std::unordered_map<uint32_t, int32_t> first_use;   // op -> earliest consumer step
+        first_use.reserve(ops_p.size());
+        for (auto it = ops_p.rbegin(); it != ops_p.rend(); ++it) {
+          auto f = first_use.find(*it);
+          if (f != first_use.end()) op_step[*it] = f->second - 1;   // else: keep ASAP
+          const int32_t st = op_step[*it];
+          const rtlsim_op &o = G.ops[*it];
+          uint32_t src[3] = {o.a, o.b, o.c};
+          for (int k = 0; k < arity(o.opcode); k++) {
+            uint32_t sg = src[k];
+            if (G.kind[sg] == RTLSIM_COMB && G.ops[def[sg]].part == p) {
+              auto g = first_use.find((uint32_t)def[sg]);
+              if (g == first_use.end()) first_use[(uint32_t)def[sg]] = st;
+              else g->second = std::min(g->second, st);
+            }
+          }
+        }
+        int32_t depth = 1;
+        for (uint32_t i : ops_p) depth = std::max(depth, op_step[i]);
+        uint32_t rr = 0;
+        for (uint32_t i : ops_p) {
+          if (first_use.count(i)) continue;
+          const rtlsim_op &o = G.ops[i];
+          uint32_t src[3] = {o.a, o.b, o.c};
+          int32_t lv = 0;
+          for (int k = 0; k < arity(o.opcode); k++) {
+            uint32_t sg = src[k];
+            if (G.kind[sg] == RTLSIM_COMB && G.ops[def[sg]].part == p) lv = std::max(lv, op_step[def[sg]] + 1);
+          }
+          op_step[i] = lv > 0 ? lv : 1 + (int32_t)(rr++ % (uint32_t)depth);
+        }
+      }
+      // Width-capped list scheduling (a working-set bound): the placement above
+      // is kept as the priority, but a step takes at most step_cap ops, so the
+      // wide front of a DAG is stretched over more steps and fewer values are
+      // live at once.
+      if (cap > 0 && ops_p.size() > cap) {
+        std::unordered_map<uint32_t, uint32_t> pending;   // op -> unscheduled local producers
+        std::unordered_map<uint32_t, std::vector<uint32_t>> succ;
+        pending.reserve(ops_p.size());
+        for (uint32_t i : ops_p) {
+          const rtlsim_op &o = G.ops[i];
+          uint32_t src[3] = {o.a, o.b, o.c};
+          uint32_t np = 0;
+          for (int k = 0; k < arity(o.opcode); k++) {
+            uint32_t sg = src[k];
+            if (G.kind[sg] == RTLSIM_COMB && G.ops[def[sg]].part == p) {
+              // a producer feeding two operands counts twice; its successor
+              // entry is added twice too, so the count still reaches zero
+              np++;
+              succ[(uint32_t)def[sg]].push_back(i);
+            }
+          }
+          pending[i] = np;
+        }
+        using QE = std::pair<int32_t, uint32_t>;   // (priority step, op)
+        std::priority_queue<QE, std::vector<QE>, std::greater<QE>> ready;
+        for (uint32_t i : ops_p)
+          if (pending[i] == 0) ready.push({op_step[i], i});
+        std::vector<uint32_t> now;
+        int32_t t = 0;
+        while (!ready.empty()) {
+          t++;
+          now.clear();
+          while (!ready.empty() && now.size() < cap) {
+            now.push_back(ready.top().second);
+            ready.pop();
+          }
+          for (uint32_t i : now) op_step[i] = t;
+          for (uint32_t i : now) {
+            auto it = succ.find(i);
+            if (it == succ.end()) continue;
+            for (uint32_t c : it->second)
+              if (--pending[c] == 0) ready.push({op_step[c], c});
           }
         }
       }
-      int32_t depth = 1;
-      for (uint32_t i : ops_p) depth = std::max(depth, op_step[i]);
-      uint32_t rr = 0;
-      for (uint32_t i : ops_p) {
-        if (first_use.count(i)) continue;
-        const rtlsim_op &o = G.ops[i];
-        uint32_t src[3] = {o.a, o.b, o.c};
-        int32_t lv = 0;
-        for (int k = 0; k < arity(o.opcode); k++) {
-          uint32_t sg = src[k];
-          if (G.kind[sg] == RTLSIM_COMB && G.ops[def[sg]].part == p) lv = std::max(lv, op_step[def[sg]] + 1);
-        }
-        op_step[i] = lv > 0 ? lv : 1 + (int32_t)(rr++ % (uint32_t)depth);
-      }
-    }
+      uint32_t part_peak = 0;
     for (uint32_t i : ops_p) {
       const uint32_t d = G.ops[i].dst;
       vid_of[d] = new_val(d, G.width[d], op_step[i], value_layout(G.width[d], false));
@@ -466,11 +553,19 @@ int compile_program(const rtlsim_ir *ir, uint32_t op_lanes, uint32_t smem_limit_
     //    L1/L2) so the value does not occupy shared memory in between.
     //    Constants <= 16 bits are immediates in the descriptors.
     std::unordered_map<uint32_t, std::vector<int32_t>> ext_uses;   // signal -> op use steps
+    // spilled local values: far uses (>= def + kSpillNear) read reloads of the
+    // spill row instead of keeping the slot live
+    std::unordered_map<uint32_t, std::vector<int32_t>> spill_uses;   // spilled signal -> far use steps
+    auto far_use = [&](uint32_t sg, int32_t st) {
+      return spilled.count(sg) && is_local(sg) && st >= op_step[def[sg]] + kSpillNear;
+    };
     for (uint32_t i : ops_p) {
       const rtlsim_op &o = G.ops[i];
       uint32_t src[3] = {o.a, o.b, o.c};
-      for (int k = 0; k < arity(o.opcode); k++)
+      for (int k = 0; k < arity(o.opcode); k++) {
         if (!is_local(src[k]) && !is_imm(src[k])) ext_uses[src[k]].push_back(op_step[i]);
+        else if (far_use(src[k], op_step[i])) spill_uses[src[k]].push_back(op_step[i]);
+      }
     }
     // sinks: register next state, outputs, cross-partition nets. A sink
     // whose source has another width (register q <= d mod 2^w_q) or is a
@@ -498,7 +593,8 @@ int compile_program(const rtlsim_ir *ir, uint32_t op_lanes, uint32_t smem_limit_
     for (uint32_t r : reg_sinks[p]) add_sink(CODE_ST_REG, G.reg_d[r], G.width[G.reg_q[r]], r);
     for (uint32_t o : out_sinks[p]) add_sink(CODE_ST_OUT, G.output_sig[o], G.width[G.output_sig[o]], o);
     for (uint32_t i : ops_p)
-      if (is_xnet[G.ops[i].dst]) add_sink(CODE_ST_X, G.ops[i].dst, G.width[G.ops[i].dst], G.ops[i].dst);
+      if (is_xnet[G.ops[i].dst] || (spilled.count(G.ops[i].dst) && spill_uses.count(G.ops[i].dst)))
+        add_sink(CODE_ST_X, G.ops[i].dst, G.width[G.ops[i].dst], G.ops[i].dst);
     // immediates: one pseudo-value per constant, always available, no slot
     std::unordered_map<uint32_t, int32_t> imm_val;
     auto imm_of = [&](uint32_t s) -> int32_t {
@@ -543,10 +639,33 @@ int compile_program(const rtlsim_ir *ir, uint32_t op_lanes, uint32_t smem_limit_
         }
         groups[s] = std::move(gs);
       }
+      // reloads of spilled values: issued after the spill store (def + 1) is
+      // visible, i.e. at step >= def + 2
+      std::vector<uint32_t> ssigs;
+      for (auto &kv : spill_uses) ssigs.push_back(kv.first);
+      std::sort(ssigs.begin(), ssigs.end());
+      for (uint32_t s : ssigs) {
+        std::vector<int32_t> &u = spill_uses[s];
+        std::sort(u.begin(), u.end());
+        u.erase(std::unique(u.begin(), u.end()), u.end());
+        const int32_t dstep = op_step[def[s]];
+        std::vector<Group> gs;
+        for (int32_t st : u) {
+          if (gs.empty() || st - gs.back().last > (int32_t)kReloadGap) gs.push_back(Group{st, st, -1});
+          else gs.back().last = st;
+        }
+        for (size_t g = 0; g < gs.size(); g++) {
+          const int32_t issue = std::max(dstep + 2, gs[g].first - load_ahead());
+          gs[g].val = new_val(s, G.width[s], issue, value_layout(G.width[s], false));
+          vals[gs[g].val].last_use = gs[g].last;
+          loads.push_back(Load{s, gs[g].val, issue, false});
+        }
+        groups[s] = std::move(gs);
+      }
     }
     // value holding signal s at step st (local comb, immediate, or the covering load)
     auto val_at = [&](uint32_t s, int32_t st) -> int32_t {
-      if (is_local(s)) return vid(s);
+      if (is_local(s) && !far_use(s, st)) return vid(s);
       if (is_imm(s)) return imm_of(s);
       const std::vector<Group> &gs = groups.at(s);
       for (const Group &g : gs)
@@ -614,10 +733,103 @@ int compile_program(const rtlsim_ir *ir, uint32_t op_lanes, uint32_t smem_limit_
         for (int32_t v : born[s]) vals[v].slot = sa.alloc(vals[v].words());
         for (int32_t v : dies[s]) sa.release(vals[v].slot, vals[v].words());
       }
-      peak = std::max(peak, sa.peak);
+      part_peak = sa.peak;
     }
+      if (part_peak > slot_budget) {
+        // spill more: local values live (beyond their near uses) across the
+        // steps whose working set exceeds the budget, most words x over-budget
+        // steps first, until the projected working set fits
+        std::vector<double> live(nsteps + 1, 0.0);
+        for (auto &v : vals) {
+          if (v.layout == LC_IMM || v.last_use < 0) continue;
+          for (int32_t t = v.def_step; t <= v.last_use; t++) live[t] += v.words();
+        }
+        // live words that fit the budget, given the allocator's fragmentation
+        const double max_live = *std::max_element(live.begin(), live.end());
+        const double target = 0.98 * slot_budget * std::min(1.0, max_live / std::max(1u, part_peak));
+        std::vector<std::pair<double, uint32_t>> cand;
+        for (auto &v : vals) {
+          if (v.layout == LC_IMM || v.last_use < 0 || !is_local(v.sig) || spilled.count(v.sig)) continue;
+          if (vid(v.sig) < 0 || &vals[vid(v.sig)] != &v) continue;   // the defining value only
+          int32_t over = 0;
+          for (int32_t t = v.def_step + kSpillNear; t <= v.last_use; t++) over += live[t] > target;
+          if (over > 0) cand.push_back({(double)v.words() * over, v.sig});
+        }
+        if (part_peak < best_peak) {
+          stall = (part_peak * 100ull > best_peak * 99ull) ? stall + 1 : 0;
+          best_peak = part_peak;
+        } else {
+          stall++;
+        }
+        const bool last_try = cand.empty() || stall >= 3 || attempt >= 24;
+        if (getenv("RTLSIM_SPILL_DEBUG") && (attempt == 0 || last_try) && getenv("RTLSIM_SPILL_DEBUG")[0] == '2') {
+          // live words per step by category: 0 local short, 1 local long, 2 loads, 3 other
+          std::vector<std::array<double, 4>> livec(nsteps + 1, {0, 0, 0, 0});
+          for (auto &v : vals) {
+            if (v.layout == LC_IMM || v.last_use < 0) continue;
+            int cat = 3;
+            if (is_local(v.sig) && vid(v.sig) >= 0 && &vals[vid(v.sig)] == &v)
+              cat = v.last_use - v.def_step >= kSpillNear ? 1 : 0;
+            else if (!is_local(v.sig)) cat = 2;
+            for (int32_t t = v.def_step; t <= v.last_use; t++) livec[t][cat] += v.words();
+          }
+          int32_t best = 0;
+          double bw = 0;
+          for (int32_t t = 0; t < nsteps; t++) {
+            double w = livec[t][0] + livec[t][1] + livec[t][2] + livec[t][3];
+            if (w > bw) bw = w, best = t;
+          }
+          fprintf(stderr, "  nsteps %d peak step %d live %.0f: short %.0f long %.0f loads %.0f other %.0f\n", nsteps, best,
+                  bw, livec[best][0], livec[best][1], livec[best][2], livec[best][3]);
+        }
+        if (cand.empty() || stall >= 3 || attempt >= 24) {
+          // spilling stalls: narrow the schedule instead and start over
+          if (cap_tries >= 4 || (cap && cap <= 16)) {
+            give_up = true;   // emit as is; the limit check below reports E_NOMEM
+            if (getenv("RTLSIM_SPILL_DEBUG"))
+              fprintf(stderr, "part %u gives up: peak %u budget %u cap %u\n", p, part_peak, slot_budget, cap);
+            goto emit;
+          }
+          int32_t depth = 1;
+          for (uint32_t i : ops_p) depth = std::max(depth, op_step[i]);
+          cap = cap ? cap / 2 : std::max<uint32_t>(16, (uint32_t)(ops_p.size() / (size_t)depth / 2));
+          cap_tries++;
+          if (getenv("RTLSIM_SPILL_DEBUG"))
+            fprintf(stderr, "part %u: peak %u budget %u, step cap -> %u\n", p, part_peak, slot_budget, cap);
+          stall = 0;
+          best_peak = 0xFFFFFFFFu;
+          attempt = -1;
+          spilled.clear();
+          for (int c = 0; c < 4; c++) spill_rows[c] = 0;
+          continue;
+        }
+        std::sort(cand.rbegin(), cand.rend());
+        std::vector<uint32_t> take;
+        for (auto &cv : cand) {
+          const Value &v = vals[vid(cv.second)];
+          bool need = false;
+          for (int32_t t = v.def_step + kSpillNear; t <= v.last_use && !need; t++) need = live[t] > target;
+          if (!need) continue;
+          for (int32_t t = v.def_step + kSpillNear; t <= v.last_use; t++) live[t] -= v.words();
+          take.push_back(cv.second);
+        }
+        if (getenv("RTLSIM_SPILL_DEBUG") && getenv("RTLSIM_SPILL_DEBUG")[0] == '2')
+          fprintf(stderr, "part %u attempt %d peak %u budget %u cand %zu spilled %zu\n", p, attempt, part_peak,
+                  slot_budget, cand.size(), spilled.size());
+        for (uint32_t sg : take) {
+          if (is_xnet[sg]) {
+            spilled[sg] = xrow.at(sg);   // its cross-partition row already holds it
+          } else {
+            const uint32_t c = width_class(G.width[sg]);
+            spilled[sg] = xnet_rows[c] + spill_rows[c];
+            spill_rows[c] += (c == CLS_U32) ? nwords(G.width[sg]) : 1;
+          }
+        }
+        continue;
+      }
+    emit:
     // 7. descriptors per step
-    std::vector<StepLists> steps(nsteps);
+    steps.assign(nsteps, StepLists{});
     for (const Load &ld : loads) {
       const uint32_t s = ld.sig, w = G.width[s];
       Desc d{};
@@ -636,8 +848,11 @@ int compile_program(const rtlsim_ir *ir, uint32_t op_lanes, uint32_t smem_limit_
         d.z = (uint32_t)const_of[s];
       } else {
         code = CODE_LD_X;
-        d.z = xrow.at(s);
-        if (ld.first) {
+        d.z = row_of_x(s);
+        if (spilled.count(s) && is_local(s)) {
+          bytes_state += lane_bytes(w);
+          bytes_spill += lane_bytes(w);
+        } else if (ld.first) {
           bytes_state += lane_bytes(w);
           bytes_part += lane_bytes(w);
         }
@@ -735,9 +950,10 @@ int compile_program(const rtlsim_ir *ir, uint32_t op_lanes, uint32_t smem_limit_
         d.z = out_word[sk.idx];
         bytes_state += 4.0 * nwords(w);
       } else {
-        d.z = xrow.at(sk.idx);
+        d.z = row_of_x(sk.idx);
         bytes_state += lane_bytes(w);
-        bytes_part += lane_bytes(w);
+        if (is_xnet[sk.idx]) bytes_part += lane_bytes(w);
+        else bytes_spill += lane_bytes(w);
       }
       d.x = sk.code | (width_class(w) << 8) | (nwords(w) << 12) | (v.layout << 18);
       G.n_st++;
@@ -758,11 +974,17 @@ int compile_program(const rtlsim_ir *ir, uint32_t op_lanes, uint32_t smem_limit_
       if (!steps.empty()) steps.back().wait = 0;
     }
     // empty steps are kept (their barrier / wait depth is part of the schedule)
+      peak = std::max(peak, part_peak);
+      break;
+    }
+    for (int c = 0; c < 4; c++) max_spill_rows[c] = std::max(max_spill_rows[c], spill_rows[c]);
     for (auto &st : steps) all_steps.push_back(std::move(st));
     G.part_steps.push_back((uint32_t)all_steps.size());
     for (uint32_t s : touched) vid_of[s] = -1;
-    for (auto &kv : groups) vid_of[kv.first] = -1;
   }
+
+  for (int c = 0; c < 4; c++) G.xrows[c] = xnet_rows[c] + max_spill_rows[c];
+  G.b_spill = bytes_spill;
 
   // -------------------------------------------------------- op lanes --
   size_t total = 0;

@@ -139,7 +139,7 @@ struct Program {
   uint32_t smem_words = 0;              // shared words per tile (slots)
   // ---- stats
   uint64_t word_ops = 0, n_bitops = 0, n_wide = 0, n_narrow = 0, n_ld = 0, n_st = 0;
-  double b_floor = 0, b_state = 0, b_part = 0;
+  double b_floor = 0, b_state = 0, b_part = 0, b_spill = 0;
 };
 
 // Returns RTLSIM_OK or a negative status with *err set.

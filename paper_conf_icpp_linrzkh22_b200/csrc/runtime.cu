@@ -830,6 +830,7 @@ extern "C" int rtlsim_stats(const rtlsim_ctx *cctx, rtlsim_stats_t *st) {
   st->b_floor = G.b_floor;
   st->b_state = G.b_state;
   st->b_part = G.b_part;
+  st->b_spill = G.b_spill;
   st->rows_bit = G.rows[CLS_BIT]; st->rows_u8 = G.rows[CLS_U8];
   st->rows_u16 = G.rows[CLS_U16]; st->rows_u32 = G.rows[CLS_U32];
   st->xrows_bit = G.xrows[CLS_BIT]; st->xrows_u8 = G.xrows[CLS_U8];

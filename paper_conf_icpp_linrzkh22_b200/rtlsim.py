@@ -71,7 +71,7 @@ class Stats(ctypes.Structure):
                 ("eval_launches", ctypes.c_uint64), ("eval_stim_cycles", ctypes.c_uint64),
                 ("jit_compile_s", ctypes.c_double), ("jit_cubin_bytes", ctypes.c_uint64),
                 ("n_bitops", ctypes.c_uint64), ("n_narrow", ctypes.c_uint64), ("n_wide", ctypes.c_uint64),
-                ("n_ld", ctypes.c_uint64), ("n_st", ctypes.c_uint64)]
+                ("n_ld", ctypes.c_uint64), ("n_st", ctypes.c_uint64), ("b_spill", ctypes.c_double)]
 
 
 PRODUCER = ctypes.CFUNCTYPE(ctypes.c_int, ctypes.c_void_p, ctypes.c_uint64, ctypes.c_uint64,

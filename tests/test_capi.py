@@ -62,6 +62,25 @@ def test_shaped_configs_fit_shared_memory(R):
         assert st["op_lanes"] >= 1
 
 
+def test_smem_budget_spills_and_narrows(R):
+    """A budget below the working set: the schedule is narrowed (more steps),
+    long-lived values spill to extra cross-partition rows, the slot area fits,
+    and the spill traffic is accounted in b_state."""
+    ir = shaped.generate(3, scale=0.25)
+    free = R.Simulator(ir, flags=R.F_HOST_ONLY, op_lanes=2).stats()
+    lim = 13000
+    st = R.Simulator(ir, flags=R.F_HOST_ONLY, op_lanes=2, smem_limit=lim).stats()
+    assert free["smem_words"] * 4 > lim and free["b_spill"] == 0
+    assert st["smem_words"] * 4 <= lim and st["b_spill"] > 0
+    assert st["n_steps"] > free["n_steps"]
+    assert st["b_state"] == pytest.approx(free["b_state"] + st["b_spill"])
+    xr = lambda s: s["xrows_bit"] + s["xrows_u8"] + s["xrows_u16"] + s["xrows_u32"]
+    assert xr(st) > xr(free)
+    with pytest.raises(R.RtlsimError) as e:     # below the unspillable floor
+        R.Simulator(ir, flags=R.F_HOST_ONLY, op_lanes=2, smem_limit=2048)
+    assert e.value.code == -5
+
+
 def _expect_error(R, ir, code):
     with pytest.raises(R.RtlsimError) as e:
         _load(R, ir)

@@ -183,3 +183,19 @@ def test_pinned_host_buffers(R, oracle_lib):
     sim.N, sim.T = N, T
     R.rtlsim_run(sim.ctx, T, pout.numpy(), None, None)
     assert np.array_equal(pout.numpy().view(np.uint32), want["out"])
+
+
+@pytest.mark.parametrize("lim,lanes,flags", [(16000, 0, 0), (13000, 2, 0), (16000, 0, "jit"), (13000, 2, "jit")])
+def test_smem_budget_spill(R, oracle_lib, lim, lanes, flags):
+    """A shared-memory budget below the design's working set: the compiler
+    narrows the schedule and spills long-lived values to HBM rows; results
+    must not change (working-set budget)."""
+    ir = shaped.generate(3, scale=0.25)
+    st = stim.stimulus(ir, stim.STIM_SEED_BASE + 3, np.arange(96), 0, 20)
+    fl = R.F_JIT if flags == "jit" else 0
+    sim = R.Simulator(ir, op_lanes=lanes, smem_limit=lim, flags=fl, chunk_cycles=8)
+    s = sim.stats()
+    assert s["b_spill"] > 0 and s["smem_words"] * 4 <= lim
+    sim.bind(st)
+    got = sim.run(20, out=True, regs=True, digest=True)
+    assert_same(got, oracle_lib.simulate(ir, st, digest=True, threads=16), f"spill {lim} {lanes} {flags}")
