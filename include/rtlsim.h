@@ -116,6 +116,9 @@ typedef struct {
 #define RTLSIM_F_TIMING 0x10u     /* bracket every evaluator launch with CUDA
                                      events on the compute stream; totals in
                                      rtlsim_stats (eval_ms, eval_launches)     */
+#define RTLSIM_F_LEGACY 0x40u     /* round-1 per-descriptor interpreter instead
+                                     of the run-based micro-op evaluator (v4,
+                                     the default); kept for A/B measurement    */
 
 typedef struct {
   int device;                /* CUDA device ordinal                           */

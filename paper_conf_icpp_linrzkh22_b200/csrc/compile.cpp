@@ -74,20 +74,27 @@ struct SlotAlloc {
   std::map<uint32_t, uint32_t> free_;   // offset -> size
   uint32_t top = 0, peak = 0;
   explicit SlotAlloc(uint32_t base) : top(base), peak(base) {}
+  // slots of 4+ words start on a 16-byte boundary (16-byte cp.async row
+  // copies, program.h uop loads / stores)
   uint32_t alloc(uint32_t n) {
+    const uint32_t al = n >= 4 ? 4u : 1u;
     for (auto it = free_.begin(); it != free_.end(); ++it) {
-      if (it->second >= n) {
-        uint32_t off = it->first, sz = it->second;
+      const uint32_t off = it->first, sz = it->second;
+      const uint32_t a = (off + al - 1) & ~(al - 1);
+      if (a + n <= off + sz) {
         free_.erase(it);
-        if (sz > n) free_[off + n] = sz - n;
-        return off;
+        if (a > off) free_[off] = a - off;
+        if (a + n < off + sz) free_[a + n] = off + sz - a - n;
+        return a;
       }
     }
-    uint32_t off = top;
-    top += n;
+    const uint32_t a = (top + al - 1) & ~(al - 1);
+    if (a > top) release_raw(top, a - top);
+    top = a + n;
     peak = std::max(peak, top);
-    return off;
+    return a;
   }
+  void release_raw(uint32_t off, uint32_t n) { free_[off] = n; }
   void release(uint32_t off, uint32_t n) {
     auto it = free_.emplace(off, n).first;
     // merge with next
@@ -725,7 +732,7 @@ int compile_program(const rtlsim_ir *ir, uint32_t op_lanes, uint32_t smem_limit_
         born[vals[v].def_step].push_back((int32_t)v);
         dies[vals[v].last_use].push_back((int32_t)v);
       }
-      SlotAlloc sa(dump_words);
+      SlotAlloc sa((dump_words + 3u) & ~3u);
       for (int32_t s = 0; s < nsteps; s++) {
         // largest first keeps wide values contiguous and packs better
         std::sort(born[s].begin(), born[s].end(),
@@ -1038,6 +1045,35 @@ int compile_program(const rtlsim_ir *ir, uint32_t op_lanes, uint32_t smem_limit_
     return fail(err, RTLSIM_E_NOMEM,
                 "per-tile working set of " + std::to_string(G.smem_words * 4) +
                     " bytes exceeds the shared-memory limit of " + std::to_string(smem_limit_words * 4));
+
+  if (getenv("RTLSIM_HIST")) {   // debugging aid: descriptor class histogram
+    std::map<std::string, std::pair<uint64_t, uint64_t>> h;   // class -> (count, words)
+    const char *ln[6] = {"U32", "BIT", "U16", "U8", "IMM", "BC"};
+    for (const Desc &q : G.desc) {
+      const uint32_t code = q.x & 0xFFu;
+      char k[96];
+      if (code < 32u) {
+        const bool hb = (q.w >> 11) & 1u, hc = (q.w >> 12) & 1u;
+        snprintf(k, sizeof k, "N op%02u %s,%s,%s->%s", code, ln[(q.x >> 8) & 7u], hb ? ln[(q.x >> 11) & 7u] : "-",
+                 hc ? ln[(q.x >> 14) & 7u] : "-", ln[(q.x >> 17) & 7u]);
+        h[k].first++;
+        h[k].second++;
+      } else if (code == CODE_WIDE) {
+        const WideRec &r = G.wide[q.y];
+        snprintf(k, sizeof k, "W op%02u", r.op);
+        h[k].first++;
+        h[k].second += nwords(std::max<uint32_t>(r.wd, std::max<uint32_t>(r.wa, r.wb)));
+      } else {
+        snprintf(k, sizeof k, "M code%u cls%u", code, (q.x >> 8) & 3u);
+        h[k].first++;
+        h[k].second += (q.x >> 12) & 63u;
+      }
+    }
+    std::vector<std::pair<uint64_t, std::string>> v;
+    for (auto &kv : h) v.push_back({kv.second.first, kv.first + " words " + std::to_string(kv.second.second)});
+    std::sort(v.rbegin(), v.rend());
+    for (size_t i = 0; i < v.size() && i < 80; i++) fprintf(stderr, "%8llu %s\n", (unsigned long long)v[i].first, v[i].second.c_str());
+  }
 
   // ---------------------------------------------------------- stats --
   double bf = 0;

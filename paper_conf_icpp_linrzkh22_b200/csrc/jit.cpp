@@ -870,6 +870,10 @@ int jit_build(const Program &G, const std::string &rt_ptx_path, uint32_t smem_by
         if (G.part_steps[q] == G.part_steps[q + 1]) continue;
         std::string ptx = jit_partition_ptx(G, q, rt);
         ptx_bytes += ptx.size();
+        if (const char *dir = getenv("RTLSIM_JIT_SAVE")) {   // debugging aid: keep the module
+          std::ofstream o(fmt("%s/part%u.ptx", dir, q));
+          o << ptx;
+        }
         if (compile_ptx(ptx, o3, &cubins[q], &errs[q]) != 0 && getenv("RTLSIM_JIT_DUMP")) {
           std::ofstream o(fmt("/tmp/rtlsim_jit_fail_%u.ptx", q));
           o << ptx;

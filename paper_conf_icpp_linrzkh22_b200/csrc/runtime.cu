@@ -69,7 +69,8 @@ struct rtlsim_ctx {
   std::vector<void *> bind_allocs;    // freed at re-bind
   std::vector<void *> host_allocs;    // pinned, freed at re-bind
   // static device data
-  uint4 *d_desc = nullptr, *d_bitdesc = nullptr;
+  uint4 *d_desc = nullptr, *d_bitdesc = nullptr, *d_ustream = nullptr;
+  uint32_t *d_uptr = nullptr;
   uint32_t *d_bitptr = nullptr, *d_stepwait = nullptr;
   WideRec *d_wide = nullptr;
   uint32_t *d_step = nullptr, *d_consts = nullptr, *d_mask = nullptr, *d_reginit = nullptr;
@@ -210,8 +211,11 @@ extern "C" int rtlsim_load(const rtlsim_ir *ir, const rtlsim_options *opt, rtlsi
     return rc;
   }
   Program &G = ctx->prog;
-  // slots + one 512-byte descriptor staging buffer per op-lane warp
-  ctx->smem_bytes = desc_smem_off(G) * 4u + G.L * 512u;
+  lower_program(G);   // run-based micro-op stream (+ the zero row)
+  const bool legacy = (ctx->opt.flags & RTLSIM_F_LEGACY) != 0;
+  // legacy interpreter: slots + one 512-byte descriptor staging buffer per
+  // op-lane warp; v4: slots (micro-ops are read from L1 / L2)
+  ctx->smem_bytes = legacy ? desc_smem_off(G) * 4u + G.L * 512u : G.smem_words * 4u;
   if (ctx->smem_bytes > smem_limit) {
     g_load_error = "per-tile working set of " + std::to_string(ctx->smem_bytes) +
                    " bytes (with descriptor buffers) exceeds the shared-memory limit";
@@ -259,6 +263,12 @@ extern "C" int rtlsim_load(const rtlsim_ir *ir, const rtlsim_options *opt, rtlsi
   padded.resize(G.desc.size() + 32, Desc{});   // chunk prefetch reads up to 32 past any start
   if (e == cudaSuccess) e = up((void **)&ctx->d_desc, padded.data(), padded.size() * sizeof(Desc));
   if (e == cudaSuccess) e = up((void **)&ctx->d_bitdesc, G.bitdesc.data(), G.bitdesc.size() * sizeof(BitDesc));
+  {
+    std::vector<Desc> us(G.ustream);
+    us.resize(G.ustream.size() + 64, Desc{});   // L1 prefetch lines past the end
+    if (e == cudaSuccess) e = up((void **)&ctx->d_ustream, us.data(), us.size() * sizeof(Desc));
+  }
+  if (e == cudaSuccess) e = up((void **)&ctx->d_uptr, G.uptr.data(), G.uptr.size() * 4);
   if (e == cudaSuccess) e = up((void **)&ctx->d_bitptr, G.bit_ptr.data(), G.bit_ptr.size() * 4);
   if (e == cudaSuccess) e = up((void **)&ctx->d_stepwait, G.step_wait.data(), G.step_wait.size() * 4);
   if (e == cudaSuccess) e = up((void **)&ctx->d_wide, G.wide.data(), G.wide.size() * sizeof(WideRec));
@@ -442,7 +452,15 @@ static EvalParams eval_params(rtlsim_ctx *ctx, int b, uint64_t cycle0, uint32_t 
   p.out = ctx->d_out[b];
   p.consts = ctx->d_consts;
   p.digest = digest ? ctx->d_dig[b] : nullptr;
+  p.ustream = ctx->d_ustream;
+  p.uptr = ctx->d_uptr;
+  p.zero_off = G.zero_off;
   return p;
+}
+
+static cudaError_t evaluator(rtlsim_ctx *ctx, const EvalParams &p, cudaStream_t st) {
+  if (ctx->opt.flags & RTLSIM_F_LEGACY) return launch_eval(p, ctx->smem_bytes, st);
+  return launch_eval_v4(p, ctx->smem_bytes, st);
 }
 
 static cudaError_t get_event(rtlsim_ctx *ctx, cudaEvent_t *e) {
@@ -484,7 +502,7 @@ static int launch_chunk(rtlsim_ctx *ctx, int b, uint64_t cycle0, uint32_t nc, bo
   }
   if (!(ctx->opt.flags & (RTLSIM_F_GRAPH | RTLSIM_F_JIT))) {
     EvalParams p = eval_params(ctx, b, cycle0, nc, digest);
-    CK(launch_eval(p, ctx->smem_bytes, ctx->st));
+    CK(evaluator(ctx, p, ctx->st));
     ctx->launches++;
     if (timing) {
       CK(cudaEventRecord(tm.b, ctx->st));
@@ -542,7 +560,7 @@ static int launch_chunk(rtlsim_ctx *ctx, int b, uint64_t cycle0, uint32_t nc, bo
         p.in.u32 = ctx->d_in[b].u32 + (size_t)c * ctx->in_stride.s[CLS_U32];
         p.out = ctx->d_out[b] + (size_t)c * G.OW * ctx->N_pad;
         if (digest) p.digest = ctx->d_dig[b] + (size_t)c * ctx->N_pad;
-        cudaError_t e = launch_eval(p, ctx->smem_bytes, cap);
+        cudaError_t e = evaluator(ctx, p, cap);
         if (e != cudaSuccess) {
           cudaGraph_t g;
           cudaStreamEndCapture(cap, &g);

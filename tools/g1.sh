@@ -1,0 +1,5 @@
+nvidia-smi --query-gpu=name,clocks.sm,clocks.max.sm --format=csv > gpurun_out/g1_smi.txt; nproc >> gpurun_out/g1_smi.txt
+python -c "import __graft_entry__ as g; g.smoke()" > gpurun_out/g1_smoke.log 2>&1
+JIT=1 timeout 900 python tools/perf_probe.py 2,3,4 > gpurun_out/g1_probe_jit.log 2>&1
+timeout 600 python tools/perf_probe.py 2,3,4 > gpurun_out/g1_probe_interp.log 2>&1
+timeout 1500 python -m pytest tests -m gpu -x -q > gpurun_out/g1_pytest.log 2>&1

@@ -20,7 +20,7 @@ for cid in cfgs:
     t0 = time.time()
     import os
     jit = R.F_JIT if os.environ.get('JIT') else 0
-    sim = R.Simulator(ir, chunk_cycles=Tc, flags=R.F_TIMING | jit, op_lanes=int(os.environ.get('LANES', '0')), stream=torch.cuda.current_stream().cuda_stream)
+    sim = R.Simulator(ir, chunk_cycles=Tc, flags=R.F_TIMING | jit, op_lanes=int(os.environ.get('LANES', '0')), smem_limit=int(os.environ.get('SMEM_KB','0'))*1024, stream=torch.cuda.current_stream().cuda_stream)
     tl = time.time() - t0
     st = sim.stats()
     d_stim = stim.stimulus_torch(ir, stim.STIM_SEED_BASE + cid, 0, N, 0, T)
@@ -38,7 +38,7 @@ for cid in cfgs:
     s1 = sim.stats()
     ems = s1['eval_ms'] - s0['eval_ms']
     stc = 3 * Tc * N
-    print(json.dumps({"cfg": cid, "gen_s": round(tg,1), "load_s": round(tl,2), "L": st['op_lanes'], "smem_KB": st['smem_words']*4/1024,
+    print(json.dumps({"cfg": cid, "env": {k: os.environ.get(k) for k in ("JIT","LANES","SMEM_KB","RTLSIM_JIT_OPT")}, "gen_s": round(tg,1), "load_s": round(tl,2), "L": st['op_lanes'], "smem_KB": st['smem_words']*4/1024,
           "steps": st['n_steps'], "desc": st['n_desc'], "b_floor": st['b_floor'], "b_state": st['b_state'],
           "ms_per_cycle_total": ms / (3*Tc), "ms_per_cycle_eval": ems / (3*Tc),
           "stim_cyc_per_s": stc / (ms/1e3), "eval_GBps_floor": st['b_floor'] * stc / (ems/1e3) / 1e9}))
