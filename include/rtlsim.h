@@ -116,9 +116,13 @@ typedef struct {
 #define RTLSIM_F_TIMING 0x10u     /* bracket every evaluator launch with CUDA
                                      events on the compute stream; totals in
                                      rtlsim_stats (eval_ms, eval_launches)     */
-#define RTLSIM_F_LEGACY 0x40u     /* round-1 per-descriptor interpreter instead
-                                     of the run-based micro-op evaluator (v4,
-                                     the default); kept for A/B measurement    */
+#define RTLSIM_F_STREAM 0x80u     /* ablation (Table 4): the per-(cycle,
+                                     partition) launches of graph mode issued
+                                     one by one into the stream, no graph     */
+#define RTLSIM_F_V4 0x40u         /* run-based micro-op evaluator (lower.cpp +
+                                     rtl_eval_v4) instead of the per-descriptor
+                                     interpreter; measured slower on configs
+                                     3-4 (run-dispatch overhead), kept for A/B */
 
 typedef struct {
   int device;                /* CUDA device ordinal                           */

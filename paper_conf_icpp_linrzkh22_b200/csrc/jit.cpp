@@ -736,7 +736,7 @@ std::string step_function(const Program &G, const std::string &name, uint32_t s0
 
 }  // namespace
 
-std::string jit_partition_ptx(const Program &G, uint32_t q, const std::string &rt_ptx) {
+std::string jit_partition_ptx(const Program &G, uint32_t q, const std::string &rt_ptx, uint32_t tmax) {
   const uint32_t s0 = G.part_steps[q], s1 = G.part_steps[q + 1];
   std::string mod;
   mod.reserve(1 << 20);
@@ -759,13 +759,18 @@ std::string jit_partition_ptx(const Program &G, uint32_t q, const std::string &r
   for (size_t g = 0; g < groups.size(); g++)
     mod += step_function(G, fmt("rtl_steps_%zu", g), groups[g].first, groups[g].second) + "\n";
   // the kernel: per-thread context, then the step functions in order
+  // A CTA holds `tpc` tiles; warp g works on tile g / L as op-lane g % L, so
+  // the warps of one op-lane (one per tile) run identical code in step
+  // lock-step and share its instruction fetch.
   mod += fmt(".visible .entry rtl_jit_part(.param .align 8 .b8 prm[%zu])\n.maxntid %u, 1, 1\n{\n",
-             sizeof(JitParams), 32u * G.L);
-  mod += "\t.reg .b32 %tidx, %tile, %s, %smb, %lane, %wl, %N;\n\t.reg .b64 %t64, %b64, %digb;\n\t.reg .pred %pz;\n\t.reg .b64 ";
+             sizeof(JitParams), 32u * G.L * std::max<uint32_t>(tmax, 1u));
+  mod += "\t.reg .b32 %tidx, %tile, %s, %smb, %lane, %wl, %N, %wg, %tsub, %tpc;\n\t.reg .b64 %t64, %b64, %digb;\n\t.reg .pred %pz;\n\t.reg .b64 ";
   for (int i = 0; i < kN64; i++) mod += fmt("%s%%%s", i ? ", " : "", kCtx64[i]);
   mod += ";\n";
-  mod += "\tmov.u32 %tidx, %tid.x;\n\tand.b32 %lane, %tidx, 31;\n\tshr.u32 %wl, %tidx, 5;\n\tmov.u32 %tile, %ctaid.x;\n"
-         "\tmad.lo.u32 %s, %tile, 32, %lane;\n";
+  mod += fmt("\tmov.u32 %%tidx, %%tid.x;\n\tand.b32 %%lane, %%tidx, 31;\n\tshr.u32 %%wg, %%tidx, 5;\n"
+             "\trem.u32 %%wl, %%wg, %u;\n\tdiv.u32 %%tsub, %%wg, %u;\n", G.L, G.L);
+  mod += fmt("\tld.param.u32 %%tpc, [prm+%zu];\n", offsetof(JitParams, tpc));
+  mod += "\tmov.u32 %tile, %ctaid.x;\n\tmad.lo.u32 %tile, %tile, %tpc, %tsub;\n\tmad.lo.u32 %s, %tile, 32, %lane;\n";
   mod += fmt("\tld.param.u32 %%N, [prm+%zu];\n", offsetof(JitParams, N));
   const size_t aoff[4] = {offsetof(JitParams, cur), offsetof(JitParams, nxt), offsetof(JitParams, xnet),
                           offsetof(JitParams, in)};
@@ -785,7 +790,9 @@ std::string jit_partition_ptx(const Program &G, uint32_t q, const std::string &r
              "\tsetp.eq.u64 %%pz, %%digb, 0;\n\tselp.b64 %%dig, 0, %%t64, %%pz;\n",
              offsetof(JitParams, digest));
   mod += fmt("\tld.param.u64 %%wide, [prm+%zu];\n", offsetof(JitParams, wide));
-  mod += "\tmov.u32 %smb, dyn_smem;\n\tcvta.shared.u64 %smg, dyn_smem;\n";
+  mod += fmt("\tmov.u32 %%smb, dyn_smem;\n\tmad.lo.u32 %%smb, %%tsub, %u, %%smb;\n\tcvta.shared.u64 %%smg, dyn_smem;\n"
+             "\tmul.wide.u32 %%t64, %%tsub, %u;\n\tadd.u64 %%smg, %%smg, %%t64;\n",
+             jit_tile_bytes(G), jit_tile_bytes(G));
   for (size_t g = 0; g < groups.size(); g++) {
     mod += "\t{\n";
     std::string args;
@@ -848,6 +855,9 @@ int jit_build(const Program &G, const std::string &rt_ptx_path, uint32_t smem_by
     rt += line + "\n";
   }
   const uint32_t NP = (uint32_t)G.part_steps.size() - 1;
+  // tiles per CTA the kernels are built for (their thread count bounds registers)
+  const uint32_t tmax = std::max<uint32_t>(1u, std::min<uint32_t>(kJitMaxTiles, smem_bytes / jit_tile_bytes(G)));
+  out->tmax = tmax;
   // ptxas -O3 schedules this code ~1.8x better (config 3) but compiles ~3x
   // slower than --Ofast-compile=mid: use it unless the design is large
   // (RTLSIM_JIT_OPT=O3 / mid overrides)
@@ -868,7 +878,7 @@ int jit_build(const Program &G, const std::string &rt_ptx_path, uint32_t smem_by
     th.emplace_back([&]() {
       for (uint32_t q; (q = next++) < NP;) {
         if (G.part_steps[q] == G.part_steps[q + 1]) continue;
-        std::string ptx = jit_partition_ptx(G, q, rt);
+        std::string ptx = jit_partition_ptx(G, q, rt, tmax);
         ptx_bytes += ptx.size();
         if (const char *dir = getenv("RTLSIM_JIT_SAVE")) {   // debugging aid: keep the module
           std::ofstream o(fmt("%s/part%u.ptx", dir, q));

@@ -26,20 +26,26 @@ struct JitParams {
   uint64_t digest;                           // digest row of this cycle [N_pad] u64, or 0
   uint64_t wide;                             // WideRec array (generic path)
   uint32_t N;                                // N_pad
-  uint32_t pad;
+  uint32_t tpc;                              // 32-stimulus tiles per CTA (warps of equal op-lane share code)
 };
 static_assert(sizeof(JitParams) == 160, "JitParams layout is hard-coded in the PTX generator");
+
+// Maximum tiles per CTA the kernels are compiled for (.maxntid 32 * L * kJitMaxTiles).
+constexpr uint32_t kJitMaxTiles = 2;
+// Bytes of shared memory per tile in a JIT CTA (16-byte aligned).
+inline uint32_t jit_tile_bytes(const Program &G) { return ((G.smem_words * 4u) + 15u) & ~15u; }
 
 struct JitKernels {
   std::vector<cudaLibrary_t> libs;
   std::vector<cudaKernel_t> kern;   // per exec-order partition (nullptr: empty partition)
   double gen_s = 0, compile_s = 0;
   bool o3 = false;
+  uint32_t tmax = 1;                // tiles per CTA the kernels were built for
   size_t ptx_bytes = 0, cubin_bytes = 0;
 };
 
 // PTX text of exec-order partition q (steps part_steps[q]..part_steps[q+1]).
-std::string jit_partition_ptx(const Program &G, uint32_t q, const std::string &rt_ptx);
+std::string jit_partition_ptx(const Program &G, uint32_t q, const std::string &rt_ptx, uint32_t tmax);
 // Generate + compile (nvPTXCompiler, all host cores) + load every partition.
 // device < 0: generate and compile only (host-only contexts, CPU tests).
 int jit_build(const Program &G, const std::string &rt_ptx_path, uint32_t smem_bytes, int device, JitKernels *out,

@@ -212,7 +212,7 @@ extern "C" int rtlsim_load(const rtlsim_ir *ir, const rtlsim_options *opt, rtlsi
   }
   Program &G = ctx->prog;
   lower_program(G);   // run-based micro-op stream (+ the zero row)
-  const bool legacy = (ctx->opt.flags & RTLSIM_F_LEGACY) != 0;
+  const bool legacy = (ctx->opt.flags & RTLSIM_F_V4) == 0;
   // legacy interpreter: slots + one 512-byte descriptor staging buffer per
   // op-lane warp; v4: slots (micro-ops are read from L1 / L2)
   ctx->smem_bytes = legacy ? desc_smem_off(G) * 4u + G.L * 512u : G.smem_words * 4u;
@@ -230,9 +230,10 @@ extern "C" int rtlsim_load(const rtlsim_ir *ir, const rtlsim_options *opt, rtlsi
       dir = info.dli_fname;
       dir = dir.substr(0, dir.find_last_of('/'));
     }
-    ctx->jit_smem = std::max<uint32_t>(G.smem_words * 4u, 16u);
+    ctx->jit_smem = std::max<uint32_t>(jit_tile_bytes(G), 16u);
     std::string jerr;
-    int jr = jit_build(G, dir + "/jit_rt.ptx", ctx->jit_smem, device, &ctx->jit, &jerr);
+    int jr = jit_build(G, dir + "/jit_rt.ptx", std::min<uint32_t>(ctx->jit_smem * kJitMaxTiles, smem_limit), device,
+                       &ctx->jit, &jerr);
     if (jr != RTLSIM_OK) g_load_error = "JIT: " + jerr;
     return jr;
   };
@@ -458,9 +459,23 @@ static EvalParams eval_params(rtlsim_ctx *ctx, int b, uint64_t cycle0, uint32_t 
   return p;
 }
 
+// JIT: tiles per CTA — as many as the shared memory holds (up to the count
+// the kernels were compiled for) that divide the tile count; env override
+// RTLSIM_JIT_TPC for measurements
+static uint32_t jit_tiles_per_cta(rtlsim_ctx *ctx) {
+  const uint32_t tiles = ctx->N_pad / 32u;
+  int optin = 232448;
+  cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, ctx->device);
+  uint32_t m = std::min<uint32_t>(ctx->jit.tmax, (uint32_t)optin / std::max<uint32_t>(ctx->jit_smem, 1u));
+  if (const char *e = getenv("RTLSIM_JIT_TPC")) m = std::min<uint32_t>(m, (uint32_t)atoi(e));
+  m = std::max<uint32_t>(m, 1u);
+  while (m > 1 && tiles % m) m--;
+  return m;
+}
+
 static cudaError_t evaluator(rtlsim_ctx *ctx, const EvalParams &p, cudaStream_t st) {
-  if (ctx->opt.flags & RTLSIM_F_LEGACY) return launch_eval(p, ctx->smem_bytes, st);
-  return launch_eval_v4(p, ctx->smem_bytes, st);
+  if (ctx->opt.flags & RTLSIM_F_V4) return launch_eval_v4(p, ctx->smem_bytes, st);
+  return launch_eval(p, ctx->smem_bytes, st);
 }
 
 static cudaError_t get_event(rtlsim_ctx *ctx, cudaEvent_t *e) {
@@ -500,7 +515,7 @@ static int launch_chunk(rtlsim_ctx *ctx, int b, uint64_t cycle0, uint32_t nc, bo
     CK(get_event(ctx, &tm.b));
     CK(cudaEventRecord(tm.a, ctx->st));
   }
-  if (!(ctx->opt.flags & (RTLSIM_F_GRAPH | RTLSIM_F_JIT))) {
+  if (!(ctx->opt.flags & (RTLSIM_F_GRAPH | RTLSIM_F_JIT | RTLSIM_F_STREAM))) {
     EvalParams p = eval_params(ctx, b, cycle0, nc, digest);
     CK(evaluator(ctx, p, ctx->st));
     ctx->launches++;
@@ -511,18 +526,13 @@ static int launch_chunk(rtlsim_ctx *ctx, int b, uint64_t cycle0, uint32_t nc, bo
     return RTLSIM_OK;
   }
   const bool jit = (ctx->opt.flags & RTLSIM_F_JIT) != 0;
-  // graph mode (and JIT mode): Tc x P per-(cycle, partition) nodes, captured
-  // once per (buffer, parity, nc, digest) and replayed
-  const uint64_t key = ((uint64_t)nc << 8) | ((uint64_t)b << 2) | ((cycle0 & 1ull) << 1) | (digest ? 1u : 0u);
-  auto it = ctx->graphs.find(key);
-  if (it == ctx->graphs.end()) {
-    cudaStream_t cap;
-    CK(cudaStreamCreateWithFlags(&cap, cudaStreamNonBlocking));
-    CK(cudaStreamBeginCapture(cap, cudaStreamCaptureModeThreadLocal));
+  // Tc x P per-(cycle, partition) kernel nodes (graph / JIT / stream modes)
+  auto issue = [&](cudaStream_t cap) -> cudaError_t {
     const uint32_t NP = (uint32_t)G.part_steps.size() - 1;
     for (uint32_t c = 0; c < nc; c++) {
       for (uint32_t q = 0; q < NP; q++) {
         if (G.part_steps[q] == G.part_steps[q + 1]) continue;
+        cudaError_t e;
         if (jit) {
           if (!ctx->jit.kern[q]) continue;
           const uint32_t par = (uint32_t)(((cycle0 & 1ull) + c) & 1ull);
@@ -541,35 +551,51 @@ static int launch_chunk(rtlsim_ctx *ctx, int b, uint64_t cycle0, uint32_t nc, bo
           jp.digest = digest ? (uint64_t)(ctx->d_dig[b] + (size_t)c * ctx->N_pad) : 0;
           jp.wide = (uint64_t)ctx->d_wide;
           jp.N = ctx->N_pad;
+          jp.tpc = jit_tiles_per_cta(ctx);
           void *args[] = {&jp};
-          cudaError_t e = cudaLaunchKernel((const void *)ctx->jit.kern[q], dim3(ctx->N_pad / 32u), dim3(32u * G.L),
-                                           args, ctx->jit_smem, cap);
-          if (e != cudaSuccess) {
-            cudaGraph_t g;
-            cudaStreamEndCapture(cap, &g);
-            return cuda_fail(ctx, e, "JIT graph capture", __LINE__);
-          }
-          continue;
+          e = cudaLaunchKernel((const void *)ctx->jit.kern[q], dim3(ctx->N_pad / 32u / jp.tpc),
+                               dim3(32u * G.L * jp.tpc), args, ctx->jit_smem * jp.tpc, cap);
+        } else {
+          EvalParams p = eval_params(ctx, b, (cycle0 & 1ull) + c, 1, digest);
+          p.step_begin = G.part_steps[q];
+          p.step_end = G.part_steps[q + 1];
+          p.in.bit = ctx->d_in[b].bit + (size_t)c * ctx->in_stride.s[CLS_BIT];
+          p.in.u8 = ctx->d_in[b].u8 + (size_t)c * ctx->in_stride.s[CLS_U8];
+          p.in.u16 = ctx->d_in[b].u16 + (size_t)c * ctx->in_stride.s[CLS_U16];
+          p.in.u32 = ctx->d_in[b].u32 + (size_t)c * ctx->in_stride.s[CLS_U32];
+          p.out = ctx->d_out[b] + (size_t)c * G.OW * ctx->N_pad;
+          if (digest) p.digest = ctx->d_dig[b] + (size_t)c * ctx->N_pad;
+          e = evaluator(ctx, p, cap);
         }
-        EvalParams p = eval_params(ctx, b, (cycle0 & 1ull) + c, 1, digest);
-        p.step_begin = G.part_steps[q];
-        p.step_end = G.part_steps[q + 1];
-        p.in.bit = ctx->d_in[b].bit + (size_t)c * ctx->in_stride.s[CLS_BIT];
-        p.in.u8 = ctx->d_in[b].u8 + (size_t)c * ctx->in_stride.s[CLS_U8];
-        p.in.u16 = ctx->d_in[b].u16 + (size_t)c * ctx->in_stride.s[CLS_U16];
-        p.in.u32 = ctx->d_in[b].u32 + (size_t)c * ctx->in_stride.s[CLS_U32];
-        p.out = ctx->d_out[b] + (size_t)c * G.OW * ctx->N_pad;
-        if (digest) p.digest = ctx->d_dig[b] + (size_t)c * ctx->N_pad;
-        cudaError_t e = evaluator(ctx, p, cap);
-        if (e != cudaSuccess) {
-          cudaGraph_t g;
-          cudaStreamEndCapture(cap, &g);
-          return cuda_fail(ctx, e, "graph capture", __LINE__);
-        }
+        if (e != cudaSuccess) return e;
       }
     }
+    return cudaSuccess;
+  };
+  if (ctx->opt.flags & RTLSIM_F_STREAM) {
+    // the paper's stream-based baseline (Table 4): the same per-(cycle,
+    // partition) launches issued one by one every chunk, no graph
+    CK(issue(ctx->st));
+    ctx->launches += (uint64_t)nc * (G.part_steps.size() - 1);
+    if (timing) {
+      CK(cudaEventRecord(tm.b, ctx->st));
+      ctx->timed_pending.push_back(tm);
+    }
+    return RTLSIM_OK;
+  }
+  // graph mode (and JIT mode): captured once per (buffer, parity, nc, digest)
+  // and replayed
+  const uint64_t key = ((uint64_t)nc << 8) | ((uint64_t)b << 2) | ((cycle0 & 1ull) << 1) | (digest ? 1u : 0u);
+  auto it = ctx->graphs.find(key);
+  if (it == ctx->graphs.end()) {
+    cudaStream_t cap;
+    CK(cudaStreamCreateWithFlags(&cap, cudaStreamNonBlocking));
+    CK(cudaStreamBeginCapture(cap, cudaStreamCaptureModeThreadLocal));
+    cudaError_t e = issue(cap);
     cudaGraph_t g;
-    CK(cudaStreamEndCapture(cap, &g));
+    cudaError_t e2 = cudaStreamEndCapture(cap, &g);
+    if (e != cudaSuccess) return cuda_fail(ctx, e, "graph capture", __LINE__);
+    CK(e2);
     cudaGraphExec_t ge;
     CK(cudaGraphInstantiate(&ge, g, 0));
     CK(cudaGraphDestroy(g));

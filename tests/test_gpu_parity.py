@@ -122,6 +122,7 @@ def test_modes_agree(R, oracle_lib):
     st = stim.stimulus(ir, 21, np.arange(70), 0, 33)
     want = oracle_lib.simulate(ir, st, digest=True, threads=8)
     for opt in (dict(flags=R.F_GRAPH, chunk_cycles=8), dict(flags=R.F_NO_PIPELINE), dict(op_lanes=1),
+                dict(flags=R.F_STREAM, chunk_cycles=6), dict(flags=R.F_V4, chunk_cycles=9), dict(flags=R.F_V4 | R.F_GRAPH, chunk_cycles=4),
                 dict(op_lanes=7, chunk_cycles=5), dict(flags=R.F_GRAPH | R.F_NO_PIPELINE, chunk_cycles=33)):
         assert_same(gpu_run(R, ir, st, **opt), want, str(opt))
 
@@ -199,3 +200,24 @@ def test_smem_budget_spill(R, oracle_lib, lim, lanes, flags):
     sim.bind(st)
     got = sim.run(20, out=True, regs=True, digest=True)
     assert_same(got, oracle_lib.simulate(ir, st, digest=True, threads=16), f"spill {lim} {lanes} {flags}")
+
+
+@pytest.mark.parametrize("tpc", ["1", "2"])
+def test_jit_tiles_per_cta(R, oracle_lib, tpc, monkeypatch):
+    """JIT CTAs holding several 32-stimulus tiles (warps of one op-lane share
+    code): results do not depend on the tiles-per-CTA choice."""
+    monkeypatch.setenv("RTLSIM_JIT_TPC", tpc)
+    ir = designs.random_dag(777, n_ops=300, n_regs=24, n_partitions=3, input_widths=(7, 33, 1, 64, 100),
+                            max_width=1024)
+    st = stim.stimulus(ir, 19, np.arange(256), 0, 21, mask=False)
+    assert_same(gpu_run(R, ir, st, chunk_cycles=8, flags=R.F_JIT),
+                oracle_lib.simulate(ir, st, digest=True, threads=8), f"jit tpc{tpc}")
+
+
+@pytest.mark.parametrize("cid,scale,N,T", [(2, 1.0, 256, 30), (3, 0.25, 160, 16), (4, 0.02, 96, 8)])
+def test_v4_shaped_reduced(R, oracle_lib, cid, scale, N, T):
+    """The run-based micro-op evaluator (RTLSIM_F_V4) on the shaped designs."""
+    ir = shaped.generate(cid, scale=scale)
+    st = stim.stimulus(ir, stim.STIM_SEED_BASE + cid, np.arange(N), 0, T)
+    assert_same(gpu_run(R, ir, st, chunk_cycles=16, flags=R.F_V4),
+                oracle_lib.simulate(ir, st, digest=True, threads=16), f"v4 config{cid}@{scale}")
