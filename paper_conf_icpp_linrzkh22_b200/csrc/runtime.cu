@@ -210,9 +210,31 @@ extern "C" int rtlsim_load(const rtlsim_ir *ir, const rtlsim_options *opt, rtlsi
     delete ctx;
     return rc;
   }
+  const bool legacy = (ctx->opt.flags & RTLSIM_F_V4) == 0;
+  // bytes after lowering: slots, the 32-word zero row (lower_program) and,
+  // for the interpreter, one 512-byte descriptor staging buffer per op-lane
+  auto final_bytes = [&](const Program &P) {
+    uint32_t w = ((P.smem_words + 3u) & ~3u) + 32u;
+    return (legacy ? ((w + 3u) & ~3u) * 4u + P.L * 512u : w * 4u);
+  };
+  if (final_bytes(ctx->prog) > smem_limit) {
+    // these come out of the same budget: recompile the slot area against
+    // what is left
+    const uint32_t L = ctx->prog.L, reserve = (legacy ? L * 512u : 0u) + 160u;
+    if (smem_limit > reserve) {
+      rtlsim::Program again;
+      std::string e2;
+      rc = compile_program(ir, L, (smem_limit - reserve) / 4u, &again, &e2);
+      if (rc != RTLSIM_OK) {
+        g_load_error = e2;
+        delete ctx;
+        return rc;
+      }
+      ctx->prog = std::move(again);
+    }
+  }
   Program &G = ctx->prog;
   lower_program(G);   // run-based micro-op stream (+ the zero row)
-  const bool legacy = (ctx->opt.flags & RTLSIM_F_V4) == 0;
   // legacy interpreter: slots + one 512-byte descriptor staging buffer per
   // op-lane warp; v4: slots (micro-ops are read from L1 / L2)
   ctx->smem_bytes = legacy ? desc_smem_off(G) * 4u + G.L * 512u : G.smem_words * 4u;
