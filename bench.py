@@ -297,7 +297,9 @@ def run_ours(a):
                 "l2": f"register state {st['b_floor'] * N / 2 / 1e9:.1f} GB per buffer >> 126 MB L2 (no flush needed)",
             },
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
-                         "frac": achieved / peak, "traffic": traffic, "kernel": "rtl_eval_kernel",
+                         "frac": achieved / peak, "traffic": traffic,
+                         "kernel": "rtl_jit_part (one per partition per cycle)" if a.backend == "jit"
+                                   else "rtl_eval_kernel",
                          "peak_source": peak_src,
                          "algorithmic_bytes_per_stim_cycle": st["b_floor"],
                          "eval_ms_per_launch": avg_ms, "eval_share_of_step": ev_ms / max(ms, 1e-9)},

@@ -231,9 +231,12 @@ class Simulator:
         self.N = self.T = 0
         self._keep = None
 
-    def __del__(self):
+    def __del__(self, _free=rtlsim_free):
         if getattr(self, "ctx", None):
-            rtlsim_free(self.ctx)
+            try:
+                _free(self.ctx)
+            except Exception:   # interpreter shutdown: the process frees it
+                pass
             self.ctx = None
 
     def stats(self) -> dict:
