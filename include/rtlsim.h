@@ -123,6 +123,11 @@ typedef struct {
                                      rtl_eval_v4) instead of the per-descriptor
                                      interpreter; measured slower on configs
                                      3-4 (run-dispatch overhead), kept for A/B */
+#define RTLSIM_F_NO_DCE 0x100u    /* ablation: keep dead logic. By default ops
+                                     whose value reaches no register D, no
+                                     output and no live op are not evaluated
+                                     (unobservable; Verilator's dead-code
+                                     elimination)      */
 
 typedef struct {
   int device;                /* CUDA device ordinal                           */
@@ -157,6 +162,8 @@ typedef struct {
   uint64_t n_bitops, n_narrow, n_wide, n_ld, n_st;   /* op stream composition    */
   double b_spill;            /* of b_state: spill stores + reloads of values that
                                 exceed the smem budget (options.smem_limit) */
+  uint64_t n_live_ops;       /* ops evaluated per cycle (n_ops minus dead logic) */
+  uint64_t live_word_ops;    /* word_ops of the live ops                       */
 } rtlsim_stats_t;
 
 typedef struct rtlsim_ctx rtlsim_ctx;

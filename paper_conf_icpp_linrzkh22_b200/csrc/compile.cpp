@@ -152,7 +152,7 @@ static uint32_t fast_handler(uint32_t opc, int ar, const uint32_t *lay, uint32_t
 }
 
 int compile_program(const rtlsim_ir *ir, uint32_t op_lanes, uint32_t smem_limit_words, Program *P,
-                    std::string *err) {
+                    std::string *err, bool dce) {
   if (!ir || !P) return fail(err, RTLSIM_E_ARG, "NULL ir");
   const uint32_t n = ir->n_signals;
   if (n == 0 || !ir->width || !ir->kind) return fail(err, RTLSIM_E_IR, "no signals");
@@ -279,6 +279,36 @@ int compile_program(const rtlsim_ir *ir, uint32_t op_lanes, uint32_t smem_limit_
     if (topo.size() != G.n_ops) return fail(err, RTLSIM_E_COMB_LOOP, "combinational loop among ops");
   }
 
+  // ---------------------------------------------- dead-logic elimination --
+  // Full-cycle simulation evaluates every node, but the only
+  // observables are the outputs and the register state: an op
+  // whose value reaches no register D, no output and no live op cannot change
+  // either, so it is not scheduled (the RTL front end the paper builds on,
+  // Verilator, removes such logic before code generation).
+  // RTLSIM_F_NO_DCE keeps it (ablation; results are identical either way).
+  std::vector<char> live(G.n_ops, 1);
+  if (dce) {
+    std::vector<char> need(n, 0);
+    for (uint32_t r = 0; r < ir->n_regs; r++) need[G.reg_d[r]] = 1;
+    for (uint32_t o = 0; o < ir->n_outputs; o++) need[G.output_sig[o]] = 1;
+    for (auto it = topo.rbegin(); it != topo.rend(); ++it) {
+      const rtlsim_op &o = G.ops[*it];
+      live[*it] = need[o.dst];
+      if (!live[*it]) continue;
+      uint32_t src[3] = {o.a, o.b, o.c};
+      for (int k = 0; k < arity(o.opcode); k++) need[src[k]] = 1;
+    }
+    topo.erase(std::remove_if(topo.begin(), topo.end(), [&](uint32_t i) { return !live[i]; }), topo.end());
+  }
+  G.n_live_ops = topo.size();
+  for (uint32_t i = 0; i < G.n_ops; i++) {   // algorithmic word-ops of the whole design
+    const rtlsim_op &o = G.ops[i];
+    uint32_t wmax = G.width[o.dst];
+    if (arity(o.opcode) >= 1) wmax = std::max<uint32_t>(wmax, G.width[o.a]);
+    if (arity(o.opcode) >= 2) wmax = std::max<uint32_t>(wmax, G.width[o.b]);
+    G.word_ops += nwords(wmax);
+  }
+
   // ---------------------------------------------------- partition order --
   const uint32_t NP = G.n_partitions;
   std::vector<uint32_t> porder;
@@ -286,7 +316,7 @@ int compile_program(const rtlsim_ir *ir, uint32_t op_lanes, uint32_t smem_limit_
     std::vector<std::vector<uint32_t>> succ(NP);
     std::vector<uint32_t> indeg(NP, 0);
     std::vector<std::vector<char>> seen(NP);
-    for (uint32_t i = 0; i < G.n_ops; i++) {
+    for (uint32_t i = 0; i < G.n_ops; i++) {   // the IR's partition DAG, dead logic included (validation)
       const rtlsim_op &o = G.ops[i];
       uint32_t src[3] = {o.a, o.b, o.c};
       for (int k = 0; k < arity(o.opcode); k++)
@@ -347,7 +377,7 @@ int compile_program(const rtlsim_ir *ir, uint32_t op_lanes, uint32_t smem_limit_
 
   // cross-partition nets
   std::vector<char> is_xnet(n, 0);
-  for (uint32_t i = 0; i < G.n_ops; i++) {
+  for (uint32_t i : topo) {
     const rtlsim_op &o = G.ops[i];
     uint32_t src[3] = {o.a, o.b, o.c};
     for (int k = 0; k < arity(o.opcode); k++)
@@ -377,14 +407,14 @@ int compile_program(const rtlsim_ir *ir, uint32_t op_lanes, uint32_t smem_limit_
   uint32_t dump_words = 0;
   {
     std::vector<char> used(n, 0);
-    for (uint32_t i = 0; i < G.n_ops; i++) {
+    for (uint32_t i : topo) {
       const rtlsim_op &o = G.ops[i];
       uint32_t src[3] = {o.a, o.b, o.c};
       for (int k = 0; k < arity(o.opcode); k++) used[src[k]] = 1;
     }
     for (uint32_t r = 0; r < ir->n_regs; r++) used[G.reg_d[r]] = 1;
     for (uint32_t o = 0; o < ir->n_outputs; o++) used[G.output_sig[o]] = 1;
-    for (uint32_t i = 0; i < G.n_ops; i++) {
+    for (uint32_t i : topo) {
       uint32_t d = G.ops[i].dst;
       if (!used[d]) dump_words = std::max(dump_words, slot_words(value_layout(G.width[d], false), G.width[d]));
     }
@@ -439,14 +469,14 @@ int compile_program(const rtlsim_ir *ir, uint32_t op_lanes, uint32_t smem_limit_
     uint32_t best_peak = 0xFFFFFFFFu;
     bool give_up = false;
     const size_t wide_base = G.wide.size();
-    const auto snap = std::make_tuple(G.word_ops, G.n_bitops, G.n_narrow, G.n_wide, G.n_ld, G.n_st, bytes_state,
+    const auto snap = std::make_tuple(G.live_word_ops, G.n_bitops, G.n_narrow, G.n_wide, G.n_ld, G.n_st, bytes_state,
                                       bytes_part, bytes_spill);
     for (int attempt = 0;; attempt++) {
       for (uint32_t s2 : touched) vid_of[s2] = -1;
       touched.clear();
       vals.clear();
       G.wide.resize(wide_base);
-      std::tie(G.word_ops, G.n_bitops, G.n_narrow, G.n_wide, G.n_ld, G.n_st, bytes_state, bytes_part, bytes_spill) =
+      std::tie(G.live_word_ops, G.n_bitops, G.n_narrow, G.n_wide, G.n_ld, G.n_st, bytes_state, bytes_part, bytes_spill) =
           snap;
       // 1. levels of the partition's own ops (ASAP)
       op_step.clear();
@@ -879,7 +909,7 @@ int compile_program(const rtlsim_ir *ir, uint32_t op_lanes, uint32_t smem_limit_
       }
       uint32_t wmax = D.width;
       for (int k = 0; k < std::min(ar, 2); k++) wmax = std::max(wmax, vals[src[k]].width);
-      G.word_ops += nwords(wmax);
+      G.live_word_ops += nwords(wmax);
       if (allbit) {
         BitDesc b{};
         uint32_t f[3] = {0, 0, 0}, immf = 0;

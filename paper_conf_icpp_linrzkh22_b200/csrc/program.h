@@ -204,6 +204,7 @@ struct Program {
   // ---- stats
   uint64_t word_ops = 0, n_bitops = 0, n_wide = 0, n_narrow = 0, n_ld = 0, n_st = 0;
   double b_floor = 0, b_state = 0, b_part = 0, b_spill = 0;
+  uint64_t n_live_ops = 0, live_word_ops = 0;
 };
 
 // Lower the descriptor schedule of a compiled Program into the run-based
@@ -215,7 +216,7 @@ bool unrolled(uint32_t cls);
 
 // Returns RTLSIM_OK or a negative status with *err set.
 int compile_program(const rtlsim_ir *ir, uint32_t op_lanes, uint32_t smem_limit_words, Program *out,
-                    std::string *err);
+                    std::string *err, bool dce = true);
 
 // 3-input truth table (bit k = f(a = k&1, b = k>>1&1, c = k>>2&1)) of an IR
 // opcode on 1-bit operands and a 1-bit result.

@@ -196,13 +196,14 @@ extern "C" int rtlsim_load(const rtlsim_ir *ir, const rtlsim_options *opt, rtlsi
   // JIT kernels are instruction-fetch bound: fewer, longer per-warp code runs
   // measure faster (config 3: 8 op-lanes 1.9 ms/cycle vs 16: 3.5 ms)
   uint32_t lanes = ctx->opt.op_lanes;
+  const bool dce = (ctx->opt.flags & RTLSIM_F_NO_DCE) == 0;
   if (!lanes && (ctx->opt.flags & RTLSIM_F_JIT)) lanes = kJitMaxLanes;
-  int rc = compile_program(ir, lanes, smem_limit / 4u, &ctx->prog, &err);
+  int rc = compile_program(ir, lanes, smem_limit / 4u, &ctx->prog, &err, dce);
   if (rc == RTLSIM_OK && !ctx->opt.op_lanes && (ctx->opt.flags & RTLSIM_F_JIT) && ctx->prog.L > 1) {
     // keep the auto choice when it is smaller than the cap
     rtlsim::Program probe;
     std::string e2;
-    if (compile_program(ir, 0, smem_limit / 4u, &probe, &e2) == RTLSIM_OK && probe.L < ctx->prog.L)
+    if (compile_program(ir, 0, smem_limit / 4u, &probe, &e2, dce) == RTLSIM_OK && probe.L < ctx->prog.L)
       ctx->prog = std::move(probe);
   }
   if (rc != RTLSIM_OK) {
@@ -224,7 +225,7 @@ extern "C" int rtlsim_load(const rtlsim_ir *ir, const rtlsim_options *opt, rtlsi
     if (smem_limit > reserve) {
       rtlsim::Program again;
       std::string e2;
-      rc = compile_program(ir, L, (smem_limit - reserve) / 4u, &again, &e2);
+      rc = compile_program(ir, L, (smem_limit - reserve) / 4u, &again, &e2, dce);
       if (rc != RTLSIM_OK) {
         g_load_error = e2;
         delete ctx;
@@ -897,6 +898,8 @@ extern "C" int rtlsim_stats(const rtlsim_ctx *cctx, rtlsim_stats_t *st) {
   st->b_state = G.b_state;
   st->b_part = G.b_part;
   st->b_spill = G.b_spill;
+  st->n_live_ops = G.n_live_ops;
+  st->live_word_ops = G.live_word_ops;
   st->rows_bit = G.rows[CLS_BIT]; st->rows_u8 = G.rows[CLS_U8];
   st->rows_u16 = G.rows[CLS_U16]; st->rows_u32 = G.rows[CLS_U32];
   st->xrows_bit = G.xrows[CLS_BIT]; st->xrows_u8 = G.xrows[CLS_U8];

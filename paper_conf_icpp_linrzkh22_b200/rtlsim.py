@@ -22,6 +22,7 @@ RTLSIM_OK = 0
 STATUS = {0: "OK", -1: "E_ARG", -2: "E_IR", -3: "E_COMB_LOOP", -4: "E_UNSUPPORTED", -5: "E_NOMEM",
           -6: "E_CUDA", -7: "E_STATE", -8: "E_RANGE"}
 F_DIGEST, F_NO_PIPELINE, F_GRAPH, F_HOST_ONLY, F_TIMING, F_JIT, F_V4, F_STREAM = 0x1, 0x2, 0x4, 0x8, 0x10, 0x20, 0x40, 0x80
+F_NO_DCE = 0x100
 
 EXPORTS = ["rtlsim_load", "rtlsim_bind", "rtlsim_bind_device", "rtlsim_bind_stream", "rtlsim_run",
            "rtlsim_run_device", "rtlsim_run_stream", "rtlsim_sync", "rtlsim_get_regs", "rtlsim_set_regs",
@@ -71,7 +72,8 @@ class Stats(ctypes.Structure):
                 ("eval_launches", ctypes.c_uint64), ("eval_stim_cycles", ctypes.c_uint64),
                 ("jit_compile_s", ctypes.c_double), ("jit_cubin_bytes", ctypes.c_uint64),
                 ("n_bitops", ctypes.c_uint64), ("n_narrow", ctypes.c_uint64), ("n_wide", ctypes.c_uint64),
-                ("n_ld", ctypes.c_uint64), ("n_st", ctypes.c_uint64), ("b_spill", ctypes.c_double)]
+                ("n_ld", ctypes.c_uint64), ("n_st", ctypes.c_uint64), ("b_spill", ctypes.c_double),
+                ("n_live_ops", ctypes.c_uint64), ("live_word_ops", ctypes.c_uint64)]
 
 
 PRODUCER = ctypes.CFUNCTYPE(ctypes.c_int, ctypes.c_void_p, ctypes.c_uint64, ctypes.c_uint64,

@@ -49,6 +49,42 @@ def test_host_only_compile_and_stats(R):
     assert st["n_steps"] >= 3 and st["smem_words"] > 0
 
 
+def _live_ops_reference(ir):
+    """Ops whose value reaches a register D or an output (reverse reachability
+    over the op DAG, written independently of csrc/compile.cpp)."""
+    import numpy as np
+    from rtlgen import ir as I
+    op = ir.ops
+    drv = {int(d): i for i, d in enumerate(op["dst"])}
+    need = set(int(s) for s in ir.reg_d) | set(int(s) for s in ir.output_sig)
+    stack, live = list(need), set()
+    while stack:
+        s = stack.pop()
+        i = drv.get(s)
+        if i is None or i in live:
+            continue
+        live.add(i)
+        for f in ("a", "b", "c"):
+            v = int(op[f][i])
+            if v != 0xFFFFFFFF and v not in need:
+                need.add(v)
+                stack.append(v)
+    return len(live)
+
+
+@pytest.mark.parametrize("cid", [2, 3])
+def test_dead_logic_elimination_counts(R, cid):
+    """Only ops that can reach an observable (register D / output) are
+    scheduled; RTLSIM_F_NO_DCE schedules all of them."""
+    ir = shaped.generate(cid)
+    st = _load(R, ir).stats()
+    assert st["n_ops"] == ir.n_ops
+    assert st["n_live_ops"] == _live_ops_reference(ir) < ir.n_ops
+    full = R.Simulator(ir, flags=R.F_HOST_ONLY | R.F_NO_DCE).stats()
+    assert full["n_live_ops"] == ir.n_ops and full["word_ops"] == st["word_ops"]
+    assert st["live_word_ops"] < full["live_word_ops"] and st["n_desc"] < full["n_desc"]
+
+
 def test_partitioned_design_uses_cross_partition_nets(R):
     ir = designs.random_dag(5, n_ops=200, n_regs=10, n_partitions=3)
     st = _load(R, ir).stats()

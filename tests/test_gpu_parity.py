@@ -88,6 +88,16 @@ def test_shaped_reduced(R, oracle_lib, cid, scale, N, T):
                 f"config{cid}@{scale}")
 
 
+@pytest.mark.parametrize("cid,scale,N,T", [(3, 0.25, 96, 12), (4, 0.01, 64, 6)])
+def test_no_dce_shaped(R, oracle_lib, cid, scale, N, T):
+    """Dead logic kept (RTLSIM_F_NO_DCE): the same bits as the default schedule and the oracle."""
+    ir = shaped.generate(cid, scale=scale)
+    st = stim.stimulus(ir, stim.STIM_SEED_BASE + cid, np.arange(N), 0, T)
+    want = oracle_lib.simulate(ir, st, digest=True, threads=16)
+    for fl in (R.F_NO_DCE, R.F_NO_DCE | R.F_JIT):
+        assert_same(gpu_run(R, ir, st, chunk_cycles=5, flags=fl), want, f"config{cid} flags={fl}")
+
+
 @pytest.mark.parametrize("seed,parts", [(0, 1), (1, 3), (2, 5)])
 def test_jit_sequential_dag(R, oracle_lib, seed, parts):
     """The JIT backend (specialized PTX per partition) on wide, partitioned designs."""
@@ -123,7 +133,8 @@ def test_modes_agree(R, oracle_lib):
     want = oracle_lib.simulate(ir, st, digest=True, threads=8)
     for opt in (dict(flags=R.F_GRAPH, chunk_cycles=8), dict(flags=R.F_NO_PIPELINE), dict(op_lanes=1),
                 dict(flags=R.F_STREAM, chunk_cycles=6), dict(flags=R.F_V4, chunk_cycles=9), dict(flags=R.F_V4 | R.F_GRAPH, chunk_cycles=4),
-                dict(op_lanes=7, chunk_cycles=5), dict(flags=R.F_GRAPH | R.F_NO_PIPELINE, chunk_cycles=33)):
+                dict(op_lanes=7, chunk_cycles=5), dict(flags=R.F_GRAPH | R.F_NO_PIPELINE, chunk_cycles=33),
+                dict(flags=R.F_NO_DCE), dict(flags=R.F_NO_DCE | R.F_JIT, chunk_cycles=11)):
         assert_same(gpu_run(R, ir, st, **opt), want, str(opt))
 
 
