@@ -50,6 +50,7 @@ constexpr int kN32 = 4, kN64 = 20;
 
 struct Em {
   std::string s;
+  bool dig = false;   // emit the per-(stimulus, cycle) digest code (check-mode kernels only)
   uint32_t nr = 0, nrd = 0, np = 0, nlab = 0;
   std::string R() { return fmt("%%r%u", nr++); }
   std::string RD() { return fmt("%%rd%u", nrd++); }
@@ -202,8 +203,56 @@ void emit_narrow(Em &e, const Desc &q) {
   std::string x = fetch_narrow(e, la, a, wa);
   std::string y = hb ? fetch_narrow(e, lb, b, wb) : std::string();
   std::string z = hc ? fetch_narrow(e, lc, c, 32) : std::string();
+  // a 1-bit compare / reduction into a packed bit slot: predicate -> ballot
+  // directly (no 0/1 materialisation, no second test)
+  if (ld == LC_BIT) {
+    const char *cc = nullptr;
+    bool sg = false;
+    std::string u = x, v = y;
+    switch (op) {
+      case RTLSIM_OP_EQ: cc = "eq"; break;
+      case RTLSIM_OP_NE: cc = "ne"; break;
+      case RTLSIM_OP_LTU: cc = "lt"; break;
+      case RTLSIM_OP_LEU: cc = "le"; break;
+      case RTLSIM_OP_GTU: cc = "gt"; break;
+      case RTLSIM_OP_GEU: cc = "ge"; break;
+      case RTLSIM_OP_LTS: cc = "lt"; sg = true; break;
+      case RTLSIM_OP_LES: cc = "le"; sg = true; break;
+      case RTLSIM_OP_GTS: cc = "gt"; sg = true; break;
+      case RTLSIM_OP_GES: cc = "ge"; sg = true; break;
+      case RTLSIM_OP_REDAND: cc = "eq"; v = fmt("%u", mask_of(wa)); break;
+      case RTLSIM_OP_REDOR: cc = "ne"; v = "0"; break;
+      default: break;
+    }
+    if (cc) {
+      if (sg) {
+        u = sext32(e, x, wa);
+        v = sext32(e, y, wb);
+      }
+      std::string p = e.P(), m = e.R();
+      e.l(fmt("setp.%s.%s %s, %s, %s", cc, sg ? "s32" : "u32", p.c_str(), u.c_str(), v.c_str()));
+      e.l(fmt("vote.sync.ballot.b32 %s, %s, 0xffffffff", m.c_str(), p.c_str()));
+      e.l(fmt("st.shared.u32 [%%smb+%u], %s", d * 4, m.c_str()));
+      return;
+    }
+  }
   std::string r = e.R();
   bool canon = false;   // result already < 2^wd
+  // bits the raw result can occupy (operands are canonical: < 2^w); no mask
+  // is needed when they fit wd, or when a byte / half-word slot store of an
+  // 8- / 16-bit value truncates by itself
+  uint32_t span = 32;
+  switch (op) {
+    case RTLSIM_OP_COPY: case RTLSIM_OP_SHRL: case RTLSIM_OP_DIVU: case RTLSIM_OP_MODU: span = wa; break;
+    case RTLSIM_OP_AND: span = std::min(wa, wb); break;
+    case RTLSIM_OP_OR: case RTLSIM_OP_XOR: span = std::max(wa, wb); break;
+    case RTLSIM_OP_ADD: span = std::max(wa, wb) + 1; break;
+    case RTLSIM_OP_MUL: span = wa + wb; break;
+    case RTLSIM_OP_CONCAT: span = wa + wb; break;
+    case RTLSIM_OP_SLICE: span = wa > imm ? wa - imm : 0; break;
+    default: break;
+  }
+  if (span <= wd || (ld == LC_U8 && wd == 8) || (ld == LC_U16 && wd == 16)) canon = true;
   // predicate-free forms (set.* gives 0 / all ones): ptxas compiles them far
   // faster than setp/selp chains and the SASS is the same length
   auto cmp = [&](const char *cc, const std::string &u, const std::string &v) {
@@ -554,6 +603,7 @@ void emit_ld(Em &e, uint32_t arena, uint32_t cls, uint32_t row, uint32_t slot, u
 }
 
 void emit_dig(Em &e, uint32_t key, const std::string &v) {
+  if (!e.dig) return;
   std::string skip = e.L("nd");
   e.l(fmt("@!%%pdig bra.uni %s", skip.c_str()));
   e.s += "\t{\n\t.param .b64 dp0;\n\t.param .b32 dp1;\n\t.param .b32 dp2;\n";
@@ -605,7 +655,7 @@ void emit_st(Em &e, uint32_t code, uint32_t cls, uint32_t nw, uint32_t lay, uint
       if (cls == CLS_U8) e.l(fmt("mad.wide.u32 %s, %%N, %u, %%tb_%s1", addr.c_str(), row, A));
       else e.l(fmt("mad.wide.u32 %s, %%N2, %u, %%tb_%s2", addr.c_str(), row, A));
       e.l(fmt("@%s st.global.u32 [%s], %s", pl, addr.c_str(), t.c_str()));
-      if (dg) emit_dig(e, aux + 1u + 0x80000000u, fetch_narrow(e, lay, slot, 16));
+      if (dg && e.dig) emit_dig(e, aux + 1u + 0x80000000u, fetch_narrow(e, lay, slot, 16));
       return;
     }
     default: {
@@ -613,7 +663,7 @@ void emit_st(Em &e, uint32_t code, uint32_t cls, uint32_t nw, uint32_t lay, uint
       e.l(fmt("ld.shared.u32 %s, [%%smb+%u]", t.c_str(), slot * 4));
       e.l(fmt("mad.wide.u32 %s, %%Nb, %u, %%tb_%s0", addr.c_str(), row, A));
       e.l(fmt("@%%pl0 st.global.u32 [%s], %s", addr.c_str(), t.c_str()));
-      if (dg) {
+      if (dg && e.dig) {
         std::string b = e.R(), b2 = e.R();
         e.l(fmt("shr.b32 %s, %s, %%lane", b.c_str(), t.c_str()));
         e.l(fmt("and.b32 %s, %s, 1", b2.c_str(), b.c_str()));
@@ -693,8 +743,9 @@ std::string func_proto(const std::string &name) {
 // (bar.sync 0, counted per CTA, not per PC) inside every warp's stream — so
 // a warp's instruction fetch is sequential across steps instead of jumping
 // over the other warps' code at every step.
-std::string step_function(const Program &G, const std::string &name, uint32_t s0, uint32_t s1) {
+std::string step_function(const Program &G, const std::string &name, uint32_t s0, uint32_t s1, bool dig) {
   Em e;
+  e.dig = dig;
   std::vector<std::string> labs(G.L);
   std::string tbl = e.L("T"), end = e.L("E");
   if (G.L > 1) {
@@ -736,7 +787,7 @@ std::string step_function(const Program &G, const std::string &name, uint32_t s0
 
 }  // namespace
 
-std::string jit_partition_ptx(const Program &G, uint32_t q, const std::string &rt_ptx, uint32_t tmax) {
+std::string jit_partition_ptx(const Program &G, uint32_t q, const std::string &rt_ptx, uint32_t tmax, bool dig) {
   const uint32_t s0 = G.part_steps[q], s1 = G.part_steps[q + 1];
   std::string mod;
   mod.reserve(1 << 20);
@@ -757,7 +808,7 @@ std::string jit_partition_ptx(const Program &G, uint32_t q, const std::string &r
     }
   }
   for (size_t g = 0; g < groups.size(); g++)
-    mod += step_function(G, fmt("rtl_steps_%zu", g), groups[g].first, groups[g].second) + "\n";
+    mod += step_function(G, fmt("rtl_steps_%zu", g), groups[g].first, groups[g].second, dig) + "\n";
   // the kernel: per-thread context, then the step functions in order
   // A CTA holds `tpc` tiles; warp g works on tile g / L as op-lane g % L, so
   // the warps of one op-lane (one per tile) run identical code in step
@@ -839,7 +890,7 @@ static int compile_ptx(const std::string &ptx, bool o3, std::vector<char> *cubin
 }
 
 int jit_build(const Program &G, const std::string &rt_ptx_path, uint32_t smem_bytes, int device, JitKernels *out,
-              std::string *err) {
+              std::string *err, bool dig) {
   std::ifstream f(rt_ptx_path);
   if (!f) {
     *err = "cannot read " + rt_ptx_path;
@@ -878,7 +929,7 @@ int jit_build(const Program &G, const std::string &rt_ptx_path, uint32_t smem_by
     th.emplace_back([&]() {
       for (uint32_t q; (q = next++) < NP;) {
         if (G.part_steps[q] == G.part_steps[q + 1]) continue;
-        std::string ptx = jit_partition_ptx(G, q, rt, tmax);
+        std::string ptx = jit_partition_ptx(G, q, rt, tmax, dig);
         ptx_bytes += ptx.size();
         if (const char *dir = getenv("RTLSIM_JIT_SAVE")) {   // debugging aid: keep the module
           std::ofstream o(fmt("%s/part%u.ptx", dir, q));

@@ -45,11 +45,12 @@ struct JitKernels {
 };
 
 // PTX text of exec-order partition q (steps part_steps[q]..part_steps[q+1]).
-std::string jit_partition_ptx(const Program &G, uint32_t q, const std::string &rt_ptx, uint32_t tmax);
+// dig: include the per-(stimulus, cycle) digest code (check-mode variant).
+std::string jit_partition_ptx(const Program &G, uint32_t q, const std::string &rt_ptx, uint32_t tmax, bool dig);
 // Generate + compile (nvPTXCompiler, all host cores) + load every partition.
 // device < 0: generate and compile only (host-only contexts, CPU tests).
 int jit_build(const Program &G, const std::string &rt_ptx_path, uint32_t smem_bytes, int device, JitKernels *out,
-              std::string *err);
+              std::string *err, bool dig);
 void jit_free(JitKernels *k);
 
 }  // namespace rtlsim

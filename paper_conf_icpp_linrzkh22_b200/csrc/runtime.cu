@@ -104,8 +104,10 @@ struct rtlsim_ctx {
   std::vector<cudaEvent_t> event_pool;
   double eval_ms = 0;
   uint64_t eval_launches = 0, eval_stim_cycles = 0;
-  JitKernels jit;        // RTLSIM_F_JIT
-  uint32_t jit_smem = 0;
+  JitKernels jit;        // RTLSIM_F_JIT (no digest code)
+  JitKernels jit_dig;    // RTLSIM_F_JIT check-mode variant, built on the first digest run
+  std::string jit_rt_path;
+  uint32_t jit_smem = 0, jit_smem_cap = 0;
 };
 
 #define CK(call)                                                                       \
@@ -254,9 +256,12 @@ extern "C" int rtlsim_load(const rtlsim_ir *ir, const rtlsim_options *opt, rtlsi
       dir = dir.substr(0, dir.find_last_of('/'));
     }
     ctx->jit_smem = std::max<uint32_t>(jit_tile_bytes(G), 16u);
+    ctx->jit_rt_path = dir + "/jit_rt.ptx";
+    ctx->jit_smem_cap = std::min<uint32_t>(ctx->jit_smem * kJitMaxTiles, smem_limit);
     std::string jerr;
-    int jr = jit_build(G, dir + "/jit_rt.ptx", std::min<uint32_t>(ctx->jit_smem * kJitMaxTiles, smem_limit), device,
-                       &ctx->jit, &jerr);
+    int jr = jit_build(G, ctx->jit_rt_path, ctx->jit_smem_cap, device, &ctx->jit, &jerr, false);
+    if (jr == RTLSIM_OK && (ctx->opt.flags & RTLSIM_F_DIGEST))
+      jr = jit_build(G, ctx->jit_rt_path, ctx->jit_smem_cap, device, &ctx->jit_dig, &jerr, true);
     if (jr != RTLSIM_OK) g_load_error = "JIT: " + jerr;
     return jr;
   };
@@ -549,6 +554,17 @@ static int launch_chunk(rtlsim_ctx *ctx, int b, uint64_t cycle0, uint32_t nc, bo
     return RTLSIM_OK;
   }
   const bool jit = (ctx->opt.flags & RTLSIM_F_JIT) != 0;
+  if (jit && digest && ctx->jit_dig.kern.empty()) {
+    // check-mode kernels (digest code compiled in) on first use
+    std::string jerr;
+    int jr = jit_build(G, ctx->jit_rt_path, ctx->jit_smem_cap, ctx->device, &ctx->jit_dig, &jerr, true);
+    if (jr != RTLSIM_OK) {
+      ctx->failed = true;
+      ctx->err = "JIT (digest variant): " + jerr;
+      return jr;
+    }
+  }
+  const JitKernels &JK = digest ? ctx->jit_dig : ctx->jit;
   // Tc x P per-(cycle, partition) kernel nodes (graph / JIT / stream modes)
   auto issue = [&](cudaStream_t cap) -> cudaError_t {
     const uint32_t NP = (uint32_t)G.part_steps.size() - 1;
@@ -557,7 +573,7 @@ static int launch_chunk(rtlsim_ctx *ctx, int b, uint64_t cycle0, uint32_t nc, bo
         if (G.part_steps[q] == G.part_steps[q + 1]) continue;
         cudaError_t e;
         if (jit) {
-          if (!ctx->jit.kern[q]) continue;
+          if (!JK.kern[q]) continue;
           const uint32_t par = (uint32_t)(((cycle0 & 1ull) + c) & 1ull);
           JitParams jp{};
           const Arena *ar[3] = {&ctx->state[par], &ctx->state[par ^ 1u], &ctx->xnet};
@@ -576,7 +592,7 @@ static int launch_chunk(rtlsim_ctx *ctx, int b, uint64_t cycle0, uint32_t nc, bo
           jp.N = ctx->N_pad;
           jp.tpc = jit_tiles_per_cta(ctx);
           void *args[] = {&jp};
-          e = cudaLaunchKernel((const void *)ctx->jit.kern[q], dim3(ctx->N_pad / 32u / jp.tpc),
+          e = cudaLaunchKernel((const void *)JK.kern[q], dim3(ctx->N_pad / 32u / jp.tpc),
                                dim3(32u * G.L * jp.tpc), args, ctx->jit_smem * jp.tpc, cap);
         } else {
           EvalParams p = eval_params(ctx, b, (cycle0 & 1ull) + c, 1, digest);
@@ -935,6 +951,7 @@ extern "C" void rtlsim_free(rtlsim_ctx *ctx) {
     if (ctx->st_d2h) cudaStreamSynchronize(ctx->st_d2h);
     free_binding(ctx);
     jit_free(&ctx->jit);
+    jit_free(&ctx->jit_dig);
     for (auto &t : ctx->timed_pending) {
       cudaEventDestroy(t.a);
       cudaEventDestroy(t.b);
