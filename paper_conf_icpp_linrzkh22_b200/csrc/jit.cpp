@@ -22,6 +22,7 @@
 #include <mutex>
 #include <sstream>
 #include <thread>
+#include <unordered_map>
 
 namespace rtlsim {
 namespace {
@@ -48,9 +49,40 @@ const char *kCtx64[] = {"tb_c0", "tb_c1", "tb_c2", "tb_c3", "tb_n0", "tb_n1", "t
                         "outb", "dig", "wide", "smg"};
 constexpr int kN32 = 4, kN64 = 20;
 
+// Shared-memory slot keys for register forwarding: (space, word offset).
+enum : uint64_t { SP_W = 1, SP_H = 2, SP_B = 3, SP_S = 4 };   // [%rw] [%rh] [%rb] [%smb]
+inline uint64_t skey(uint64_t sp, uint32_t off) { return (sp << 32) | off; }
+
+// Writes of one step function, by (step, warp), per slot key (dry pass).
+struct WriteLog {
+  std::unordered_map<uint64_t, std::vector<std::pair<int32_t, uint32_t>>> w;
+  // another warp wrote `key` in steps (s0, s1]
+  bool other(uint64_t key, uint32_t warp, int32_t s0, int32_t s1) const {
+    auto it = w.find(key);
+    if (it == w.end()) return false;
+    for (const auto &x : it->second)
+      if (x.second != warp && x.first > s0 && x.first <= s1) return true;
+    return false;
+  }
+};
+
 struct Em {
   std::string s;
   bool dig = false;   // emit the per-(stimulus, cycle) digest code (check-mode kernels only)
+  // register forwarding of slot values within one step function: a slot this
+  // warp stored (or already loaded) is read from the register that holds it,
+  // unless another warp (or a cp.async / the generic wide path) wrote the slot
+  // since. Stores are always kept (other warps / later functions read them).
+  bool dry = true;           // dry pass: only record writes
+  WriteLog *log = nullptr;
+  int32_t step = 0;
+  uint32_t warp = 0;
+  int32_t fwd_max = 0;       // forwarding distance in steps (0: off)
+  struct Fwd {
+    std::string reg;
+    int32_t step;
+  };
+  std::unordered_map<uint64_t, Fwd> fwd;
   uint32_t nr = 0, nrd = 0, np = 0, nlab = 0;
   std::string R() { return fmt("%%r%u", nr++); }
   std::string RD() { return fmt("%%rd%u", nrd++); }
@@ -69,39 +101,76 @@ struct Em {
 
 inline uint32_t mask_of(uint32_t w) { return w >= 32 ? 0xFFFFFFFFu : ((1u << w) - 1u); }
 
+const char *kSpBase[5] = {"", "%rw", "%rh", "%rb", "%smb"};
+const char *kSpTy[5] = {"", "u32", "u16", "u8", "u32"};
+
+// slot read (forwarded from a register when valid)
+std::string lds(Em &e, uint64_t sp, uint32_t off) {
+  const uint64_t k = skey(sp, off);
+  if (!e.dry && e.fwd_max > 0) {
+    auto it = e.fwd.find(k);
+    if (it != e.fwd.end()) {
+      if (e.step - it->second.step <= e.fwd_max && !e.log->other(k, e.warp, it->second.step, e.step))
+        return it->second.reg;
+      e.fwd.erase(it);
+    }
+  }
+  std::string r = e.R();
+  e.l(fmt("ld.shared.%s %s, [%s+%u]", kSpTy[sp], r.c_str(), kSpBase[sp], off * 4));
+  if (!e.dry) e.fwd[k] = Em::Fwd{r, e.step};
+  return r;
+}
+// slot write from a register
+void sts(Em &e, uint64_t sp, uint32_t off, const std::string &r) {
+  const uint64_t k = skey(sp, off);
+  e.l(fmt("st.shared.%s [%s+%u], %s", kSpTy[sp], kSpBase[sp], off * 4, r.c_str()));
+  if (e.dry) e.log->w[k].push_back({e.step, e.warp});
+  else e.fwd[k] = Em::Fwd{r, e.step};
+}
+// a write this warp cannot forward (cp.async, generic path)
+void opaque_write(Em &e, uint64_t sp, uint32_t off) {
+  const uint64_t k = skey(sp, off);
+  if (e.dry) e.log->w[k].push_back({e.step, e.warp});
+  else e.fwd.erase(k);
+}
+uint64_t layout_space(uint32_t lay) {
+  return lay == LC_U32 ? SP_W : lay == LC_U16 ? SP_H : lay == LC_U8 ? SP_B : SP_S;
+}
+
 // ------------------------------------------------------------- operands --
 // narrow (<= 32-bit) value from a slot of layout `lay` (or an immediate)
 std::string fetch_narrow(Em &e, uint32_t lay, uint32_t off, uint32_t /*w*/) {
-  std::string r = e.R();
   switch (lay) {
-    case LC_U32: e.l(fmt("ld.shared.u32 %s, [%%rw+%u]", r.c_str(), off * 4)); break;
-    case LC_U16: e.l(fmt("ld.shared.u16 %s, [%%rh+%u]", r.c_str(), off * 4)); break;
-    case LC_U8: e.l(fmt("ld.shared.u8 %s, [%%rb+%u]", r.c_str(), off * 4)); break;
+    case LC_U32: return lds(e, SP_W, off);
+    case LC_U16: return lds(e, SP_H, off);
+    case LC_U8: return lds(e, SP_B, off);
     case LC_BIT: {
-      std::string t = e.R(), t2 = e.R();
-      e.l(fmt("ld.shared.u32 %s, [%%smb+%u]", t.c_str(), off * 4));
+      std::string t = lds(e, SP_S, off), t2 = e.R(), r = e.R();
       e.l(fmt("shr.b32 %s, %s, %%lane", t2.c_str(), t.c_str()));
       e.l(fmt("and.b32 %s, %s, 1", r.c_str(), t2.c_str()));
-      break;
+      return r;
     }
-    case LC_BCAST: e.l(fmt("ld.shared.u32 %s, [%%smb+%u]", r.c_str(), off * 4)); break;
-    default: e.l(fmt("mov.u32 %s, %u", r.c_str(), off)); break;   // LC_IMM
+    case LC_BCAST: return lds(e, SP_S, off);
+    default: {   // LC_IMM
+      std::string r = e.R();
+      e.l(fmt("mov.u32 %s, %u", r.c_str(), off));
+      return r;
+    }
   }
-  return r;
 }
 
 void store_narrow(Em &e, uint32_t lay, uint32_t off, const std::string &r) {
   switch (lay) {
-    case LC_U32: e.l(fmt("st.shared.u32 [%%rw+%u], %s", off * 4, r.c_str())); break;
-    case LC_U16: e.l(fmt("st.shared.u16 [%%rh+%u], %s", off * 4, r.c_str())); break;
-    case LC_U8: e.l(fmt("st.shared.u8 [%%rb+%u], %s", off * 4, r.c_str())); break;
+    case LC_U32: sts(e, SP_W, off, r); break;
+    case LC_U16: sts(e, SP_H, off, r); break;
+    case LC_U8: sts(e, SP_B, off, r); break;
     default: {   // LC_BIT: pack the warp's 32 results
       std::string p = e.P(), m = e.R();
       e.l(fmt("setp.ne.u32 %s, %s, 0", p.c_str(), r.c_str()));
       e.l(fmt("vote.sync.ballot.b32 %s, %s, 0xffffffff", m.c_str(), p.c_str()));
       // every lane holds the same ballot word: an unpredicated store is one
       // same-address wavefront (and compiles much faster than a predicated one)
-      e.l(fmt("st.shared.u32 [%%smb+%u], %s", off * 4, m.c_str()));
+      sts(e, SP_S, off, m);
       break;
     }
   }
@@ -138,9 +207,7 @@ std::string wword(Em &e, WOp &o, uint32_t i, bool sx) {
       if (o.narrow.empty()) o.narrow = fetch_narrow(e, o.lay, o.off, o.w);
       r = o.narrow;
     } else {
-      r = e.R();
-      if (o.lay == LC_BCAST) e.l(fmt("ld.shared.u32 %s, [%%smb+%u]", r.c_str(), (o.off + j) * 4));
-      else e.l(fmt("ld.shared.u32 %s, [%%rw+%u]", r.c_str(), (o.off + 32 * j) * 4));
+      r = o.lay == LC_BCAST ? lds(e, SP_S, o.off + j) : lds(e, SP_W, o.off + 32 * j);
     }
     o.zw[j] = r;
     return r;
@@ -181,7 +248,7 @@ void wstore(Em &e, uint32_t off, uint32_t wd, uint32_t i, const std::string &v) 
     e.l(fmt("and.b32 %s, %s, %u", m.c_str(), x.c_str(), mask_of(rem)));
     x = m;
   }
-  e.l(fmt("st.shared.u32 [%%rw+%u], %s", (off + 32 * i) * 4, x.c_str()));
+  sts(e, SP_W, off + 32 * i, x);
 }
 
 std::string reg_of(Em &e, const std::string &v) {
@@ -232,7 +299,7 @@ void emit_narrow(Em &e, const Desc &q) {
       std::string p = e.P(), m = e.R();
       e.l(fmt("setp.%s.%s %s, %s, %s", cc, sg ? "s32" : "u32", p.c_str(), u.c_str(), v.c_str()));
       e.l(fmt("vote.sync.ballot.b32 %s, %s, 0xffffffff", m.c_str(), p.c_str()));
-      e.l(fmt("st.shared.u32 [%%smb+%u], %s", d * 4, m.c_str()));
+      sts(e, SP_S, d, m);
       return;
     }
   }
@@ -346,6 +413,14 @@ void emit_generic_call(Em &e, uint32_t idx) {
   e.l("st.param.b32 [wp2], %lane");
   e.l("call.uni rtl_exec_wide, (wp0, wp1, wp2)");
   e.s += "\t}\n";
+}
+void generic_wide(Em &e, const WideRec &w, uint32_t idx) {
+  emit_generic_call(e, idx);
+  if (w.wd <= 32) {
+    opaque_write(e, layout_space(value_layout(w.wd, false)), w.d);
+  } else {
+    for (uint32_t i = 0; i < nwords(w.wd); i++) opaque_write(e, SP_W, w.d + 32 * i);
+  }
 }
 
 void emit_wide(Em &e, const WideRec &w, uint32_t idx) {
@@ -568,7 +643,7 @@ void emit_wide(Em &e, const WideRec &w, uint32_t idx) {
       return;
     }
     default:   // SHL / SHRL / SHRA by a variable amount: generic path
-      emit_generic_call(e, idx);
+      generic_wide(e, w, idx);
       return;
   }
 }
@@ -585,19 +660,23 @@ void emit_ld(Em &e, uint32_t arena, uint32_t cls, uint32_t row, uint32_t slot, u
         std::string ai = i == 0 ? addr : e.RD();
         e.l(fmt("mad.wide.u32 %s, %%N4, %u, %%tb_%s3", ai.c_str(), row + i, A));
         e.l(fmt("cp.async.ca.shared.global [%%rw+%u], [%s], 4", (slot + 32 * i) * 4, ai.c_str()));
+        opaque_write(e, SP_W, slot + 32 * i);
       }
       break;
     case CLS_U16:
       e.l(fmt("mad.wide.u32 %s, %%N2, %u, %%tb_%s2", addr.c_str(), row, A));
       e.l(fmt("@%%pl16 cp.async.ca.shared.global [%%rw+%u], [%s], 4", slot * 4, addr.c_str()));
+      opaque_write(e, SP_H, slot);
       break;
     case CLS_U8:
       e.l(fmt("mad.wide.u32 %s, %%N, %u, %%tb_%s1", addr.c_str(), row, A));
       e.l(fmt("@%%pl8 cp.async.ca.shared.global [%%rw+%u], [%s], 4", slot * 4, addr.c_str()));
+      opaque_write(e, SP_B, slot);
       break;
     default:
       e.l(fmt("mad.wide.u32 %s, %%Nb, %u, %%tb_%s0", addr.c_str(), row, A));
       e.l(fmt("@%%pl0 cp.async.ca.shared.global [%%smb+%u], [%s], 4", slot * 4, addr.c_str()));
+      opaque_write(e, SP_S, slot);
       break;
   }
 }
@@ -622,8 +701,7 @@ void emit_st(Em &e, uint32_t code, uint32_t cls, uint32_t nw, uint32_t lay, uint
     for (uint32_t i = 0; i < nw; i++) {
       std::string v;
       if (lay == LC_U32) {
-        v = e.R();
-        e.l(fmt("ld.shared.u32 %s, [%%rw+%u]", v.c_str(), (slot + 32 * i) * 4));
+        v = lds(e, SP_W, slot + 32 * i);
       } else {
         v = fetch_narrow(e, lay, slot, 32);
       }
@@ -639,8 +717,7 @@ void emit_st(Em &e, uint32_t code, uint32_t cls, uint32_t nw, uint32_t lay, uint
   switch (cls) {
     case CLS_U32:
       for (uint32_t i = 0; i < nw; i++) {
-        std::string v = e.R(), ai = e.RD();
-        e.l(fmt("ld.shared.u32 %s, [%%rw+%u]", v.c_str(), (slot + 32 * i) * 4));
+        std::string v = lds(e, SP_W, slot + 32 * i), ai = e.RD();
         e.l(fmt("mad.wide.u32 %s, %%N4, %u, %%tb_%s3", ai.c_str(), row + i, A));
         e.l(fmt("st.global.u32 [%s], %s", ai.c_str(), v.c_str()));
         if (dg) emit_dig(e, aux + i + 1u + 0x80000000u, v);
@@ -659,8 +736,7 @@ void emit_st(Em &e, uint32_t code, uint32_t cls, uint32_t nw, uint32_t lay, uint
       return;
     }
     default: {
-      std::string t = e.R();
-      e.l(fmt("ld.shared.u32 %s, [%%smb+%u]", t.c_str(), slot * 4));
+      std::string t = lds(e, SP_S, slot);
       e.l(fmt("mad.wide.u32 %s, %%Nb, %u, %%tb_%s0", addr.c_str(), row, A));
       e.l(fmt("@%%pl0 st.global.u32 [%s], %s", addr.c_str(), t.c_str()));
       if (dg && e.dig) {
@@ -678,8 +754,8 @@ void emit_ld_const(Em &e, const Program &G, uint32_t slot, uint32_t pool, uint32
   for (uint32_t i = 0; i < nw; i++) {
     std::string v = e.R();
     e.l(fmt("mov.u32 %s, %u", v.c_str(), G.const_pool[pool + i]));
-    if (bcast) e.l(fmt("st.shared.u32 [%%smb+%u], %s", (slot + i) * 4, v.c_str()));
-    else e.l(fmt("st.shared.u32 [%%rw+%u], %s", (slot + 32 * i) * 4, v.c_str()));
+    if (bcast) sts(e, SP_S, slot + i, v);
+    else sts(e, SP_W, slot + 32 * i, v);
   }
 }
 
@@ -701,11 +777,11 @@ void emit_bit(Em &e, const BitDesc &q) {
   for (int k = 0; k < 3; k++) {
     v[k] = e.R();
     if (immf & (1u << k)) e.l(fmt("mov.u32 %s, %u", v[k].c_str(), (f[k] & 1u) ? 0xFFFFFFFFu : 0u));
-    else e.l(fmt("ld.shared.u32 %s, [%%smb+%u]", v[k].c_str(), f[k] * 4));
+    else v[k] = lds(e, SP_S, f[k]);
   }
   std::string r = e.R();
   e.l(fmt("lop3.b32 %s, %s, %s, %s, 0x%02x", r.c_str(), v[0].c_str(), v[1].c_str(), v[2].c_str(), lop3_lut(lut)));
-  e.l(fmt("st.shared.u32 [%%smb+%u], %s", (q.y & 0xFFFFu) * 4, r.c_str()));
+  sts(e, SP_S, q.y & 0xFFFFu, r);
 }
 
 void emit_desc(Em &e, const Program &G, const Desc &q) {
@@ -731,6 +807,12 @@ void emit_desc(Em &e, const Program &G, const Desc &q) {
   }
 }
 
+// forwarding distance in steps (RTLSIM_JIT_FWD; 0 disables)
+int32_t jit_fwd_steps() {
+  static const int32_t d = getenv("RTLSIM_JIT_FWD") ? atoi(getenv("RTLSIM_JIT_FWD")) : 2;
+  return d;
+}
+
 std::string func_proto(const std::string &name) {
   std::string s = ".func " + name + "(";
   for (int i = 0; i < kN32; i++) s += fmt("%s.param .b32 a_%s", i ? ", " : "", kCtx32[i]);
@@ -744,8 +826,26 @@ std::string func_proto(const std::string &name) {
 // a warp's instruction fetch is sequential across steps instead of jumping
 // over the other warps' code at every step.
 std::string step_function(const Program &G, const std::string &name, uint32_t s0, uint32_t s1, bool dig) {
+  // dry pass: which warp writes which slot in which step (forwarding validity)
+  WriteLog log;
+  {
+    Em d;
+    d.dig = dig;
+    d.dry = true;
+    d.log = &log;
+    for (uint32_t w = 0; w < G.L; w++)
+      for (uint32_t s = s0; s < s1; s++) {
+        d.warp = w;
+        d.step = (int32_t)s;
+        for (uint32_t k = G.bit_ptr[s] + w; k < G.bit_ptr[s + 1]; k += G.L) emit_bit(d, G.bitdesc[k]);
+        for (uint32_t k = G.step_ptr[s * G.L + w]; k < G.step_ptr[s * G.L + w + 1]; k++) emit_desc(d, G, G.desc[k]);
+      }
+  }
   Em e;
   e.dig = dig;
+  e.dry = false;
+  e.log = &log;
+  e.fwd_max = jit_fwd_steps();
   std::vector<std::string> labs(G.L);
   std::string tbl = e.L("T"), end = e.L("E");
   if (G.L > 1) {
@@ -759,7 +859,10 @@ std::string step_function(const Program &G, const std::string &name, uint32_t s0
   }
   for (uint32_t w = 0; w < G.L; w++) {
     if (G.L > 1) e.lab(labs[w]);
+    e.fwd.clear();
+    e.warp = w;
     for (uint32_t s = s0; s < s1; s++) {
+      e.step = (int32_t)s;
       for (uint32_t k = G.bit_ptr[s] + w; k < G.bit_ptr[s + 1]; k += G.L) emit_bit(e, G.bitdesc[k]);
       for (uint32_t k = G.step_ptr[s * G.L + w]; k < G.step_ptr[s * G.L + w + 1]; k++) emit_desc(e, G, G.desc[k]);
       e.l("cp.async.commit_group");
@@ -907,7 +1010,9 @@ int jit_build(const Program &G, const std::string &rt_ptx_path, uint32_t smem_by
   }
   const uint32_t NP = (uint32_t)G.part_steps.size() - 1;
   // tiles per CTA the kernels are built for (their thread count bounds registers)
-  const uint32_t tmax = std::max<uint32_t>(1u, std::min<uint32_t>(kJitMaxTiles, smem_bytes / jit_tile_bytes(G)));
+  const uint32_t tmax = std::max<uint32_t>(
+      1u, std::min<uint32_t>(std::min<uint32_t>(jit_default_tiles(), 32u / std::max<uint32_t>(G.L, 1u)),
+                             smem_bytes / jit_tile_bytes(G)));
   out->tmax = tmax;
   // ptxas -O3 schedules this code ~1.8x better (config 3) but compiles ~3x
   // slower than --Ofast-compile=mid: use it unless the design is large
@@ -967,6 +1072,11 @@ int jit_build(const Program &G, const std::string &rt_ptx_path, uint32_t smem_by
     }
   }
   return RTLSIM_OK;
+}
+
+uint32_t jit_default_tiles() {
+  const char *e = getenv("RTLSIM_JIT_TMAX");   // read per load (tests vary it)
+  return e ? std::min<uint32_t>(kJitMaxTiles, (uint32_t)std::max(1, atoi(e))) : 2u;
 }
 
 void jit_free(JitKernels *k) {

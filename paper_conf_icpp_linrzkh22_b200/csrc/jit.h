@@ -31,7 +31,10 @@ struct JitParams {
 static_assert(sizeof(JitParams) == 160, "JitParams layout is hard-coded in the PTX generator");
 
 // Maximum tiles per CTA the kernels are compiled for (.maxntid 32 * L * kJitMaxTiles).
-constexpr uint32_t kJitMaxTiles = 2;
+constexpr uint32_t kJitMaxTiles = 8;
+// Tiles per CTA the kernels are compiled for by default (RTLSIM_JIT_TMAX
+// overrides, up to kJitMaxTiles and 1024 threads per CTA).
+uint32_t jit_default_tiles();
 // Bytes of shared memory per tile in a JIT CTA (16-byte aligned).
 inline uint32_t jit_tile_bytes(const Program &G) { return ((G.smem_words * 4u) + 15u) & ~15u; }
 

@@ -257,7 +257,7 @@ extern "C" int rtlsim_load(const rtlsim_ir *ir, const rtlsim_options *opt, rtlsi
     }
     ctx->jit_smem = std::max<uint32_t>(jit_tile_bytes(G), 16u);
     ctx->jit_rt_path = dir + "/jit_rt.ptx";
-    ctx->jit_smem_cap = std::min<uint32_t>(ctx->jit_smem * kJitMaxTiles, smem_limit);
+    ctx->jit_smem_cap = std::min<uint32_t>(ctx->jit_smem * jit_default_tiles(), smem_limit);
     std::string jerr;
     int jr = jit_build(G, ctx->jit_rt_path, ctx->jit_smem_cap, device, &ctx->jit, &jerr, false);
     if (jr == RTLSIM_OK && (ctx->opt.flags & RTLSIM_F_DIGEST))

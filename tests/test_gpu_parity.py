@@ -108,6 +108,24 @@ def test_jit_sequential_dag(R, oracle_lib, seed, parts):
                 oracle_lib.simulate(ir, st, digest=True, threads=8), f"jit seq{seed}")
 
 
+@pytest.mark.parametrize("lanes,tmax", [(1, "4"), (2, "3"), (3, "1"), (5, "2")])
+def test_jit_lanes_and_forwarding(R, oracle_lib, lanes, tmax, monkeypatch):
+    """JIT kernels at several op-lane counts and tiles per CTA: register
+    forwarding of slot values is only valid when no other warp wrote the slot
+    in between, which the op-lane count changes."""
+    monkeypatch.setenv("RTLSIM_JIT_TMAX", tmax)
+    monkeypatch.setenv("RTLSIM_JIT_TPC", tmax)
+    ir = designs.random_dag(700 + lanes, n_ops=400, n_regs=30, n_partitions=3,
+                            input_widths=(7, 33, 1, 64, 100, 1, 1), max_width=300)
+    st = stim.stimulus(ir, 31 + lanes, np.arange(160), 0, 24, mask=False)
+    assert_same(gpu_run(R, ir, st, chunk_cycles=8, flags=R.F_JIT, op_lanes=lanes),
+                oracle_lib.simulate(ir, st, digest=True, threads=8), f"jit lanes={lanes}")
+    ir = shaped.generate(3, scale=0.2)
+    st = stim.stimulus(ir, stim.STIM_SEED_BASE + 3, np.arange(128), 0, 12)
+    assert_same(gpu_run(R, ir, st, chunk_cycles=6, flags=R.F_JIT, op_lanes=lanes),
+                oracle_lib.simulate(ir, st, digest=True, threads=16), f"jit config3@0.2 lanes={lanes}")
+
+
 @pytest.mark.parametrize("seed", range(4))
 def test_jit_comb_dag_exhaustive(R, oracle_lib, seed):
     ir = designs.random_dag(seed, n_ops=60 + 25 * seed, input_widths=(3, 5, 1, 4, 3))
