@@ -1076,7 +1076,7 @@ int jit_build(const Program &G, const std::string &rt_ptx_path, uint32_t smem_by
 
 uint32_t jit_default_tiles() {
   const char *e = getenv("RTLSIM_JIT_TMAX");   // read per load (tests vary it)
-  return e ? std::min<uint32_t>(kJitMaxTiles, (uint32_t)std::max(1, atoi(e))) : 2u;
+  return e ? std::min<uint32_t>(kJitMaxTiles, (uint32_t)std::max(1, atoi(e))) : 4u;
 }
 
 void jit_free(JitKernels *k) {

@@ -159,7 +159,7 @@ static void free_binding(rtlsim_ctx *ctx) {
 }
 
 
-constexpr uint32_t kJitMaxLanes = 8;
+constexpr uint32_t kJitMaxLanes = 4;
 
 // descriptor staging buffers start after the slots, 16-byte aligned
 static uint32_t desc_smem_off(const Program &G) { return (G.smem_words + 3u) & ~3u; }
@@ -196,7 +196,8 @@ extern "C" int rtlsim_load(const rtlsim_ir *ir, const rtlsim_options *opt, rtlsi
   }
   std::string err;
   // JIT kernels are instruction-fetch bound: fewer, longer per-warp code runs
-  // measure faster (config 3: 8 op-lanes 1.9 ms/cycle vs 16: 3.5 ms)
+  // and more tiles sharing them measure faster (config 3: 4 op-lanes x 4
+  // tiles 0.74 ms/cycle, 8 x 2 1.08 ms, 16 x 1 3.5 ms)
   uint32_t lanes = ctx->opt.op_lanes;
   const bool dce = (ctx->opt.flags & RTLSIM_F_NO_DCE) == 0;
   if (!lanes && (ctx->opt.flags & RTLSIM_F_JIT)) lanes = kJitMaxLanes;
@@ -214,6 +215,18 @@ extern "C" int rtlsim_load(const rtlsim_ir *ir, const rtlsim_options *opt, rtlsi
     return rc;
   }
   const bool legacy = (ctx->opt.flags & RTLSIM_F_V4) == 0;
+  if ((ctx->opt.flags & RTLSIM_F_JIT) && !ctx->opt.smem_limit &&
+      (ctx->prog.smem_words + 64u) * 4u > smem_limit / 2u) {
+    // JIT kernels are instruction-fetch bound: two tiles per CTA (the warps
+    // of one op-lane share every fetched instruction) beat one tile with the
+    // whole working set on chip (config 4: 193 vs 306 ms/cycle), so the
+    // working set is budgeted to half the shared memory (long-lived values
+    // spill to HBM rows)
+    rtlsim::Program half;
+    std::string e2;
+    if (compile_program(ir, ctx->prog.L, (smem_limit / 2u - 1024u) / 4u, &half, &e2, dce) == RTLSIM_OK)
+      ctx->prog = std::move(half);
+  }
   // bytes after lowering: slots, the 32-word zero row (lower_program) and,
   // for the interpreter, one 512-byte descriptor staging buffer per op-lane
   auto final_bytes = [&](const Program &P) {
