@@ -306,8 +306,9 @@ void emit_narrow(Em &e, const Desc &q) {
   std::string r = e.R();
   bool canon = false;   // result already < 2^wd
   // bits the raw result can occupy (operands are canonical: < 2^w); no mask
-  // is needed when they fit wd, or when a byte / half-word slot store of an
-  // 8- / 16-bit value truncates by itself
+  // is needed when they fit wd. (A byte / half-word slot store would truncate
+  // an 8- / 16-bit value by itself, but the register is forwarded to later
+  // reads, so it must be canonical too.)
   uint32_t span = 32;
   switch (op) {
     case RTLSIM_OP_COPY: case RTLSIM_OP_SHRL: case RTLSIM_OP_DIVU: case RTLSIM_OP_MODU: span = wa; break;
@@ -319,7 +320,7 @@ void emit_narrow(Em &e, const Desc &q) {
     case RTLSIM_OP_SLICE: span = wa > imm ? wa - imm : 0; break;
     default: break;
   }
-  if (span <= wd || (ld == LC_U8 && wd == 8) || (ld == LC_U16 && wd == 16)) canon = true;
+  if (span <= wd) canon = true;
   // predicate-free forms (set.* gives 0 / all ones): ptxas compiles them far
   // faster than setp/selp chains and the SASS is the same length
   auto cmp = [&](const char *cc, const std::string &u, const std::string &v) {
