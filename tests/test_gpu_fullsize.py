@@ -21,7 +21,7 @@ def _sample(N, extra, seed=stim.SAMPLE_SEED):
     return np.array(sorted(i for i in idx if 0 <= i < N))
 
 
-def _run(cid, cycles, chunk, extra, s_offset=0, n=None):
+def _run(cid, cycles, chunk, extra, s_offset=0, n=None, jit=True):
     import torch
     import oracle
     from paper_conf_icpp_linrzkh22_b200 import build, rtlsim as R
@@ -31,22 +31,29 @@ def _run(cid, cycles, chunk, extra, s_offset=0, n=None):
     seed = stim.STIM_SEED_BASE + cid
     s = torch.cuda.Stream()
     torch.cuda.set_stream(s)
-    sim = R.Simulator(ir, chunk_cycles=chunk, stream=s.cuda_stream)
+    # bench.py's backend (JIT partition kernels) unless jit=False (interpreter)
+    sim = R.Simulator(ir, chunk_cycles=chunk, stream=s.cuda_stream, flags=(R.F_JIT if jit else 0) | R.F_TIMING)
     d_stim = stim.stimulus_torch(ir, seed, s_offset, N, 0, cycles)
     out = torch.zeros((N, cycles, ir.OW), dtype=torch.int32, device="cuda")
     dig = torch.zeros((N, cycles), dtype=torch.int64, device="cuda")
     sim.bind_device(d_stim, N, cycles)
-    sim.run_device(cycles, out, dig)
+    # 1. the kernels bench.py times (no digest code): outputs + final registers
+    sim.run_device(cycles, out)
     sim.sync()
     regs = sim.get_regs()
     pick = _sample(N, extra)
     st = stim.stimulus(ir, seed, pick + s_offset, 0, cycles)
     want = oracle.Design(ir).simulate(st, digest=True, threads=16)
     got_out = out.cpu().numpy().view(np.uint32)[pick]
-    got_dig = dig.cpu().numpy().view(np.uint64)[pick]
-    assert np.array_equal(got_dig, want["digest"]), "per-cycle digest differs"
     assert np.array_equal(got_out, want["out"])
     assert np.array_equal(regs[pick], want["regs"])
+    # 2. check mode: per-cycle digest over every output and next-state register word
+    sim.reset()
+    sim.run_device(cycles, out, dig)
+    sim.sync()
+    got_dig = dig.cpu().numpy().view(np.uint64)[pick]
+    assert np.array_equal(got_dig, want["digest"]), "per-cycle digest differs"
+    assert np.array_equal(sim.get_regs()[pick], want["regs"])
     return len(pick)
 
 
@@ -56,6 +63,10 @@ def test_config2_full_size():
 
 def test_config3_full_size():
     assert _run(3, cycles=25, chunk=25, extra=40) > 40
+
+
+def test_config3_full_size_interpreter():
+    assert _run(3, cycles=12, chunk=12, extra=20, jit=False) > 20
 
 
 def test_config4_full_size():
