@@ -250,3 +250,29 @@ def test_v4_shaped_reduced(R, oracle_lib, cid, scale, N, T):
     st = stim.stimulus(ir, stim.STIM_SEED_BASE + cid, np.arange(N), 0, T)
     assert_same(gpu_run(R, ir, st, chunk_cycles=16, flags=R.F_V4),
                 oracle_lib.simulate(ir, st, digest=True, threads=16), f"v4 config{cid}@{scale}")
+
+
+def test_mcmc_merged_partitions(R, oracle_lib):
+    """A task graph proposed by the MCMC partitioner (Alg 1) is the
+    same design: bit-identical to the oracle on the JIT and interpreter paths."""
+    from paper_conf_icpp_linrzkh22_b200 import partition as MP
+    ir = designs.random_dag(910, n_ops=600, n_regs=40, n_partitions=6, input_widths=(9, 40, 1, 3))
+    opt = MP.Optimizer(ir, n_tasks=3, seed=2)
+    for _ in range(3):
+        opt.random_increase()
+        opt.update_weights()
+    merged = MP.apply(ir, opt.propose(opt.weights))
+    assert merged.n_partitions <= 3
+    st = stim.stimulus(ir, 77, np.arange(100), 0, 20)
+    want = oracle_lib.simulate(ir, st, digest=True, threads=8)
+    for fl in (R.F_JIT, 0):
+        assert_same(gpu_run(R, merged, st, chunk_cycles=7, flags=fl), want, f"merged flags={fl}")
+
+
+def test_mcmc_gpu_estimator(R):
+    """The estimator of Algorithm 1 runs a candidate on the GPU and returns a
+    positive per-cycle time."""
+    from paper_conf_icpp_linrzkh22_b200 import partition as MP
+    ir = shaped.generate(3, scale=0.1)
+    c = MP.gpu_estimator(n_stim=256, cycles=4)(ir)
+    assert c > 0
