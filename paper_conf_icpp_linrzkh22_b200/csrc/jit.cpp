@@ -21,6 +21,7 @@
 #include <fstream>
 #include <mutex>
 #include <sstream>
+#include <map>
 #include <thread>
 #include <unordered_map>
 
@@ -267,6 +268,22 @@ void emit_narrow(Em &e, const Desc &q) {
   const uint32_t wd = (q.x >> 20) & 63u, wa = q.x >> 26, wb = q.w & 63u, imm = (q.w >> 6) & 31u;
   const bool hb = (q.w >> 11) & 1u, hc = (q.w >> 12) & 1u;
   const uint32_t d = q.y & 0xFFFFu, a = q.y >> 16, b = q.z & 0xFFFFu, c = q.z >> 16;
+  if (op == RTLSIM_OP_MUX && la == LC_BIT && hb && hc) {
+    // 1-bit select straight from its packed word: the lane's bit moved to
+    // bit 31 and sign-filled is the all-ones / zero mask of the LOP3 mux
+    std::string t = lds(e, SP_S, a), y = fetch_narrow(e, lb, b, wb), z = fetch_narrow(e, lc, c, 32);
+    std::string m1 = e.R(), m = e.R(), r = e.R();
+    e.l(fmt("shl.b32 %s, %s, %%lsh", m1.c_str(), t.c_str()));
+    e.l(fmt("shr.s32 %s, %s, 31", m.c_str(), m1.c_str()));
+    e.l(fmt("lop3.b32 %s, %s, %s, %s, 0xca", r.c_str(), m.c_str(), y.c_str(), z.c_str()));
+    std::string res = r;
+    if (wd < 32) {
+      res = e.R();
+      e.l(fmt("and.b32 %s, %s, %u", res.c_str(), r.c_str(), mask_of(wd)));
+    }
+    store_narrow(e, ld, d, res);
+    return;
+  }
   std::string x = fetch_narrow(e, la, a, wa);
   std::string y = hb ? fetch_narrow(e, lb, b, wb) : std::string();
   std::string z = hc ? fetch_narrow(e, lc, c, 32) : std::string();
@@ -785,7 +802,44 @@ void emit_bit(Em &e, const BitDesc &q) {
   sts(e, SP_S, q.y & 0xFFFFu, r);
 }
 
+// RTLSIM_JIT_STATS: PTX instruction lines per descriptor kind (stderr at exit)
+struct EmitStats {
+  std::mutex mu;
+  std::map<std::string, std::pair<uint64_t, uint64_t>> m;   // kind -> (count, lines)
+  ~EmitStats() {
+    if (m.empty()) return;
+    for (auto &kv : m)
+      fprintf(stderr, "jit-stats %-14s %9llu ops %11llu ptx lines %6.1f/op\n", kv.first.c_str(),
+              (unsigned long long)kv.second.first, (unsigned long long)kv.second.second,
+              (double)kv.second.second / (double)std::max<uint64_t>(kv.second.first, 1));
+  }
+};
+EmitStats g_emit_stats;
+size_t count_lines(const std::string &s, size_t from) {
+  size_t n = 0;
+  for (size_t i = from; i < s.size(); i++) n += s[i] == ';';
+  return n;
+}
+void note_kind(Em &e, const std::string &kind, size_t from) {
+  static const bool on = getenv("RTLSIM_JIT_STATS") != nullptr;
+  if (!on || e.dry) return;
+  std::lock_guard<std::mutex> g(g_emit_stats.mu);
+  auto &x = g_emit_stats.m[kind];
+  x.first++;
+  x.second += count_lines(e.s, from);
+}
+
+void emit_desc_(Em &e, const Program &G, const Desc &q);
 void emit_desc(Em &e, const Program &G, const Desc &q) {
+  const size_t from = e.s.size();
+  emit_desc_(e, G, q);
+  const uint32_t code = q.x & 0xFFu;
+  std::string kind = code < 32u ? "narrow" : code == CODE_WIDE ? "wide" : code == CODE_LD_CONST ? "ld_const"
+                   : (code == CODE_LD_REG || code == CODE_LD_X || code == CODE_LD_IN) ? "ld" : "st";
+  if (code < 32u) kind += ((q.x >> 17) & 7u) == LC_BIT ? ":bit" : "";
+  note_kind(e, kind, from);
+}
+void emit_desc_(Em &e, const Program &G, const Desc &q) {
   const uint32_t code = q.x & 0xFFu;
   if (code < 32u) {
     emit_narrow(e, q);
@@ -864,7 +918,11 @@ std::string step_function(const Program &G, const std::string &name, uint32_t s0
     e.warp = w;
     for (uint32_t s = s0; s < s1; s++) {
       e.step = (int32_t)s;
-      for (uint32_t k = G.bit_ptr[s] + w; k < G.bit_ptr[s + 1]; k += G.L) emit_bit(e, G.bitdesc[k]);
+      for (uint32_t k = G.bit_ptr[s] + w; k < G.bit_ptr[s + 1]; k += G.L) {
+        const size_t from = e.s.size();
+        emit_bit(e, G.bitdesc[k]);
+        note_kind(e, "bit", from);
+      }
       for (uint32_t k = G.step_ptr[s * G.L + w]; k < G.step_ptr[s * G.L + w + 1]; k++) emit_desc(e, G, G.desc[k]);
       e.l("cp.async.commit_group");
       e.l(fmt("cp.async.wait_group %u", G.step_wait[s]));
@@ -875,7 +933,7 @@ std::string step_function(const Program &G, const std::string &name, uint32_t s0
   e.lab(end);
   std::string out = func_proto(name) + "\n{\n";
   out += fmt("\t.reg .b32 %%r<%u>;\n\t.reg .b64 %%rd<%u>;\n\t.reg .pred %%p<%u>;\n", e.nr + 1, e.nrd + 1, e.np + 1);
-  out += "\t.reg .b32 %smb, %lane, %wl, %N, %rw, %rh, %rb, %N4, %N2, %Nb;\n\t.reg .b64 ";
+  out += "\t.reg .b32 %smb, %lane, %wl, %N, %rw, %rh, %rb, %N4, %N2, %Nb, %lsh;\n\t.reg .b64 ";
   for (int i = 0; i < kN64; i++) out += fmt("%s%%%s", i ? ", " : "", kCtx64[i]);
   out += ";\n\t.reg .pred %pl0, %pl8, %pl16, %pdig;\n";
   for (int i = 0; i < kN32; i++) out += fmt("\tld.param.u32 %%%s, [a_%s];\n", kCtx32[i], kCtx32[i]);
@@ -883,7 +941,7 @@ std::string step_function(const Program &G, const std::string &name, uint32_t s0
   out += "\tmad.lo.u32 %rw, %lane, 4, %smb;\n\tmad.lo.u32 %rh, %lane, 2, %smb;\n\tadd.u32 %rb, %lane, %smb;\n"
          "\tshl.b32 %N4, %N, 2;\n\tshl.b32 %N2, %N, 1;\n\tshr.u32 %Nb, %N, 3;\n"
          "\tsetp.eq.u32 %pl0, %lane, 0;\n\tsetp.lt.u32 %pl8, %lane, 8;\n\tsetp.lt.u32 %pl16, %lane, 16;\n"
-         "\tsetp.ne.u64 %pdig, %dig, 0;\n";
+         "\tsetp.ne.u64 %pdig, %dig, 0;\n\tsub.u32 %lsh, 31, %lane;\n";
   out += e.s;
   out += "\tret;\n}\n";
   return out;
