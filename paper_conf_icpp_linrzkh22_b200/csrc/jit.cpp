@@ -19,6 +19,9 @@
 #include <cstdlib>
 #include <cstring>
 #include <fstream>
+#include <iterator>
+#include <sys/stat.h>
+#include <unistd.h>
 #include <mutex>
 #include <sstream>
 #include <map>
@@ -1086,6 +1089,9 @@ int jit_build(const Program &G, const std::string &rt_ptx_path, uint32_t smem_by
   std::vector<std::string> errs(NP);
   std::atomic<uint32_t> next{0};
   std::atomic<size_t> ptx_bytes{0};
+  std::atomic<uint32_t> cache_hits{0};
+  if (const char *cdir = getenv("RTLSIM_JIT_CACHE"))
+    if (*cdir) mkdir(cdir, 0777);   // one level; an existing directory is fine
   auto t0 = std::chrono::steady_clock::now();
   unsigned nth = std::max(1u, std::thread::hardware_concurrency());
   std::vector<std::thread> th;
@@ -1099,9 +1105,40 @@ int jit_build(const Program &G, const std::string &rt_ptx_path, uint32_t smem_by
           std::ofstream o(fmt("%s/part%u.ptx", dir, q));
           o << ptx;
         }
-        if (compile_ptx(ptx, o3, &cubins[q], &errs[q]) != 0 && getenv("RTLSIM_JIT_DUMP")) {
-          std::ofstream o(fmt("/tmp/rtlsim_jit_fail_%u.ptx", q));
-          o << ptx;
+        // RTLSIM_JIT_CACHE=dir: cubins keyed by a hash of (PTX, options);
+        // lets the ranks of one node (bench.py) and repeated loads share work
+        const char *cdir = getenv("RTLSIM_JIT_CACHE");
+        std::string cpath;
+        if (cdir && *cdir) {
+          uint64_t h = 1469598103934665603ull;   // FNV-1a
+          auto mixin = [&](const std::string &x) {
+            for (unsigned char ch : x) h = (h ^ ch) * 1099511628211ull;
+          };
+          mixin(ptx);
+          mixin(o3 ? "|O3|sm_100a" : "|mid|sm_100a");
+          cpath = fmt("%s/%016llx.cubin", cdir, (unsigned long long)h);
+          std::ifstream in(cpath, std::ios::binary);
+          if (in) {
+            std::vector<char> buf((std::istreambuf_iterator<char>(in)), std::istreambuf_iterator<char>());
+            if (!buf.empty()) {
+              cubins[q] = std::move(buf);
+              cache_hits++;
+              continue;
+            }
+          }
+        }
+        if (compile_ptx(ptx, o3, &cubins[q], &errs[q]) != 0) {
+          if (getenv("RTLSIM_JIT_DUMP")) {
+            std::ofstream o(fmt("/tmp/rtlsim_jit_fail_%u.ptx", q));
+            o << ptx;
+          }
+        } else if (!cpath.empty()) {
+          const std::string tmp = cpath + fmt(".tmp%d.%u", (int)getpid(), q);
+          {
+            std::ofstream o(tmp, std::ios::binary);
+            o.write(cubins[q].data(), (std::streamsize)cubins[q].size());
+          }
+          std::rename(tmp.c_str(), cpath.c_str());
         }
       }
     });
@@ -1110,6 +1147,7 @@ int jit_build(const Program &G, const std::string &rt_ptx_path, uint32_t smem_by
   auto t1 = std::chrono::steady_clock::now();
   out->compile_s = std::chrono::duration<double>(t1 - t0).count();
   out->ptx_bytes = ptx_bytes;
+  out->cache_hits = cache_hits;
   for (uint32_t q = 0; q < NP; q++)
     if (!errs[q].empty()) {
       *err = fmt("partition %u: ", q) + errs[q];

@@ -45,6 +45,7 @@ struct JitKernels {
   bool o3 = false;
   uint32_t tmax = 1;                // tiles per CTA the kernels were built for
   size_t ptx_bytes = 0, cubin_bytes = 0;
+  uint32_t cache_hits = 0;          // partitions served from RTLSIM_JIT_CACHE
 };
 
 // PTX text of exec-order partition q (steps part_steps[q]..part_steps[q+1]).
