@@ -186,3 +186,16 @@ def test_product_does_not_import_oracle():
             if f.endswith((".py", ".cu", ".cpp", ".h")):
                 src = open(os.path.join(dirpath, f)).read()
                 assert "import oracle" not in src and "from oracle" not in src and "oracle.h" not in src, f
+
+
+def test_jit_cubin_cache(R, tmp_path, monkeypatch):
+    """RTLSIM_JIT_CACHE: the first load writes one cubin per partition
+    module, a second load of the same design reads them back (same bytes)."""
+    monkeypatch.setenv("RTLSIM_JIT_CACHE", str(tmp_path / "jc"))
+    ir = designs.random_dag(5, n_ops=200, n_regs=10, n_partitions=3)
+    a = R.Simulator(ir, flags=R.F_HOST_ONLY | R.F_JIT).stats()
+    files = sorted(p.name for p in (tmp_path / "jc").iterdir())
+    assert len(files) == 3 and all(f.endswith(".cubin") for f in files)
+    b = R.Simulator(ir, flags=R.F_HOST_ONLY | R.F_JIT).stats()
+    assert b["jit_cubin_bytes"] == a["jit_cubin_bytes"] > 0
+    assert sorted(p.name for p in (tmp_path / "jc").iterdir()) == files
