@@ -152,7 +152,7 @@ static uint32_t fast_handler(uint32_t opc, int ar, const uint32_t *lay, uint32_t
 }
 
 int compile_program(const rtlsim_ir *ir, uint32_t op_lanes, uint32_t smem_limit_words, Program *P,
-                    std::string *err, bool dce) {
+                    std::string *err, bool dce, bool fold_conv) {
   if (!ir || !P) return fail(err, RTLSIM_E_ARG, "NULL ir");
   const uint32_t n = ir->n_signals;
   if (n == 0 || !ir->width || !ir->kind) return fail(err, RTLSIM_E_IR, "no signals");
@@ -612,6 +612,7 @@ int compile_program(const rtlsim_ir *ir, uint32_t op_lanes, uint32_t smem_limit_
       uint32_t src_sig;  // signal whose value is stored
       int32_t src_val;   // value id; -2-k: synthesized copy k
       uint32_t idx;      // register or output index, or xnet signal
+      bool conv = false; // register store converting the width itself (CODE_ST_REGC)
     };
     std::vector<Sink> sinks;
     struct Synth {
@@ -621,7 +622,11 @@ int compile_program(const rtlsim_ir *ir, uint32_t op_lanes, uint32_t smem_limit_
     std::vector<Synth> synth;
     auto add_sink = [&](uint32_t code, uint32_t s, uint32_t w_target, uint32_t idx) {
       sinks.push_back(Sink{code, s, -1, idx});
-      if (G.width[s] != w_target || G.kind[s] == RTLSIM_CONST) {
+      if (fold_conv && code == CODE_ST_REG && G.kind[s] != RTLSIM_CONST && G.width[s] != w_target) {
+        // JIT kernels store q <- d mod 2^w_q straight from d's slot: no
+        // conversion copy, no extra slot live until the store
+        sinks.back().conv = true;
+      } else if (G.width[s] != w_target || G.kind[s] == RTLSIM_CONST) {
         synth.push_back(Synth{s, w_target, -1, is_local(s) ? op_step[def[s]] + 1 : -1});
         sinks.back().src_val = -2 - (int32_t)(synth.size() - 1);
       }
@@ -993,8 +998,16 @@ int compile_program(const rtlsim_ir *ir, uint32_t op_lanes, uint32_t smem_limit_
         else bytes_spill += lane_bytes(w);
       }
       d.x = sk.code | (width_class(w) << 8) | (nwords(w) << 12) | (v.layout << 18);
+      uint32_t cost = 1 + nwords(w);
+      if (sk.conv) {
+        const RegInfo &ri = G.regs[sk.idx];
+        if (ri.row >= (1u << 20)) return fail(err, RTLSIM_E_UNSUPPORTED, "more than 2^20 state rows in one class");
+        d.x = CODE_ST_REGC | (ri.cls << 8) | (nwords(ri.width) << 12) | (v.layout << 18) | (w << 21);
+        d.z = ri.row | (ri.width << 20);
+        cost = 1 + nwords(ri.width);
+      }
       G.n_st++;
-      steps[sink_step[k]].lane.push_back({d, 1 + nwords(w)});
+      steps[sink_step[k]].lane.push_back({d, cost});
     }
     // wait depth: at the end of step e at most w_e of the most recent
     // per-step cp.async groups may be pending; a load issued at step i and

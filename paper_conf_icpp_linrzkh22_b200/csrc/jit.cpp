@@ -771,6 +771,61 @@ void emit_st(Em &e, uint32_t code, uint32_t cls, uint32_t nw, uint32_t lay, uint
   }
 }
 
+// register store with the width conversion folded in (CODE_ST_REGC):
+// q <- d mod 2^w_q, d read from its own slot (layout slay, width sw)
+void emit_st_conv(Em &e, uint32_t tcls, uint32_t tnw, uint32_t slay, uint32_t sw, uint32_t slot, uint32_t row,
+                  uint32_t tw, uint32_t aux) {
+  WOp S;
+  S.off = slot;
+  S.w = sw;
+  S.lay = slay;
+  auto word = [&](uint32_t i) { return reg_of(e, wword(e, S, i, false)); };
+  auto masked = [&](const std::string &v, uint32_t bits) {
+    if (bits >= 32) return v;
+    std::string m = e.R();
+    e.l(fmt("and.b32 %s, %s, %u", m.c_str(), v.c_str(), mask_of(bits)));
+    return m;
+  };
+  switch (tcls) {
+    case CLS_U32:
+      for (uint32_t i = 0; i < tnw; i++) {
+        std::string v = word(i);
+        if (i == tnw - 1 && (tw & 31u)) v = masked(v, tw & 31u);
+        std::string ai = e.RD();
+        e.l(fmt("mad.wide.u32 %s, %%N4, %u, %%tb_n3", ai.c_str(), row + i));
+        e.l(fmt("st.global.u32 [%s], %s", ai.c_str(), v.c_str()));
+        emit_dig(e, aux + i + 1u + 0x80000000u, v);
+      }
+      return;
+    case CLS_U16:
+    case CLS_U8: {   // one byte / half-word per lane, 32 / 64 contiguous bytes
+      std::string v = masked(word(0), tw), ai = e.RD();
+      if (tcls == CLS_U8) {
+        e.l(fmt("mad.wide.u32 %s, %%N, %u, %%tbb1", ai.c_str(), row));
+        e.l(fmt("st.global.u8 [%s], %s", ai.c_str(), v.c_str()));
+      } else {
+        e.l(fmt("mad.wide.u32 %s, %%N2, %u, %%tbb2", ai.c_str(), row));
+        e.l(fmt("st.global.u16 [%s], %s", ai.c_str(), v.c_str()));
+      }
+      emit_dig(e, aux + 1u + 0x80000000u, v);
+      return;
+    }
+    default: {   // 1-bit register: bit 0 of the source, packed by ballot
+      std::string v = word(0), p = e.P(), m = e.R(), ai = e.RD();
+      e.l(fmt("setp.ne.u32 %s, %s, 0", p.c_str(), masked(v, 1).c_str()));
+      e.l(fmt("vote.sync.ballot.b32 %s, %s, 0xffffffff", m.c_str(), p.c_str()));
+      e.l(fmt("mad.wide.u32 %s, %%Nb, %u, %%tb_n0", ai.c_str(), row));
+      e.l(fmt("@%%pl0 st.global.u32 [%s], %s", ai.c_str(), m.c_str()));
+      if (e.dig) {
+        std::string b = e.R();
+        e.l(fmt("selp.u32 %s, 1, 0, %s", b.c_str(), p.c_str()));
+        emit_dig(e, aux + 1u + 0x80000000u, b);
+      }
+      return;
+    }
+  }
+}
+
 void emit_ld_const(Em &e, const Program &G, uint32_t slot, uint32_t pool, uint32_t nw, bool bcast) {
   for (uint32_t i = 0; i < nw; i++) {
     std::string v = e.R();
@@ -838,7 +893,8 @@ void emit_desc(Em &e, const Program &G, const Desc &q) {
   emit_desc_(e, G, q);
   const uint32_t code = q.x & 0xFFu;
   std::string kind = code < 32u ? "narrow" : code == CODE_WIDE ? "wide" : code == CODE_LD_CONST ? "ld_const"
-                   : (code == CODE_LD_REG || code == CODE_LD_X || code == CODE_LD_IN) ? "ld" : "st";
+                   : (code == CODE_LD_REG || code == CODE_LD_X || code == CODE_LD_IN) ? "ld"
+                   : code == CODE_ST_REGC ? "st_conv" : "st";
   if (code < 32u) kind += ((q.x >> 17) & 7u) == LC_BIT ? ":bit" : "";
   note_kind(e, kind, from);
 }
@@ -860,6 +916,9 @@ void emit_desc_(Em &e, const Program &G, const Desc &q) {
     case CODE_LD_CONST: emit_ld_const(e, G, q.y, q.z, nw, ((q.x >> 18) & 1u) != 0); break;
     case CODE_ST_REG: case CODE_ST_X: case CODE_ST_OUT:
       emit_st(e, code, cls, nw, (q.x >> 18) & 7u, q.y, q.z, q.w);
+      break;
+    case CODE_ST_REGC:
+      emit_st_conv(e, cls, nw, (q.x >> 18) & 7u, q.x >> 21, q.y, q.z & 0xFFFFFu, q.z >> 20, q.w);
       break;
     default: break;
   }
@@ -936,7 +995,7 @@ std::string step_function(const Program &G, const std::string &name, uint32_t s0
   e.lab(end);
   std::string out = func_proto(name) + "\n{\n";
   out += fmt("\t.reg .b32 %%r<%u>;\n\t.reg .b64 %%rd<%u>;\n\t.reg .pred %%p<%u>;\n", e.nr + 1, e.nrd + 1, e.np + 1);
-  out += "\t.reg .b32 %smb, %lane, %wl, %N, %rw, %rh, %rb, %N4, %N2, %Nb, %lsh;\n\t.reg .b64 ";
+  out += "\t.reg .b32 %smb, %lane, %wl, %N, %rw, %rh, %rb, %N4, %N2, %Nb, %lsh;\n\t.reg .b64 %tbb1, %tbb2, %tlw, ";
   for (int i = 0; i < kN64; i++) out += fmt("%s%%%s", i ? ", " : "", kCtx64[i]);
   out += ";\n\t.reg .pred %pl0, %pl8, %pl16, %pdig;\n";
   for (int i = 0; i < kN32; i++) out += fmt("\tld.param.u32 %%%s, [a_%s];\n", kCtx32[i], kCtx32[i]);
@@ -944,7 +1003,9 @@ std::string step_function(const Program &G, const std::string &name, uint32_t s0
   out += "\tmad.lo.u32 %rw, %lane, 4, %smb;\n\tmad.lo.u32 %rh, %lane, 2, %smb;\n\tadd.u32 %rb, %lane, %smb;\n"
          "\tshl.b32 %N4, %N, 2;\n\tshl.b32 %N2, %N, 1;\n\tshr.u32 %Nb, %N, 3;\n"
          "\tsetp.eq.u32 %pl0, %lane, 0;\n\tsetp.lt.u32 %pl8, %lane, 8;\n\tsetp.lt.u32 %pl16, %lane, 16;\n"
-         "\tsetp.ne.u64 %pdig, %dig, 0;\n\tsub.u32 %lsh, 31, %lane;\n";
+         "\tsetp.ne.u64 %pdig, %dig, 0;\n\tsub.u32 %lsh, 31, %lane;\n"
+         "\tmul.wide.u32 %tlw, %lane, 3;\n\tsub.s64 %tbb1, %tb_n1, %tlw;\n"
+         "\tmul.wide.u32 %tlw, %lane, 2;\n\tsub.s64 %tbb2, %tb_n2, %tlw;\n";
   out += e.s;
   out += "\tret;\n}\n";
   return out;

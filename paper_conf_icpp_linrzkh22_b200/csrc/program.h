@@ -48,6 +48,8 @@ enum : uint32_t {
   CODE_ST_REG = 96,     // state_next[cls][row z ..] <- slot y ; w = register word index
   CODE_ST_X = 97,       // xnet[cls][row z ..] <- slot y
   CODE_ST_OUT = 98,     // out_chunk[c][word z ..] <- slot y
+  CODE_ST_REGC = 99,    // JIT only: state_next <- slot y converted from the source's
+                        // width / layout (x >> 21) to the register's (z >> 20); z & 0xFFFFF = row
 };
 
 inline uint32_t nwords(uint32_t w) { return (w + 31u) / 32u; }
@@ -216,7 +218,7 @@ bool unrolled(uint32_t cls);
 
 // Returns RTLSIM_OK or a negative status with *err set.
 int compile_program(const rtlsim_ir *ir, uint32_t op_lanes, uint32_t smem_limit_words, Program *out,
-                    std::string *err, bool dce = true);
+                    std::string *err, bool dce = true, bool fold_conv = false);
 
 // 3-input truth table (bit k = f(a = k&1, b = k>>1&1, c = k>>2&1)) of an IR
 // opcode on 1-bit operands and a 1-bit result.

@@ -200,13 +200,14 @@ extern "C" int rtlsim_load(const rtlsim_ir *ir, const rtlsim_options *opt, rtlsi
   // tiles 0.74 ms/cycle, 8 x 2 1.08 ms, 16 x 1 3.5 ms)
   uint32_t lanes = ctx->opt.op_lanes;
   const bool dce = (ctx->opt.flags & RTLSIM_F_NO_DCE) == 0;
+  const bool fold = (ctx->opt.flags & RTLSIM_F_JIT) != 0;   // JIT-only store-with-conversion descriptors
   if (!lanes && (ctx->opt.flags & RTLSIM_F_JIT)) lanes = kJitMaxLanes;
-  int rc = compile_program(ir, lanes, smem_limit / 4u, &ctx->prog, &err, dce);
+  int rc = compile_program(ir, lanes, smem_limit / 4u, &ctx->prog, &err, dce, fold);
   if (rc == RTLSIM_OK && !ctx->opt.op_lanes && (ctx->opt.flags & RTLSIM_F_JIT) && ctx->prog.L > 1) {
     // keep the auto choice when it is smaller than the cap
     rtlsim::Program probe;
     std::string e2;
-    if (compile_program(ir, 0, smem_limit / 4u, &probe, &e2, dce) == RTLSIM_OK && probe.L < ctx->prog.L)
+    if (compile_program(ir, 0, smem_limit / 4u, &probe, &e2, dce, fold) == RTLSIM_OK && probe.L < ctx->prog.L)
       ctx->prog = std::move(probe);
   }
   if (rc != RTLSIM_OK) {
@@ -224,7 +225,7 @@ extern "C" int rtlsim_load(const rtlsim_ir *ir, const rtlsim_options *opt, rtlsi
     // spill to HBM rows)
     rtlsim::Program half;
     std::string e2;
-    if (compile_program(ir, ctx->prog.L, (smem_limit / 2u - 1024u) / 4u, &half, &e2, dce) == RTLSIM_OK)
+    if (compile_program(ir, ctx->prog.L, (smem_limit / 2u - 1024u) / 4u, &half, &e2, dce, fold) == RTLSIM_OK)
       ctx->prog = std::move(half);
   }
   // bytes after lowering: slots, the 32-word zero row (lower_program) and,
@@ -240,7 +241,7 @@ extern "C" int rtlsim_load(const rtlsim_ir *ir, const rtlsim_options *opt, rtlsi
     if (smem_limit > reserve) {
       rtlsim::Program again;
       std::string e2;
-      rc = compile_program(ir, L, (smem_limit - reserve) / 4u, &again, &e2, dce);
+      rc = compile_program(ir, L, (smem_limit - reserve) / 4u, &again, &e2, dce, fold);
       if (rc != RTLSIM_OK) {
         g_load_error = e2;
         delete ctx;
