@@ -1020,9 +1020,11 @@ std::string jit_partition_ptx(const Program &G, uint32_t q, const std::string &r
   mod += ".version 8.8\n.target sm_100a\n.address_size 64\n\n";
   mod += rt_ptx;
   mod += "\n.extern .shared .align 16 .b8 dyn_smem[];\n\n";
-  // step groups of bounded size (ptxas time is superlinear in function size)
+  // step groups of bounded size (ptxas time is superlinear in function size;
+  // 800 ops per function measured 5-10 % faster than 400: fewer call
+  // boundaries, more register forwarding)
   std::vector<std::pair<uint32_t, uint32_t>> groups;
-  static const uint64_t kGroupOps = getenv("RTLSIM_JIT_GROUP") ? strtoull(getenv("RTLSIM_JIT_GROUP"), nullptr, 10) : 400;
+  static const uint64_t kGroupOps = getenv("RTLSIM_JIT_GROUP") ? strtoull(getenv("RTLSIM_JIT_GROUP"), nullptr, 10) : 800;
   uint32_t g0 = s0;
   uint64_t acc = 0;
   for (uint32_t s = s0; s < s1; s++) {
@@ -1137,12 +1139,13 @@ int jit_build(const Program &G, const std::string &rt_ptx_path, uint32_t smem_by
       1u, std::min<uint32_t>(std::min<uint32_t>(jit_default_tiles(), 32u / std::max<uint32_t>(G.L, 1u)),
                              smem_bytes / jit_tile_bytes(G)));
   out->tmax = tmax;
-  // ptxas -O3 schedules this code ~1.8x better (config 3) but compiles ~3x
-  // slower than --Ofast-compile=mid: use it unless the design is large
-  // (RTLSIM_JIT_OPT=O3 / mid overrides)
+  // ptxas -O3 schedules this code better than --Ofast-compile=mid (config 3
+  // ~1.8x, config 4 175 vs 185 ms/cycle) but compiles ~3x slower (config 4:
+  // 116 s on 16 cores); the cubin cache amortises it (RTLSIM_JIT_OPT=O3 / mid
+  // overrides)
   const uint64_t nops = G.desc.size() + G.bitdesc.size();
   const char *lvl = getenv("RTLSIM_JIT_OPT");
-  const bool o3 = lvl ? strcmp(lvl, "O3") == 0 : nops <= 250000;
+  const bool o3 = lvl ? strcmp(lvl, "O3") == 0 : nops <= 2000000;
   out->o3 = o3;
   out->kern.assign(NP, nullptr);
   out->libs.assign(NP, nullptr);
