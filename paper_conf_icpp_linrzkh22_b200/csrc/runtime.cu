@@ -200,7 +200,7 @@ extern "C" int rtlsim_load(const rtlsim_ir *ir, const rtlsim_options *opt, rtlsi
   // tiles 0.74 ms/cycle, 8 x 2 1.08 ms, 16 x 1 3.5 ms)
   uint32_t lanes = ctx->opt.op_lanes;
   const bool dce = (ctx->opt.flags & RTLSIM_F_NO_DCE) == 0;
-  const bool fold = (ctx->opt.flags & RTLSIM_F_JIT) != 0;   // JIT-only store-with-conversion descriptors
+  const bool fold = (ctx->opt.flags & RTLSIM_F_JIT) != 0 && !getenv("RTLSIM_NO_FOLD");   // JIT-only store-with-conversion descriptors
   if (!lanes && (ctx->opt.flags & RTLSIM_F_JIT)) lanes = kJitMaxLanes;
   int rc = compile_program(ir, lanes, smem_limit / 4u, &ctx->prog, &err, dce, fold);
   if (rc == RTLSIM_OK && !ctx->opt.op_lanes && (ctx->opt.flags & RTLSIM_F_JIT) && ctx->prog.L > 1) {
