@@ -121,7 +121,10 @@ std::string lds(Em &e, uint64_t sp, uint32_t off) {
   }
   std::string r = e.R();
   e.l(fmt("ld.shared.%s %s, [%s+%u]", kSpTy[sp], r.c_str(), kSpBase[sp], off * 4));
-  if (!e.dry) e.fwd[k] = Em::Fwd{r, e.step};
+  // a read-created entry is only as good as the read itself: a write by
+  // another warp in this same step is not ordered with it, so the validity
+  // window starts one step earlier
+  if (!e.dry) e.fwd[k] = Em::Fwd{r, e.step - 1};
   return r;
 }
 // slot write from a register
@@ -852,7 +855,13 @@ void emit_bit(Em &e, const BitDesc &q) {
   std::string v[3];
   for (int k = 0; k < 3; k++) {
     v[k] = e.R();
-    if (immf & (1u << k)) e.l(fmt("mov.u32 %s, %u", v[k].c_str(), (f[k] & 1u) ? 0xFFFFFFFFu : 0u));
+    // an input the truth table ignores (unary / binary ops) is not read: a
+    // load of its placeholder slot would race with the slot's real writers
+    bool used = false;
+    for (uint32_t idx = 0; idx < 8; idx++)
+      used |= ((lut >> idx) & 1u) != ((lut >> (idx ^ (1u << k))) & 1u);
+    if (!used) e.l(fmt("mov.u32 %s, 0", v[k].c_str()));
+    else if (immf & (1u << k)) e.l(fmt("mov.u32 %s, %u", v[k].c_str(), (f[k] & 1u) ? 0xFFFFFFFFu : 0u));
     else v[k] = lds(e, SP_S, f[k]);
   }
   std::string r = e.R();
