@@ -933,13 +933,14 @@ void emit_desc_(Em &e, const Program &G, const Desc &q) {
   }
 }
 
-// forwarding distance in steps (RTLSIM_JIT_FWD; 0 disables). Off by default:
-// combined with the store-with-conversion schedule it produced wrong register
-// values in one config-4 partition (full-size parity, B200; bisected to the
-// pair), not yet explained — correctness first.
+// forwarding distance in steps (RTLSIM_JIT_FWD; 0 disables). A first version
+// let bit ops load the placeholder slot of an operand their truth table
+// ignores; that racy read seeded a stale forwarded value (wrong registers in
+// one config-4 partition; found by tools/bisect4.py, compute-sanitizer
+// racecheck and tools/fwd_hazard_check.py, fixed in emit_bit / lds).
 int32_t jit_fwd_steps() {
   const char *e = getenv("RTLSIM_JIT_FWD");
-  return e ? atoi(e) : 0;
+  return e ? atoi(e) : 2;
 }
 
 std::string func_proto(const std::string &name) {
@@ -1033,10 +1034,10 @@ std::string jit_partition_ptx(const Program &G, uint32_t q, const std::string &r
   mod += rt_ptx;
   mod += "\n.extern .shared .align 16 .b8 dyn_smem[];\n\n";
   // step groups of bounded size (ptxas time is superlinear in function size;
-  // 800 ops per function measured 5-10 % faster than 400: fewer call
-  // boundaries, more register forwarding)
+  // 1600 ops per function measured 2-5 % faster than 800, 800 5-10 % faster
+  // than 400: fewer call boundaries, more register forwarding)
   std::vector<std::pair<uint32_t, uint32_t>> groups;
-  static const uint64_t kGroupOps = getenv("RTLSIM_JIT_GROUP") ? strtoull(getenv("RTLSIM_JIT_GROUP"), nullptr, 10) : 800;
+  static const uint64_t kGroupOps = getenv("RTLSIM_JIT_GROUP") ? strtoull(getenv("RTLSIM_JIT_GROUP"), nullptr, 10) : 1600;
   uint32_t g0 = s0;
   uint64_t acc = 0;
   for (uint32_t s = s0; s < s1; s++) {
