@@ -922,6 +922,9 @@ int compile_program(const rtlsim_ir *ir, uint32_t op_lanes, uint32_t smem_limit_
           f[k] = vals[src[k]].slot;
           if (vals[src[k]].layout == LC_IMM) immf |= 1u << k;
         }
+        // operands the op does not have are immediate zeros: no evaluator
+        // reads a placeholder slot (such a read races with the slot's writer)
+        for (int k = ar; k < 3; k++) immf |= 1u << k;
         b.x = bit_lut(opc) | (immf << 8);
         b.y = D.slot | (f[0] << 16);
         b.z = f[1] | (f[2] << 16);
