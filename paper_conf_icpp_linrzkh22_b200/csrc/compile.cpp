@@ -162,6 +162,9 @@ int compile_program(const rtlsim_ir *ir, uint32_t op_lanes, uint32_t smem_limit_
     return fail(err, RTLSIM_E_ARG, "NULL array with non-zero count");
   Program &G = *P;
   G = Program();
+  // JIT schedules balance op-lanes by generated SASS (RTLSIM_OLD_COST: the
+  // interpreter's costs, for A/B)
+  const bool jcost = fold_conv && !getenv("RTLSIM_OLD_COST");
   G.n_signals = n;
   G.n_ops = ir->n_ops;
   G.n_partitions = std::max<uint32_t>(1, ir->n_partitions);
@@ -901,7 +904,7 @@ int compile_program(const rtlsim_ir *ir, uint32_t op_lanes, uint32_t smem_limit_
       }
       d.x = code | (width_class(w) << 8) | (nwords(w) << 12) | ((vals[ld.val].layout == LC_BCAST ? 1u : 0u) << 18);
       G.n_ld++;
-      steps[ld.step].lane.push_back({d, 1 + nwords(w)});
+      steps[ld.step].lane.push_back({d, jcost ? 1 + 4 * nwords(w) : 1 + nwords(w)});
     }
     // compute op -> bit-sliced, narrow or wide descriptor
     auto emit_compute = [&](uint32_t opc, int32_t vd, int ar, const int32_t *src, uint32_t imm, int32_t step) {
@@ -947,7 +950,10 @@ int compile_program(const rtlsim_ir *ir, uint32_t op_lanes, uint32_t smem_limit_
         d.w = wsrc[1] | (imm << 6) | ((ar >= 2 ? 1u : 0u) << 11) | ((ar >= 3 ? 1u : 0u) << 12) |
               (fast_handler(opc, ar, lay, D.layout, wsrc, D.width) << 13);
         G.n_narrow++;
+        // lane-balancing cost: interpreter issue slots, or (JIT schedules,
+        // fold_conv) the SASS the generated code takes (RTLSIM_JIT_STATS)
         uint32_t cost = (opc == RTLSIM_OP_DIVU || opc == RTLSIM_OP_MODU) ? 6 : 2;
+        if (jcost) cost = (opc == RTLSIM_OP_DIVU || opc == RTLSIM_OP_MODU) ? 20 : D.layout == LC_BIT ? 12 : 9;
         steps[step].lane.push_back({d, cost});
         return;
       }
@@ -968,7 +974,7 @@ int compile_program(const rtlsim_ir *ir, uint32_t op_lanes, uint32_t smem_limit_
       d.y = (uint32_t)G.wide.size();
       G.wide.push_back(r);
       G.n_wide++;
-      steps[step].lane.push_back({d, 4 + 2 * nwords(wmax)});
+      steps[step].lane.push_back({d, jcost ? 6 + 6 * nwords(wmax) : 4 + 2 * nwords(wmax)});
     };
     for (size_t j = 0; j < ops_p.size(); j++) {
       const uint32_t i = ops_p[j];
@@ -1001,13 +1007,13 @@ int compile_program(const rtlsim_ir *ir, uint32_t op_lanes, uint32_t smem_limit_
         else bytes_spill += lane_bytes(w);
       }
       d.x = sk.code | (width_class(w) << 8) | (nwords(w) << 12) | (v.layout << 18);
-      uint32_t cost = 1 + nwords(w);
+      uint32_t cost = jcost ? 5 * nwords(w) : 1 + nwords(w);
       if (sk.conv) {
         const RegInfo &ri = G.regs[sk.idx];
         if (ri.row >= (1u << 20)) return fail(err, RTLSIM_E_UNSUPPORTED, "more than 2^20 state rows in one class");
         d.x = CODE_ST_REGC | (ri.cls << 8) | (nwords(ri.width) << 12) | (v.layout << 18) | (w << 21);
         d.z = ri.row | (ri.width << 20);
-        cost = 1 + nwords(ri.width);
+        cost = jcost ? 4 + 4 * nwords(ri.width) : 1 + nwords(ri.width);
       }
       G.n_st++;
       steps[sink_step[k]].lane.push_back({d, cost});
