@@ -88,6 +88,14 @@ struct Em {
   };
   std::unordered_map<uint64_t, Fwd> fwd;
   uint32_t nr = 0, nrd = 0, np = 0, nlab = 0;
+  // N_pad the code is specialised for (0: generic, row stride from %N at run
+  // time). Specialised code addresses a state row as [window + immediate]:
+  // one 64-bit window register per arena base stays valid across the rows
+  // within the ±8 MB immediate range of LDGSTS/STG (no IMAD.WIDE + IADD3 +
+  // IADD3.X per access). Windows live within one basic block (cleared at
+  // every label) so each use is dominated by its definition.
+  uint32_t nspec = 0;
+  std::map<std::string, std::pair<std::string, int64_t>> win;   // base -> (reg, row)
   std::string R() { return fmt("%%r%u", nr++); }
   std::string RD() { return fmt("%%rd%u", nrd++); }
   std::string P() { return fmt("%%p%u", np++); }
@@ -98,12 +106,40 @@ struct Em {
     s += ";\n";
   }
   void lab(const std::string &x) {
+    win.clear();
     s += x;
     s += ":\n";
   }
 };
 
 inline uint32_t mask_of(uint32_t w) { return w >= 32 ? 0xFFFFFFFFu : ((1u << w) - 1u); }
+
+// Global address of `row` in the arena at base register `base` whose row
+// stride is `sreg` (N4 / N2 / N / Nb bytes): "reg" or "reg+imm" for [..].
+std::string gaddr(Em &e, const char *sreg, uint32_t row, const char *base) {
+  if (!e.nspec) {
+    std::string a = e.RD();
+    e.l(fmt("mad.wide.u32 %s, %%%s, %u, %%%s", a.c_str(), sreg, row, base));
+    return a;
+  }
+  const int64_t n = e.nspec;
+  const int64_t stride = !strcmp(sreg, "N4") ? 4 * n : !strcmp(sreg, "N2") ? 2 * n : !strcmp(sreg, "N") ? n : n / 8;
+  const int64_t lim = (1 << 23) - 64;   // signed 24-bit immediate, margin for the access width
+  auto off_str = [](const std::string &r, int64_t off) {
+    return off ? fmt("%s+%lld", r.c_str(), (long long)off) : r;
+  };
+  auto it = e.win.find(base);
+  if (it != e.win.end()) {
+    const int64_t off = ((int64_t)row - it->second.second) * stride;
+    if (off >= -lim && off < lim) return off_str(it->second.first, off);
+  }
+  // new window: this row plus the rows up to ~12 MB above and ~4 MB below it
+  const int64_t wrow = (int64_t)row + std::max<int64_t>(0, ((int64_t)1 << 22) / stride);
+  std::string a = e.RD();
+  e.l(fmt("add.s64 %s, %%%s, %lld", a.c_str(), base, (long long)(wrow * stride)));
+  e.win[base] = {a, wrow};
+  return off_str(a, ((int64_t)row - wrow) * stride);
+}
 
 const char *kSpBase[5] = {"", "%rw", "%rh", "%rb", "%smb"};
 const char *kSpTy[5] = {"", "u32", "u16", "u8", "u32"};
@@ -677,28 +713,27 @@ const char *kArenaTag[4] = {"c", "n", "x", "i"};   // cur, nxt, xnet, in
 
 void emit_ld(Em &e, uint32_t arena, uint32_t cls, uint32_t row, uint32_t slot, uint32_t nw) {
   const char *A = kArenaTag[arena];
-  std::string addr = e.RD();
+  std::string addr;
   switch (cls) {
     case CLS_U32:
       for (uint32_t i = 0; i < nw; i++) {
-        std::string ai = i == 0 ? addr : e.RD();
-        e.l(fmt("mad.wide.u32 %s, %%N4, %u, %%tb_%s3", ai.c_str(), row + i, A));
+        std::string ai = gaddr(e, "N4", row + i, fmt("tb_%s3", A).c_str());
         e.l(fmt("cp.async.ca.shared.global [%%rw+%u], [%s], 4", (slot + 32 * i) * 4, ai.c_str()));
         opaque_write(e, SP_W, slot + 32 * i);
       }
       break;
     case CLS_U16:
-      e.l(fmt("mad.wide.u32 %s, %%N2, %u, %%tb_%s2", addr.c_str(), row, A));
+      addr = gaddr(e, "N2", row, fmt("tb_%s2", A).c_str());
       e.l(fmt("@%%pl16 cp.async.ca.shared.global [%%rw+%u], [%s], 4", slot * 4, addr.c_str()));
       opaque_write(e, SP_H, slot);
       break;
     case CLS_U8:
-      e.l(fmt("mad.wide.u32 %s, %%N, %u, %%tb_%s1", addr.c_str(), row, A));
+      addr = gaddr(e, "N", row, fmt("tb_%s1", A).c_str());
       e.l(fmt("@%%pl8 cp.async.ca.shared.global [%%rw+%u], [%s], 4", slot * 4, addr.c_str()));
       opaque_write(e, SP_B, slot);
       break;
     default:
-      e.l(fmt("mad.wide.u32 %s, %%Nb, %u, %%tb_%s0", addr.c_str(), row, A));
+      addr = gaddr(e, "Nb", row, fmt("tb_%s0", A).c_str());
       e.l(fmt("@%%pl0 cp.async.ca.shared.global [%%smb+%u], [%s], 4", slot * 4, addr.c_str()));
       opaque_write(e, SP_S, slot);
       break;
@@ -729,20 +764,19 @@ void emit_st(Em &e, uint32_t code, uint32_t cls, uint32_t nw, uint32_t lay, uint
       } else {
         v = fetch_narrow(e, lay, slot, 32);
       }
-      std::string addr = e.RD();
-      e.l(fmt("mad.wide.u32 %s, %%N4, %u, %%outb", addr.c_str(), row + i));
+      std::string addr = gaddr(e, "N4", row + i, "outb");
       e.l(fmt("st.global.u32 [%s], %s", addr.c_str(), v.c_str()));
       emit_dig(e, row + i + 1, v);
     }
     return;
   }
   const char *A = code == CODE_ST_REG ? "n" : "x";
-  std::string addr = e.RD();
+  std::string addr;
   switch (cls) {
     case CLS_U32:
       for (uint32_t i = 0; i < nw; i++) {
-        std::string v = lds(e, SP_W, slot + 32 * i), ai = e.RD();
-        e.l(fmt("mad.wide.u32 %s, %%N4, %u, %%tb_%s3", ai.c_str(), row + i, A));
+        std::string v = lds(e, SP_W, slot + 32 * i);
+        std::string ai = gaddr(e, "N4", row + i, fmt("tb_%s3", A).c_str());
         e.l(fmt("st.global.u32 [%s], %s", ai.c_str(), v.c_str()));
         if (dg) emit_dig(e, aux + i + 1u + 0x80000000u, v);
       }
@@ -753,15 +787,14 @@ void emit_st(Em &e, uint32_t code, uint32_t cls, uint32_t nw, uint32_t lay, uint
       std::string t = e.R();
       const char *pl = cls == CLS_U8 ? "%pl8" : "%pl16";
       e.l(fmt("@%s ld.shared.u32 %s, [%%rw+%u]", pl, t.c_str(), slot * 4));
-      if (cls == CLS_U8) e.l(fmt("mad.wide.u32 %s, %%N, %u, %%tb_%s1", addr.c_str(), row, A));
-      else e.l(fmt("mad.wide.u32 %s, %%N2, %u, %%tb_%s2", addr.c_str(), row, A));
+      addr = cls == CLS_U8 ? gaddr(e, "N", row, fmt("tb_%s1", A).c_str()) : gaddr(e, "N2", row, fmt("tb_%s2", A).c_str());
       e.l(fmt("@%s st.global.u32 [%s], %s", pl, addr.c_str(), t.c_str()));
       if (dg && e.dig) emit_dig(e, aux + 1u + 0x80000000u, fetch_narrow(e, lay, slot, 16));
       return;
     }
     default: {
       std::string t = lds(e, SP_S, slot);
-      e.l(fmt("mad.wide.u32 %s, %%Nb, %u, %%tb_%s0", addr.c_str(), row, A));
+      addr = gaddr(e, "Nb", row, fmt("tb_%s0", A).c_str());
       e.l(fmt("@%%pl0 st.global.u32 [%s], %s", addr.c_str(), t.c_str()));
       if (dg && e.dig) {
         std::string b = e.R(), b2 = e.R();
@@ -794,30 +827,29 @@ void emit_st_conv(Em &e, uint32_t tcls, uint32_t tnw, uint32_t slay, uint32_t sw
       for (uint32_t i = 0; i < tnw; i++) {
         std::string v = word(i);
         if (i == tnw - 1 && (tw & 31u)) v = masked(v, tw & 31u);
-        std::string ai = e.RD();
-        e.l(fmt("mad.wide.u32 %s, %%N4, %u, %%tb_n3", ai.c_str(), row + i));
+        std::string ai = gaddr(e, "N4", row + i, "tb_n3");
         e.l(fmt("st.global.u32 [%s], %s", ai.c_str(), v.c_str()));
         emit_dig(e, aux + i + 1u + 0x80000000u, v);
       }
       return;
     case CLS_U16:
     case CLS_U8: {   // one byte / half-word per lane, 32 / 64 contiguous bytes
-      std::string v = masked(word(0), tw), ai = e.RD();
+      std::string v = masked(word(0), tw), ai;
       if (tcls == CLS_U8) {
-        e.l(fmt("mad.wide.u32 %s, %%N, %u, %%tbb1", ai.c_str(), row));
+        ai = gaddr(e, "N", row, "tbb1");
         e.l(fmt("st.global.u8 [%s], %s", ai.c_str(), v.c_str()));
       } else {
-        e.l(fmt("mad.wide.u32 %s, %%N2, %u, %%tbb2", ai.c_str(), row));
+        ai = gaddr(e, "N2", row, "tbb2");
         e.l(fmt("st.global.u16 [%s], %s", ai.c_str(), v.c_str()));
       }
       emit_dig(e, aux + 1u + 0x80000000u, v);
       return;
     }
     default: {   // 1-bit register: bit 0 of the source, packed by ballot
-      std::string v = word(0), p = e.P(), m = e.R(), ai = e.RD();
+      std::string v = word(0), p = e.P(), m = e.R();
       e.l(fmt("setp.ne.u32 %s, %s, 0", p.c_str(), masked(v, 1).c_str()));
       e.l(fmt("vote.sync.ballot.b32 %s, %s, 0xffffffff", m.c_str(), p.c_str()));
-      e.l(fmt("mad.wide.u32 %s, %%Nb, %u, %%tb_n0", ai.c_str(), row));
+      std::string ai = gaddr(e, "Nb", row, "tb_n0");
       e.l(fmt("@%%pl0 st.global.u32 [%s], %s", ai.c_str(), m.c_str()));
       if (e.dig) {
         std::string b = e.R();
@@ -955,7 +987,8 @@ std::string func_proto(const std::string &name) {
 // (bar.sync 0, counted per CTA, not per PC) inside every warp's stream — so
 // a warp's instruction fetch is sequential across steps instead of jumping
 // over the other warps' code at every step.
-std::string step_function(const Program &G, const std::string &name, uint32_t s0, uint32_t s1, bool dig) {
+std::string step_function(const Program &G, const std::string &name, uint32_t s0, uint32_t s1, bool dig,
+                          uint32_t nspec) {
   // dry pass: which warp writes which slot in which step (forwarding validity)
   WriteLog log;
   {
@@ -974,6 +1007,7 @@ std::string step_function(const Program &G, const std::string &name, uint32_t s0
   Em e;
   e.dig = dig;
   e.dry = false;
+  e.nspec = nspec;
   e.log = &log;
   e.fwd_max = jit_fwd_steps();
   std::vector<std::string> labs(G.L);
@@ -1026,7 +1060,8 @@ std::string step_function(const Program &G, const std::string &name, uint32_t s0
 
 }  // namespace
 
-std::string jit_partition_ptx(const Program &G, uint32_t q, const std::string &rt_ptx, uint32_t tmax, bool dig) {
+std::string jit_partition_ptx(const Program &G, uint32_t q, const std::string &rt_ptx, uint32_t tmax, bool dig,
+                              uint32_t nspec) {
   const uint32_t s0 = G.part_steps[q], s1 = G.part_steps[q + 1];
   std::string mod;
   mod.reserve(1 << 20);
@@ -1049,7 +1084,7 @@ std::string jit_partition_ptx(const Program &G, uint32_t q, const std::string &r
     }
   }
   for (size_t g = 0; g < groups.size(); g++)
-    mod += step_function(G, fmt("rtl_steps_%zu", g), groups[g].first, groups[g].second, dig) + "\n";
+    mod += step_function(G, fmt("rtl_steps_%zu", g), groups[g].first, groups[g].second, dig, nspec) + "\n";
   // the kernel: per-thread context, then the step functions in order
   // A CTA holds `tpc` tiles; warp g works on tile g / L as op-lane g % L, so
   // the warps of one op-lane (one per tile) run identical code in step
@@ -1064,6 +1099,8 @@ std::string jit_partition_ptx(const Program &G, uint32_t q, const std::string &r
   mod += fmt("\tld.param.u32 %%tpc, [prm+%zu];\n", offsetof(JitParams, tpc));
   mod += "\tmov.u32 %tile, %ctaid.x;\n\tmad.lo.u32 %tile, %tile, %tpc, %tsub;\n\tmad.lo.u32 %s, %tile, 32, %lane;\n";
   mod += fmt("\tld.param.u32 %%N, [prm+%zu];\n", offsetof(JitParams, N));
+  if (nspec)   // row offsets are immediates for this N_pad: refuse any other
+    mod += fmt("\t{\n\t.reg .pred %%pn;\n\tsetp.ne.u32 %%pn, %%N, %u;\n\t@%%pn trap;\n\t}\n", nspec);
   const size_t aoff[4] = {offsetof(JitParams, cur), offsetof(JitParams, nxt), offsetof(JitParams, xnet),
                           offsetof(JitParams, in)};
   const char *tag[4] = {"c", "n", "x", "i"};
@@ -1131,7 +1168,7 @@ static int compile_ptx(const std::string &ptx, bool o3, std::vector<char> *cubin
 }
 
 int jit_build(const Program &G, const std::string &rt_ptx_path, uint32_t smem_bytes, int device, JitKernels *out,
-              std::string *err, bool dig) {
+              std::string *err, bool dig, uint32_t nspec) {
   std::ifstream f(rt_ptx_path);
   if (!f) {
     *err = "cannot read " + rt_ptx_path;
@@ -1152,6 +1189,7 @@ int jit_build(const Program &G, const std::string &rt_ptx_path, uint32_t smem_by
       1u, std::min<uint32_t>(std::min<uint32_t>(jit_default_tiles(), 32u / std::max<uint32_t>(G.L, 1u)),
                              smem_bytes / jit_tile_bytes(G)));
   out->tmax = tmax;
+  out->nspec = nspec;
   // ptxas -O3 schedules this code better than --Ofast-compile=mid (config 3
   // ~1.8x, config 4 175 vs 185 ms/cycle) but compiles ~3x slower (config 4:
   // 116 s on 16 cores); the cubin cache amortises it (RTLSIM_JIT_OPT=O3 / mid
@@ -1176,7 +1214,7 @@ int jit_build(const Program &G, const std::string &rt_ptx_path, uint32_t smem_by
     th.emplace_back([&]() {
       for (uint32_t q; (q = next++) < NP;) {
         if (G.part_steps[q] == G.part_steps[q + 1]) continue;
-        std::string ptx = jit_partition_ptx(G, q, rt, tmax, dig);
+        std::string ptx = jit_partition_ptx(G, q, rt, tmax, dig, nspec);
         ptx_bytes += ptx.size();
         if (const char *dir = getenv("RTLSIM_JIT_SAVE")) {   // debugging aid: keep the module
           std::ofstream o(fmt("%s/part%u.ptx", dir, q));

@@ -44,17 +44,22 @@ struct JitKernels {
   double gen_s = 0, compile_s = 0;
   bool o3 = false;
   uint32_t tmax = 1;                // tiles per CTA the kernels were built for
+  uint32_t nspec = 0;               // N_pad the row offsets were specialised for (0: generic)
   size_t ptx_bytes = 0, cubin_bytes = 0;
   uint32_t cache_hits = 0;          // partitions served from RTLSIM_JIT_CACHE
 };
 
 // PTX text of exec-order partition q (steps part_steps[q]..part_steps[q+1]).
 // dig: include the per-(stimulus, cycle) digest code (check-mode variant).
-std::string jit_partition_ptx(const Program &G, uint32_t q, const std::string &rt_ptx, uint32_t tmax, bool dig);
+// nspec: N_pad the code is specialised for (state-row offsets become
+// immediates; the kernel traps on any other N), 0 = generic (row stride read
+// from the launch parameters).
+std::string jit_partition_ptx(const Program &G, uint32_t q, const std::string &rt_ptx, uint32_t tmax, bool dig,
+                              uint32_t nspec);
 // Generate + compile (nvPTXCompiler, all host cores) + load every partition.
 // device < 0: generate and compile only (host-only contexts, CPU tests).
 int jit_build(const Program &G, const std::string &rt_ptx_path, uint32_t smem_bytes, int device, JitKernels *out,
-              std::string *err, bool dig);
+              std::string *err, bool dig, uint32_t nspec = 0);
 void jit_free(JitKernels *k);
 
 }  // namespace rtlsim

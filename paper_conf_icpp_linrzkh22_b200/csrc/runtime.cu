@@ -116,6 +116,10 @@ struct rtlsim_ctx {
     if (e_ != cudaSuccess) return cuda_fail(ctx, e_, #call, __LINE__);                 \
   } while (0)
 
+// JIT kernels specialised for the bound N_pad (state-row offsets as
+// immediates, jit.cpp gaddr) unless RTLSIM_JIT_GENERIC is set (A/B)
+static bool jit_specialise() { return getenv("RTLSIM_JIT_GENERIC") == nullptr; }
+
 static int cuda_fail(rtlsim_ctx *ctx, cudaError_t e, const char *what, int line) {
   ctx->failed = true;
   ctx->err = std::string("CUDA error ") + cudaGetErrorString(e) + " at runtime.cu:" + std::to_string(line) +
@@ -272,10 +276,16 @@ extern "C" int rtlsim_load(const rtlsim_ir *ir, const rtlsim_options *opt, rtlsi
     ctx->jit_smem = std::max<uint32_t>(jit_tile_bytes(G), 16u);
     ctx->jit_rt_path = dir + "/jit_rt.ptx";
     ctx->jit_smem_cap = std::min<uint32_t>(ctx->jit_smem * jit_default_tiles(), smem_limit);
+    // device contexts compile at the first run, specialised for the bound
+    // N_pad (jit_ensure); RTLSIM_JIT_GENERIC=1 keeps the N-generic kernels,
+    // built here. Host-only: generic, or RTLSIM_JIT_NSPEC=<N_pad> (inspection)
+    uint32_t nspec = 0;
+    if (device < 0 && getenv("RTLSIM_JIT_NSPEC")) nspec = (uint32_t)atoi(getenv("RTLSIM_JIT_NSPEC"));
+    if (device >= 0 && jit_specialise()) return RTLSIM_OK;
     std::string jerr;
-    int jr = jit_build(G, ctx->jit_rt_path, ctx->jit_smem_cap, device, &ctx->jit, &jerr, false);
+    int jr = jit_build(G, ctx->jit_rt_path, ctx->jit_smem_cap, device, &ctx->jit, &jerr, false, nspec);
     if (jr == RTLSIM_OK && (ctx->opt.flags & RTLSIM_F_DIGEST))
-      jr = jit_build(G, ctx->jit_rt_path, ctx->jit_smem_cap, device, &ctx->jit_dig, &jerr, true);
+      jr = jit_build(G, ctx->jit_rt_path, ctx->jit_smem_cap, device, &ctx->jit_dig, &jerr, true, nspec);
     if (jr != RTLSIM_OK) g_load_error = "JIT: " + jerr;
     return jr;
   };
@@ -501,6 +511,25 @@ static EvalParams eval_params(rtlsim_ctx *ctx, int b, uint64_t cycle0, uint32_t 
   return p;
 }
 
+// JIT kernels for the bound N_pad (specialised unless RTLSIM_JIT_GENERIC):
+// built on first use and whenever a rebind changed N_pad; check-mode
+// (digest) kernels separately, on first use
+static int jit_ensure(rtlsim_ctx *ctx, bool dig) {
+  JitKernels &K = dig ? ctx->jit_dig : ctx->jit;
+  const uint32_t want = jit_specialise() ? ctx->N_pad : 0;
+  if (!K.kern.empty() && K.nspec == want) return RTLSIM_OK;
+  CK(cudaStreamSynchronize(ctx->st));
+  jit_free(&K);
+  std::string jerr;
+  int jr = jit_build(ctx->prog, ctx->jit_rt_path, ctx->jit_smem_cap, ctx->device, &K, &jerr, dig, want);
+  if (jr != RTLSIM_OK) {
+    ctx->failed = true;
+    ctx->err = std::string(dig ? "JIT (digest variant): " : "JIT: ") + jerr;
+    return jr;
+  }
+  return RTLSIM_OK;
+}
+
 // JIT: tiles per CTA — as many as the shared memory holds (up to the count
 // the kernels were compiled for) that divide the tile count; env override
 // RTLSIM_JIT_TPC for measurements
@@ -568,15 +597,9 @@ static int launch_chunk(rtlsim_ctx *ctx, int b, uint64_t cycle0, uint32_t nc, bo
     return RTLSIM_OK;
   }
   const bool jit = (ctx->opt.flags & RTLSIM_F_JIT) != 0;
-  if (jit && digest && ctx->jit_dig.kern.empty()) {
-    // check-mode kernels (digest code compiled in) on first use
-    std::string jerr;
-    int jr = jit_build(G, ctx->jit_rt_path, ctx->jit_smem_cap, ctx->device, &ctx->jit_dig, &jerr, true);
-    if (jr != RTLSIM_OK) {
-      ctx->failed = true;
-      ctx->err = "JIT (digest variant): " + jerr;
-      return jr;
-    }
+  if (jit) {   // normally built by run_impl already
+    int jr = jit_ensure(ctx, digest);
+    if (jr != RTLSIM_OK) return jr;
   }
   const JitKernels &JK = digest ? ctx->jit_dig : ctx->jit;
   // Tc x P per-(cycle, partition) kernel nodes (graph / JIT / stream modes)
@@ -675,6 +698,10 @@ static int run_impl(rtlsim_ctx *ctx, uint64_t cycles, const Dest &dst, bool dige
   const bool host_side = ctx->src != SRC_DEVICE || dst.out_host || dst.dig_host || dst.cons;
   if (host_side) {
     int rc = ensure_host_staging(ctx);
+    if (rc) return rc;
+  }
+  if (ctx->opt.flags & RTLSIM_F_JIT) {
+    int rc = jit_ensure(ctx, digest);
     if (rc) return rc;
   }
   const bool serial = (ctx->opt.flags & RTLSIM_F_NO_PIPELINE) != 0;

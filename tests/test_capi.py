@@ -199,3 +199,23 @@ def test_jit_cubin_cache(R, tmp_path, monkeypatch):
     b = R.Simulator(ir, flags=R.F_HOST_ONLY | R.F_JIT).stats()
     assert b["jit_cubin_bytes"] == a["jit_cubin_bytes"] > 0
     assert sorted(p.name for p in (tmp_path / "jc").iterdir()) == files
+
+
+def test_jit_nspec_windows(R, tmp_path, monkeypatch):
+    """N-specialised JIT code (state-row offsets as immediates from a window
+    register per arena base) compiles, differs from the generic code, and
+    carries the N_pad guard; the generic code keeps the run-time row stride."""
+    ir = designs.random_dag(7, n_ops=300, n_regs=12, n_partitions=2)
+    gen, spec = tmp_path / "g", tmp_path / "s"
+    gen.mkdir()
+    spec.mkdir()
+    monkeypatch.setenv("RTLSIM_JIT_SAVE", str(gen))
+    R.Simulator(ir, flags=R.F_HOST_ONLY | R.F_JIT)
+    monkeypatch.setenv("RTLSIM_JIT_SAVE", str(spec))
+    monkeypatch.setenv("RTLSIM_JIT_NSPEC", "4096")
+    assert R.Simulator(ir, flags=R.F_HOST_ONLY | R.F_JIT).stats()["jit_cubin_bytes"] > 0
+    g = "".join(p.read_text() for p in sorted(gen.iterdir()))
+    s = "".join(p.read_text() for p in sorted(spec.iterdir()))
+    assert "mad.wide.u32" in g and "%N4," in g and "trap" not in g
+    assert "setp.ne.u32 %pn, %N, 4096" in s and "@%pn trap" in s
+    assert "mad.wide.u32 %rd" not in s.split(".entry")[0].split("rtl_steps_0")[-1]
