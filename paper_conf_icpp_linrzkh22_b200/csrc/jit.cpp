@@ -1068,11 +1068,15 @@ std::string jit_partition_ptx(const Program &G, uint32_t q, const std::string &r
   mod += ".version 8.8\n.target sm_100a\n.address_size 64\n\n";
   mod += rt_ptx;
   mod += "\n.extern .shared .align 16 .b8 dyn_smem[];\n\n";
-  // step groups of bounded size (ptxas time is superlinear in function size;
-  // 1600 ops per function measured 2-5 % faster than 800, 800 5-10 % faster
-  // than 400: fewer call boundaries, more register forwarding)
+  // step groups of bounded size (ptxas time is superlinear in function size).
+  // Default: one function per partition. With several called functions
+  // ptxas keeps the global-memory descriptor in a uniform register only in
+  // the first one; the others hold it in a GPR pair and issue two R2UR
+  // before every LDGSTS/STG (~10 % of their SASS, config 3). 1600 ops per
+  // function was 2-5 % faster than 800, 800 5-10 % faster than 400.
   std::vector<std::pair<uint32_t, uint32_t>> groups;
-  static const uint64_t kGroupOps = getenv("RTLSIM_JIT_GROUP") ? strtoull(getenv("RTLSIM_JIT_GROUP"), nullptr, 10) : 1600;
+  static const uint64_t kGroupOps =
+      getenv("RTLSIM_JIT_GROUP") ? strtoull(getenv("RTLSIM_JIT_GROUP"), nullptr, 10) : (1ull << 40);
   uint32_t g0 = s0;
   uint64_t acc = 0;
   for (uint32_t s = s0; s < s1; s++) {
