@@ -60,6 +60,25 @@ inline uint64_t skey(uint64_t sp, uint32_t off) { return (sp << 32) | off; }
 // Writes of one step function, by (step, warp), per slot key (dry pass).
 struct WriteLog {
   std::unordered_map<uint64_t, std::vector<std::pair<int32_t, uint32_t>>> w;
+  // steps of the shared-memory reads of `key` (any warp), recorded by the
+  // probe pass for dead slot-store elimination
+  std::unordered_map<uint64_t, std::vector<int32_t>> rd;
+  // a slot store of `key` in step s is dead when no shared-memory read of
+  // the key lies in [s, next write step] (to the end if `to_end` and no later
+  // write): every reader got the value from the writer's register
+  bool dead_store(uint64_t key, int32_t s, bool to_end) const {
+    int32_t nxt = INT32_MAX;
+    auto it = w.find(key);
+    if (it != w.end())
+      for (const auto &x : it->second)
+        if (x.first > s && x.first < nxt) nxt = x.first;
+    if (nxt == INT32_MAX && !to_end) return false;
+    auto r = rd.find(key);
+    if (r == rd.end()) return true;
+    for (int32_t t : r->second)
+      if (t >= s && t <= nxt) return false;
+    return true;
+  }
   // another warp wrote `key` in steps (s0, s1]
   bool other(uint64_t key, uint32_t warp, int32_t s0, int32_t s1) const {
     auto it = w.find(key);
@@ -79,6 +98,9 @@ struct Em {
   // since. Stores are always kept (other warps / later functions read them).
   bool dry = true;           // dry pass: only record writes
   WriteLog *log = nullptr;
+  bool probe = false;        // probe pass: record shared-memory reads in log->rd
+  bool dse = false;          // drop dead slot stores (final pass, after a probe)
+  bool to_end = false;       // this function runs to the end of the partition
   int32_t step = 0;
   uint32_t warp = 0;
   int32_t fwd_max = 0;       // forwarding distance in steps (0: off)
@@ -157,6 +179,7 @@ std::string lds(Em &e, uint64_t sp, uint32_t off) {
   }
   std::string r = e.R();
   e.l(fmt("ld.shared.%s %s, [%s+%u]", kSpTy[sp], r.c_str(), kSpBase[sp], off * 4));
+  if (e.probe) e.log->rd[k].push_back(e.step);
   // a read-created entry is only as good as the read itself: a write by
   // another warp in this same step is not ordered with it, so the validity
   // window starts one step earlier
@@ -166,7 +189,8 @@ std::string lds(Em &e, uint64_t sp, uint32_t off) {
 // slot write from a register
 void sts(Em &e, uint64_t sp, uint32_t off, const std::string &r) {
   const uint64_t k = skey(sp, off);
-  e.l(fmt("st.shared.%s [%s+%u], %s", kSpTy[sp], kSpBase[sp], off * 4, r.c_str()));
+  if (!(e.dse && e.log->dead_store(k, e.step, e.to_end)))
+    e.l(fmt("st.shared.%s [%s+%u], %s", kSpTy[sp], kSpBase[sp], off * 4, r.c_str()));
   if (e.dry) e.log->w[k].push_back({e.step, e.warp});
   else e.fwd[k] = Em::Fwd{r, e.step};
 }
@@ -178,6 +202,16 @@ void opaque_write(Em &e, uint64_t sp, uint32_t off) {
 }
 uint64_t layout_space(uint32_t lay) {
   return lay == LC_U32 ? SP_W : lay == LC_U16 ? SP_H : lay == LC_U8 ? SP_B : SP_S;
+}
+// a shared-memory read that bypasses lds (direct loads, the generic path)
+void note_read(Em &e, uint64_t sp, uint32_t off) {
+  if (e.probe) e.log->rd[skey(sp, off)].push_back(e.step);
+}
+// every slot word an operand (offset, width, layout) of the generic path may read
+void note_operand_reads(Em &e, uint32_t off, uint32_t w, uint32_t lay) {
+  if (lay == LC_IMM || w == 0) return;
+  const uint64_t sp = layout_space(lay);
+  for (uint32_t i = 0; i < nwords(w); i++) note_read(e, sp, sp == SP_W ? off + 32 * i : off + i);
 }
 
 // ------------------------------------------------------------- operands --
@@ -475,6 +509,9 @@ void emit_generic_call(Em &e, uint32_t idx) {
   e.s += "\t}\n";
 }
 void generic_wide(Em &e, const WideRec &w, uint32_t idx) {
+  note_operand_reads(e, w.a, w.wa, w.lays & 0xFFu);
+  note_operand_reads(e, w.b, w.wb, (w.lays >> 8) & 0xFFu);
+  note_operand_reads(e, w.c, w.wc, (w.lays >> 16) & 0xFFu);
   emit_generic_call(e, idx);
   if (w.wd <= 32) {
     opaque_write(e, layout_space(value_layout(w.wd, false)), w.d);
@@ -787,6 +824,8 @@ void emit_st(Em &e, uint32_t code, uint32_t cls, uint32_t nw, uint32_t lay, uint
       std::string t = e.R();
       const char *pl = cls == CLS_U8 ? "%pl8" : "%pl16";
       e.l(fmt("@%s ld.shared.u32 %s, [%%rw+%u]", pl, t.c_str(), slot * 4));
+      note_read(e, cls == CLS_U8 ? SP_B : SP_H, slot);
+      note_read(e, layout_space(lay), slot);
       addr = cls == CLS_U8 ? gaddr(e, "N", row, fmt("tb_%s1", A).c_str()) : gaddr(e, "N2", row, fmt("tb_%s2", A).c_str());
       e.l(fmt("@%s st.global.u32 [%s], %s", pl, addr.c_str(), t.c_str()));
       if (dg && e.dig) emit_dig(e, aux + 1u + 0x80000000u, fetch_narrow(e, lay, slot, 16));
@@ -921,7 +960,7 @@ size_t count_lines(const std::string &s, size_t from) {
 }
 void note_kind(Em &e, const std::string &kind, size_t from) {
   static const bool on = getenv("RTLSIM_JIT_STATS") != nullptr;
-  if (!on || e.dry) return;
+  if (!on || e.dry || e.probe) return;
   std::lock_guard<std::mutex> g(g_emit_stats.mu);
   auto &x = g_emit_stats.m[kind];
   x.first++;
@@ -970,6 +1009,10 @@ void emit_desc_(Em &e, const Program &G, const Desc &q) {
 // ignores; that racy read seeded a stale forwarded value (wrong registers in
 // one config-4 partition; found by tools/bisect4.py, compute-sanitizer
 // racecheck and tools/fwd_hazard_check.py, fixed in emit_bit / lds).
+bool jit_dse() {
+  const char *e = getenv("RTLSIM_JIT_DSE");
+  return e ? atoi(e) != 0 : false;
+}
 int32_t jit_fwd_steps() {
   const char *e = getenv("RTLSIM_JIT_FWD");
   return e ? atoi(e) : 2;
@@ -988,7 +1031,7 @@ std::string func_proto(const std::string &name) {
 // a warp's instruction fetch is sequential across steps instead of jumping
 // over the other warps' code at every step.
 std::string step_function(const Program &G, const std::string &name, uint32_t s0, uint32_t s1, bool dig,
-                          uint32_t nspec) {
+                          uint32_t nspec, bool to_end) {
   // dry pass: which warp writes which slot in which step (forwarding validity)
   WriteLog log;
   {
@@ -1004,9 +1047,12 @@ std::string step_function(const Program &G, const std::string &name, uint32_t s0
         for (uint32_t k = G.step_ptr[s * G.L + w]; k < G.step_ptr[s * G.L + w + 1]; k++) emit_desc(d, G, G.desc[k]);
       }
   }
-  Em e;
+  auto emit_real = [&](Em &e, bool probe, bool dse) {
   e.dig = dig;
   e.dry = false;
+  e.probe = probe;
+  e.dse = dse;
+  e.to_end = to_end;
   e.nspec = nspec;
   e.log = &log;
   e.fwd_max = jit_fwd_steps();
@@ -1040,6 +1086,18 @@ std::string step_function(const Program &G, const std::string &name, uint32_t s0
     if (G.L > 1) e.l(fmt("bra.uni %s", end.c_str()));
   }
   e.lab(end);
+  };
+  // dead slot-store elimination (RTLSIM_JIT_DSE=1): a probe pass
+  // records which slot reads still go to shared memory once forwarding is
+  // applied; the final pass drops the stores nobody reads from there
+  Em e;
+  if (jit_dse()) {
+    Em pe;
+    emit_real(pe, true, false);
+    emit_real(e, false, true);
+  } else {
+    emit_real(e, false, false);
+  }
   std::string out = func_proto(name) + "\n{\n";
   out += fmt("\t.reg .b32 %%r<%u>;\n\t.reg .b64 %%rd<%u>;\n\t.reg .pred %%p<%u>;\n", e.nr + 1, e.nrd + 1, e.np + 1);
   out += "\t.reg .b32 %smb, %lane, %wl, %N, %rw, %rh, %rb, %N4, %N2, %Nb, %lsh;\n\t.reg .b64 %tbb1, %tbb2, %tlw, ";
@@ -1088,7 +1146,8 @@ std::string jit_partition_ptx(const Program &G, uint32_t q, const std::string &r
     }
   }
   for (size_t g = 0; g < groups.size(); g++)
-    mod += step_function(G, fmt("rtl_steps_%zu", g), groups[g].first, groups[g].second, dig, nspec) + "\n";
+    mod += step_function(G, fmt("rtl_steps_%zu", g), groups[g].first, groups[g].second, dig, nspec,
+                         groups[g].second == s1) + "\n";
   // the kernel: per-thread context, then the step functions in order
   // A CTA holds `tpc` tiles; warp g works on tile g / L as op-lane g % L, so
   // the warps of one op-lane (one per tile) run identical code in step
