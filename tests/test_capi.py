@@ -219,3 +219,21 @@ def test_jit_nspec_windows(R, tmp_path, monkeypatch):
     assert "mad.wide.u32" in g and "%N4," in g and "trap" not in g
     assert "setp.ne.u32 %pn, %N, 4096" in s and "@%pn trap" in s
     assert "mad.wide.u32 %rd" not in s.split(".entry")[0].split("rtl_steps_0")[-1]
+
+
+def test_jit_dead_store_elimination_compiles(R, tmp_path, monkeypatch):
+    """RTLSIM_JIT_DSE=1 drops slot stores whose readers all take the value
+    from the writer's register: fewer st.shared, the code still compiles,
+    every remaining ld.shared is unchanged in number (reads are not moved)."""
+    ir = designs.random_dag(11, n_ops=400, n_regs=16, n_partitions=2)
+    counts = {}
+    for dse in ("0", "1"):
+        d = tmp_path / dse
+        d.mkdir()
+        monkeypatch.setenv("RTLSIM_JIT_SAVE", str(d))
+        monkeypatch.setenv("RTLSIM_JIT_DSE", dse)
+        assert R.Simulator(ir, flags=R.F_HOST_ONLY | R.F_JIT).stats()["jit_cubin_bytes"] > 0
+        txt = "".join(p.read_text().split(".func rtl_steps_0")[-1] for p in sorted(d.iterdir()))
+        counts[dse] = (txt.count("st.shared"), txt.count("ld.shared"))
+    assert counts["1"][0] < counts["0"][0]
+    assert counts["1"][1] == counts["0"][1]
