@@ -110,9 +110,14 @@ typedef struct {
 #define RTLSIM_F_HOST_ONLY 0x8u   /* compile the schedule only; no device work
                                      (load/stats only; bind/run return E_STATE) */
 #define RTLSIM_F_JIT 0x20u        /* specialized per-partition kernels: the
-                                     schedule translated to PTX and compiled at
-                                     load (nvPTXCompiler); one launch per
-                                     (cycle, partition), graph-captured        */
+                                     schedule translated to PTX and compiled
+                                     (nvPTXCompiler) at the first rtlsim_run*
+                                     after a bind, specialised for the bound
+                                     N rounded up to 32 (a rebind with another
+                                     padded N recompiles; host-only contexts
+                                     compile N-generic code at load); one
+                                     launch per (cycle, partition),
+                                     graph-captured                           */
 #define RTLSIM_F_TIMING 0x10u     /* bracket every evaluator launch with CUDA
                                      events on the compute stream; totals in
                                      rtlsim_stats (eval_ms, eval_launches)     */
