@@ -1011,7 +1011,7 @@ void emit_desc_(Em &e, const Program &G, const Desc &q) {
 // racecheck and tools/fwd_hazard_check.py, fixed in emit_bit / lds).
 bool jit_dse() {
   const char *e = getenv("RTLSIM_JIT_DSE");
-  return e ? atoi(e) != 0 : false;
+  return e ? atoi(e) != 0 : true;
 }
 int32_t jit_fwd_steps() {
   const char *e = getenv("RTLSIM_JIT_FWD");
@@ -1087,7 +1087,7 @@ std::string step_function(const Program &G, const std::string &name, uint32_t s0
   }
   e.lab(end);
   };
-  // dead slot-store elimination (RTLSIM_JIT_DSE=1): a probe pass
+  // dead slot-store elimination (RTLSIM_JIT_DSE, default on; =0 for A/B): a probe pass
   // records which slot reads still go to shared memory once forwarding is
   // applied; the final pass drops the stores nobody reads from there
   Em e;
