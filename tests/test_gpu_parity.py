@@ -276,3 +276,20 @@ def test_mcmc_gpu_estimator(R):
     ir = shaped.generate(3, scale=0.1)
     c = MP.gpu_estimator(n_stim=256, cycles=4)(ir)
     assert c > 0
+
+
+@pytest.mark.parametrize("generic", ["0", "1"])
+def test_jit_rebind_new_n(R, oracle_lib, generic, monkeypatch):
+    """JIT kernels are specialised for the bound N_pad (row offsets as
+    immediates): one context rebound with different N recompiles and stays
+    bit-exact; RTLSIM_JIT_GENERIC=1 (run-time row stride) agrees too."""
+    if generic == "1":
+        monkeypatch.setenv("RTLSIM_JIT_GENERIC", "1")
+    ir = designs.random_dag(601, n_ops=300, n_regs=24, n_partitions=3,
+                            input_widths=(7, 33, 1, 64, 100), max_width=1024)
+    sim = R.Simulator(ir, chunk_cycles=5, flags=R.F_JIT)
+    for N in (96, 200, 33, 96):
+        st = stim.stimulus(ir, 40 + N, np.arange(N), 0, 12, mask=False)
+        sim.bind(st)
+        got = sim.run(12, out=True, regs=True, digest=N != 33)   # both kernel variants
+        assert_same(got, oracle_lib.simulate(ir, st, digest=True, threads=8), f"jit rebind N={N}")
