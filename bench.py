@@ -9,10 +9,13 @@ evaluation of every partition's ops N1, register update, output transpose N3).
 Stimulus and outputs stay in HBM for `value`; `e2e` repeats the measurement
 through the C ABI with pinned HOST buffers (H2D + D2H inside the timed region).
 
-Multi-GPU (one process per GPU under torchrun, NCCL): stimuli are sharded in
-contiguous blocks (weak scaling, 65536 per GPU: N=4 is config 5's 262144); no
-collective runs inside the timed region; the elapsed time is the max over
-ranks; an all_gather of per-rank output checksums runs after timing.
+Multi-GPU (one process per GPU under torchrun, NCCL): config 5 — the 262144
+stimuli of BASELINE.json configs[4] in contiguous blocks of 262144/G per GPU
+(strong scaling; --stimuli-per-gpu K switches to weak scaling). The run goes
+through paper_conf_icpp_linrzkh22_b200.parallel.run_sharded, the harness the
+gloo tests cover: no collective inside the timed region, the elapsed time is
+the max over ranks, and the per-stimulus register digests (N x 8 B) are
+gathered to rank 0 after timing.
 
 `--impl reference` times the CPU oracle (oracle/liboracle.so), the only
 reference this tier has, on a bounded sample of the same workload.
@@ -36,6 +39,7 @@ from rtlgen import designs, shaped, stim  # noqa: E402
 
 CONFIG_NAMES = {1: "tiny", 2: "riscv-mini-shaped", 3: "spinal-shaped", 4: "nvdla-shaped"}
 CONFIG_N = {1: 1024, 2: 4096, 3: 16384, 4: 65536}
+CONFIG5_N = 262144   # config 5: the NVDLA-shaped design sharded over 2/4/8 GPUs
 
 
 def parse():
@@ -113,27 +117,44 @@ class ClockSampler:
                 "sm_max_mhz": self.max_mhz, "reasons": sorted(self.reasons), "samples": len(self.samples)}
 
 
-def cpu_oracle_rate(ir, cid, seed, budget_s=15.0):
-    """The oracle as it stands, multi-threaded over stimuli on the host cores,
-    on a bounded sample of the same workload (stimuli 0..S-1, cycles 0..C-1)."""
+def cpu_oracle_rate(ir, cid, seed, budget_s=15.0, single_s=10.0):
+    """The oracle as it stands on a bounded sample of the same workload
+    (stimuli 0..S-1, cycles 0..C-1): multi-threaded over stimuli on all host
+    cores for ~budget_s, and single-threaded for >= single_s seconds."""
     import oracle
     d = oracle.Design(ir)
     cores = len(os.sched_getaffinity(0))
+
+    def sample(S, C):
+        if cid == 1:
+            return stim.tiny_stimulus(seed, np.arange(S), 100, 0, C)
+        return stim.stimulus(ir, seed, np.arange(S), 0, C)
     # calibrate on one stimulus-cycle
-    st1 = stim.stimulus(ir, seed, [0], 0, 1) if cid != 1 else stim.tiny_stimulus(seed, [0], 1)
     t = time.perf_counter()
-    d.simulate(st1, out=False, regs=False, threads=1)
+    d.simulate(sample(1, 1), out=False, regs=False, threads=1)
     per = max(time.perf_counter() - t, 1e-6)
+    # single thread, >= single_s seconds of simulation
+    n1 = max(1, int(single_s / per))
+    C1 = max(1, min(100, int(np.sqrt(n1))))
+    S1 = max(1, -(-n1 // C1))
+    st1 = sample(S1, C1)
+    t = time.perf_counter()
+    d.simulate(st1, out=True, regs=True, threads=1)
+    el1 = time.perf_counter() - t
+    # all cores
     total = max(cores, int(budget_s * cores / per))
     C = max(1, min(100, int(np.sqrt(total / cores))))
     S = max(cores, total // C)
-    st = stim.stimulus(ir, seed, np.arange(S), 0, C) if cid != 1 else stim.tiny_stimulus(seed, np.arange(S), 100, 0, C)
+    st = sample(S, C)
     t = time.perf_counter()
     d.simulate(st, out=True, regs=True, threads=cores)
     el = time.perf_counter() - t
     return {"value": S * C / el, "unit": "stimulus-cycles/s", "cores": cores, "kind": "oracle",
-            "sample": f"{S} stimuli x {C} cycles of the same design/seed, multi-threaded over stimuli",
-            "single_thread_value": 1.0 / per}
+            "sample": f"{S} stimuli x {C} cycles of the same design/seed, multi-threaded over stimuli "
+                      f"({el:.1f} s)",
+            "single_thread_value": S1 * C1 / el1,
+            "single_thread_sample": f"{S1} stimuli x {C1} cycles, 1 thread ({el1:.1f} s)",
+            "host": host_info()}
 
 
 def run_reference(a):
@@ -168,15 +189,37 @@ def run_reference(a):
             "config": {"workload": f"{CONFIG_NAMES[cid]} (config {cid}): CPU oracle on a bounded sample",
                        "stimuli_per_step": S, "cycles_per_step": 1},
             "cpu_baseline": {"value": v, "unit": "stimulus-cycles/s", "cores": cores, "kind": "oracle",
-                             "sample": f"{S} stimuli x 1 cycle per step"},
+                             "sample": f"{S} stimuli x 1 cycle per step", "host": host_info()},
             "e2e": {"value": v, "unit": "stimulus-cycles/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
+
+
+def host_info():
+    """CPU model, logical cores available to this process and RAM (for the
+    cpu_baseline record)."""
+    model = None
+    try:
+        for line in open("/proc/cpuinfo"):
+            if line.startswith("model name"):
+                model = line.split(":", 1)[1].strip()
+                break
+    except OSError:
+        pass
+    ram = None
+    try:
+        for line in open("/proc/meminfo"):
+            if line.startswith("MemTotal"):
+                ram = round(int(line.split()[1]) / 1024 / 1024, 1)
+                break
+    except OSError:
+        pass
+    return {"cpu_model": model, "cores": len(os.sched_getaffinity(0)), "ram_gb": ram}
 
 
 def run_ours(a):
     import torch
     import torch.distributed as dist
-    from paper_conf_icpp_linrzkh22_b200 import build, rtlsim as R
+    from paper_conf_icpp_linrzkh22_b200 import build, parallel, rtlsim as R
 
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
@@ -195,74 +238,104 @@ def run_ours(a):
             dist.barrier()
         return r
 
-    os.environ.setdefault("RTLSIM_JIT_CACHE", "/tmp/rtlsim_jit_cache")
+    os.environ.setdefault("RTLSIM_JIT_CACHE", f"/tmp/rtlsim_jit_cache-{os.getuid()}")
     staged(build.build)
     cid = a.config
-    N = a.stimuli_per_gpu or CONFIG_N[cid]
+    # N=1: config 4 (65536 stimuli). N>1: config 5 — 262144 stimuli in total
+    # over the G GPUs (strong scaling, 262144/G per GPU), unless
+    # --stimuli-per-gpu asks for weak scaling.
+    if a.stimuli_per_gpu:
+        n_total, scaling = a.stimuli_per_gpu * world, "weak"
+    elif world > 1 and cid == 4:
+        n_total, scaling = CONFIG5_N, "strong"
+    else:
+        n_total, scaling = CONFIG_N[cid] * world, "weak"
     Tc = a.cycles_per_step or (10 if cid == 4 else 100)
     ir = make_design(cid)
     seed = stim.STIM_SEED_BASE + cid
     stream = torch.cuda.Stream()
     torch.cuda.set_stream(stream)
     flags = R.F_TIMING | (R.F_GRAPH if a.graph else 0) | (R.F_JIT if a.backend == "jit" else 0)
-    t_load = time.perf_counter()
-    sim = staged(lambda: R.Simulator(ir, device=local, stream=stream.cuda_stream, chunk_cycles=Tc, flags=flags))
-    t_load = time.perf_counter() - t_load
-    st = sim.stats()
-    T = (a.warmup + a.steps) * Tc
-    s0 = rank * N
-    if cid == 1:
-        host = stim.tiny_stimulus(seed, np.arange(s0, s0 + N), T)
-        d_stim = torch.from_numpy(host.view(np.int32)).cuda()
-    else:
-        d_stim = torch.empty((N, T, ir.IW), dtype=torch.int32, device="cuda")
-        for c0 in range(0, T, Tc):     # generate in chunks to bound temporaries
-            d_stim[:, c0:c0 + Tc] = stim.stimulus_torch(ir, seed, s0, N, c0, min(Tc, T - c0))
-    out = torch.empty((N, Tc, ir.OW), dtype=torch.int32, device="cuda")
-    sim.bind_device(d_stim, N, T)
+    info = {}
 
-    def first_run():   # JIT kernels are compiled here, specialised for N_pad
-        sim.run_device(Tc, out)
-        sim.sync()
-    t_jit = time.perf_counter()
-    staged(first_run)
-    t_jit = time.perf_counter() - t_jit
-    for _ in range(a.warmup - 1):
-        sim.run_device(Tc, out)
-    sim.sync()
-    st = sim.stats()
-    torch.cuda.synchronize()
-    if world > 1:
-        dist.barrier()
-    s_before = sim.stats()
-    l_before = sim.launch_count()
-    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-    with ClockSampler(local) as clk:
-        e0.record(stream)
-        for _ in range(a.steps):
+    def simulate(s0, N):
+        """This rank's shard [s0, s0+N): device-resident stimulus, W warm-up
+        steps, K timed steps between CUDA events on the launching stream, then
+        (after timing) the per-stimulus register digests for the rank-0 gather
+        and the pinned-host e2e measurement."""
+        t_load = time.perf_counter()
+        sim = staged(lambda: R.Simulator(ir, device=local, stream=stream.cuda_stream, chunk_cycles=Tc,
+                                         flags=flags))
+        info["load_s"] = time.perf_counter() - t_load
+        T = (a.warmup + a.steps) * Tc
+        if cid == 1:
+            host = stim.tiny_stimulus(seed, np.arange(s0, s0 + N), T)
+            d_stim = torch.from_numpy(host.view(np.int32)).cuda()
+        else:
+            d_stim = torch.empty((N, T, ir.IW), dtype=torch.int32, device="cuda")
+            for c0 in range(0, T, Tc):     # generate in chunks to bound temporaries
+                d_stim[:, c0:c0 + Tc] = stim.stimulus_torch(ir, seed, s0, N, c0, min(Tc, T - c0))
+        out = torch.empty((N, Tc, ir.OW), dtype=torch.int32, device="cuda")
+        sim.bind_device(d_stim, N, T)
+
+        def first_run():   # JIT kernels are compiled here, specialised for N_pad
             sim.run_device(Tc, out)
-        e1.record(stream)
+            sim.sync()
+        t_jit = time.perf_counter()
+        staged(first_run)
+        info["first_run_s"] = time.perf_counter() - t_jit
+        for _ in range(a.warmup - 1):
+            sim.run_device(Tc, out)
+        sim.sync()
         torch.cuda.synchronize()
-    if world > 1:
-        dist.barrier()
-    ms = e0.elapsed_time(e1)
-    s_after = sim.stats()
-    launches = sim.launch_count() - l_before
-    ms_t = torch.tensor([ms], dtype=torch.float64, device="cuda")
-    if world > 1:
-        dist.all_reduce(ms_t, op=dist.ReduceOp.MAX)
-        # gather per-rank output checksums (the only collective: after timing)
-        chk = torch.tensor([int(out.view(torch.int64).sum().item()) & ((1 << 62) - 1)], device="cuda")
-        gathered = [torch.zeros_like(chk) for _ in range(world)]
-        dist.all_gather(gathered, chk)
-    ms_max = float(ms_t.item())
-    total = N * world * Tc * a.steps
+        if world > 1:
+            dist.barrier()
+        s_before = sim.stats()
+        l_before = sim.launch_count()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        with ClockSampler(local) as clk:
+            e0.record(stream)
+            for _ in range(a.steps):
+                sim.run_device(Tc, out)
+            e1.record(stream)
+            torch.cuda.synchronize()
+        if world > 1:
+            dist.barrier()
+        ms = e0.elapsed_time(e1)
+        info.update(stats=sim.stats(), s_before=s_before, launches=sim.launch_count() - l_before,
+                    clocks=clk.summary(), ms=ms, N=N)
+        # after timing: the final register state of every stimulus, as digests
+        reg_dig = sim.reg_digest()
+        # e2e: the same metric through the C ABI with pinned HOST buffers
+        if not a.no_e2e:
+            h_stim = d_stim.cpu().pin_memory()
+            del d_stim
+            h_out = torch.empty((N, Tc, ir.OW), dtype=torch.int32).pin_memory()
+            R.rtlsim_bind(sim.ctx, h_stim.numpy())
+            for _ in range(a.warmup):
+                R.rtlsim_run(sim.ctx, Tc, h_out.numpy(), None, None)
+            if world > 1:
+                dist.barrier()
+            t = time.perf_counter()
+            for _ in range(a.steps):
+                R.rtlsim_run(sim.ctx, Tc, h_out.numpy(), None, None)
+            el = torch.tensor([time.perf_counter() - t], dtype=torch.float64, device="cuda")
+            if world > 1:
+                dist.all_reduce(el, op=dist.ReduceOp.MAX)
+            info["e2e_s"] = float(el.item())
+        del sim
+        return {"elapsed": ms / 1e3, "reg_digest": reg_dig, "coverage": None}
+
+    res = parallel.run_sharded(simulate, n_total, device="cuda")
+    st, s_before, ms, N = info["stats"], info["s_before"], info["ms"], info["N"]
+    ms_max = res.elapsed_max * 1e3
+    total = n_total * Tc * a.steps
     value = total / (ms_max / 1e3)
 
     # roofline of the dominant kernel (the evaluator), measured live
-    ev_ms = s_after["eval_ms"] - s_before["eval_ms"]
-    ev_n = s_after["eval_launches"] - s_before["eval_launches"]
-    ev_sc = s_after["eval_stim_cycles"] - s_before["eval_stim_cycles"]
+    ev_ms = st["eval_ms"] - s_before["eval_ms"]
+    ev_n = st["eval_launches"] - s_before["eval_launches"]
+    ev_sc = st["eval_stim_cycles"] - s_before["eval_stim_cycles"]
     avg_ms = ev_ms / max(ev_n, 1)
     bytes_per_launch = st["b_floor"] * ev_sc / max(ev_n, 1)
     achieved = bytes_per_launch / (avg_ms / 1e3) / 1e9
@@ -273,24 +346,9 @@ def run_ours(a):
         pj = json.load(open(prof))
         if pj.get("dram_bytes_per_stim_cycle"):
             traffic = pj["dram_bytes_per_stim_cycle"] * ev_sc / max(ev_n, 1)
-
-    # e2e: same metric through the C ABI with pinned HOST buffers
     e2e = None
-    if not a.no_e2e:
-        h_stim = d_stim.cpu().pin_memory()
-        h_out = torch.empty((N, Tc, ir.OW), dtype=torch.int32).pin_memory()
-        R.rtlsim_bind(sim.ctx, h_stim.numpy())
-        for _ in range(a.warmup):
-            R.rtlsim_run(sim.ctx, Tc, h_out.numpy(), None, None)
-        if world > 1:
-            dist.barrier()
-        t = time.perf_counter()
-        for _ in range(a.steps):
-            R.rtlsim_run(sim.ctx, Tc, h_out.numpy(), None, None)
-        el = torch.tensor([time.perf_counter() - t], dtype=torch.float64, device="cuda")
-        if world > 1:
-            dist.all_reduce(el, op=dist.ReduceOp.MAX)
-        e2e = {"value": total / float(el.item()), "unit": "stimulus-cycles/s",
+    if "e2e_s" in info:
+        e2e = {"value": total / info["e2e_s"], "unit": "stimulus-cycles/s",
                "h2d_bytes_per_step": N * Tc * ir.IW * 4, "d2h_bytes_per_step": N * Tc * ir.OW * 4,
                "path": "rtlsim_bind(pinned host stim) + rtlsim_run(cycles, pinned host out)"}
 
@@ -299,22 +357,29 @@ def run_ours(a):
         cpu = cpu_oracle_rate(ir, cid, seed)
 
     if rank == 0:
+        dig = res.reg_digest
         line = {
             "metric": "stimulus-cycles/sec", "value": value, "unit": "stimulus-cycles/s",
             "n_gpus": world, "steps": a.steps, "warmup": a.warmup, "ms_per_step": ms_max / a.steps,
-            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u32",
+            "higher_is_better": True, "scaling": scaling, "vs_baseline": None, "dtype": "u32",
             "data": "synthetic",
             "config": {
-                "workload": f"{CONFIG_NAMES[cid]} (config {cid}): {st['n_ops']} ops, {st['n_partitions']} partitions, "
-                            f"{N} stimuli/GPU x {Tc} cycles per step",
-                "stimuli_per_gpu": N, "stimuli_total": N * world, "cycles_per_step": Tc,
+                "workload": (f"{CONFIG_NAMES[cid]} (config {5 if scaling == 'strong' else cid}): "
+                             f"{st['n_ops']} ops ({st['n_live_ops']} live after dead-logic elimination), "
+                             f"{st['n_partitions']} partitions, {n_total} stimuli over {world} GPU(s) "
+                             f"x {Tc} cycles per step"),
+                "stimuli_total": n_total, "stimuli_per_gpu": N, "cycles_per_step": Tc,
+                "n_ops": st["n_ops"], "n_live_ops": st["n_live_ops"], "word_ops": st["word_ops"],
+                "live_word_ops": st["live_word_ops"],
                 "design_seed": hex(stim.DESIGN_SEED_BASE + cid), "stim_seed": hex(seed),
-                "parallelism": f"stimulus shards x{world}",
+                "parallelism": f"contiguous stimulus shards x{world} (parallel.run_sharded)",
                 "schedule": "jit per-(cycle, partition) kernels, graph-launched" if a.backend == "jit"
                             else ("graph" if a.graph else "fused interpreter"),
-                "backend": a.backend, "load_s": round(t_load, 1),
-                "jit_compile_s": round(st["jit_compile_s"], 1), "first_run_s": round(t_jit, 1),
+                "backend": a.backend, "load_s": round(info["load_s"], 1),
+                "jit_compile_s": round(st["jit_compile_s"], 1), "first_run_s": round(info["first_run_s"], 1),
                 "l2": f"register state {st['b_floor'] * N / 2 / 1e9:.1f} GB per buffer >> 126 MB L2 (no flush needed)",
+                "final_reg_digest_xor": None if dig is None else hex(int(np.bitwise_xor.reduce(dig))),
+                "final_reg_digests_gathered": None if dig is None else int(dig.size),
             },
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                          "frac": achieved / peak, "traffic": traffic,
@@ -323,10 +388,9 @@ def run_ours(a):
                          "peak_source": peak_src,
                          "algorithmic_bytes_per_stim_cycle": st["b_floor"],
                          "eval_ms_per_launch": avg_ms, "eval_share_of_step": ev_ms / max(ms, 1e-9)},
-            "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": launches, "clocks": clk.summary(),
+            "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": info["launches"], "clocks": info["clocks"],
         }
         print(json.dumps(line), flush=True)
-    del sim
     if world > 1:
         dist.destroy_process_group()
 

@@ -128,6 +128,12 @@ typedef struct {
                                      rtl_eval_v4) instead of the per-descriptor
                                      interpreter; measured slower on configs
                                      3-4 (run-dispatch overhead), kept for A/B */
+#define RTLSIM_F_COVERAGE 0x200u  /* toggle coverage (N5): after every cycle,
+                                     bit j of register word k is set when it
+                                     differs between R_c and R_{c+1} in any
+                                     stimulus; read with rtlsim_coverage. The
+                                     fused interpreter then runs per-(cycle,
+                                     partition) launches (needs a cycle edge) */
 #define RTLSIM_F_NO_DCE 0x100u    /* ablation: keep dead logic. By default ops
                                      whose value reaches no register D, no
                                      output and no live op are not evaluated
@@ -176,7 +182,15 @@ typedef struct rtlsim_ctx rtlsim_ctx;
 /* Called by rtlsim_run_stream / bind_stream in cycle order.
  * producer: fill dst[N][nc][IW] (host, pinned) with stimulus cycles c0..c0+nc-1.
  * consumer: read out[N][nc][OW] (host) and digest[N][nc] (or NULL).
- * A non-zero return aborts the run with RTLSIM_E_ARG. */
+ * A non-zero return aborts the run with RTLSIM_E_ARG. The chunks already
+ * simulated stay simulated: the cycle cursor and the register state are those
+ * at the end of the last simulated chunk (for a consumer abort this can be one
+ * chunk past the refused one, whose outputs were computed; rtlsim_stats does
+ * not report the cursor — use rtlsim_reset / rtlsim_set_regs to restart from a
+ * known state). The ctx stays usable (not sticky-failed).
+ * PAPER.md §3.2.3 (Fig 11): stimulus groups flow through the
+ * set_inputs (CPU) / evaluate (GPU) pipeline; these callbacks are its CPU
+ * ends, producing inputs and consuming outputs one chunk (group) at a time. */
 typedef int (*rtlsim_producer)(void *user, uint64_t c0, uint64_t nc, uint32_t *dst);
 typedef int (*rtlsim_consumer)(void *user, uint64_t c0, uint64_t nc, const uint32_t *out,
                                const uint64_t *digest);
@@ -190,7 +204,8 @@ int rtlsim_load(const rtlsim_ir *ir, const rtlsim_options *opt, rtlsim_ctx **out
  * last run that reads it returns). Input bits above each input's width are
  * ignored (reading 15). Resets registers to reg_init and the cycle cursor to 0.
  * The stimulus is staged chunk by chunk (P:L919-963 pipeline), never copied
- * whole. */
+ * whole. N is 1..2097120 (65535 tiles of 32) per context: shard larger
+ * batches over contexts / GPUs (§8(e)); a larger N returns RTLSIM_E_ARG. */
 int rtlsim_bind(rtlsim_ctx *ctx, uint64_t N, uint64_t T, const uint32_t *stim);
 /* Same with a DEVICE pointer to stim[N][T][IW] (resident in HBM). */
 int rtlsim_bind_device(rtlsim_ctx *ctx, uint64_t N, uint64_t T, const uint32_t *stim_dev);
@@ -214,6 +229,21 @@ int rtlsim_sync(rtlsim_ctx *ctx);
 int rtlsim_get_regs(rtlsim_ctx *ctx, uint32_t *regs);
 int rtlsim_set_regs(rtlsim_ctx *ctx, const uint32_t *regs);
 int rtlsim_reset(rtlsim_ctx *ctx);
+
+/* Toggle coverage bitmap (RTLSIM_F_COVERAGE contexts): bitmap[k] (host, RW
+ * words) = OR over every simulated cycle c since the bind (or the last clear)
+ * and every stimulus s of R_c[s][k] ^ R_{c+1}[s][k] — "bit toggled in any
+ * stimulus". clear != 0 zeroes the device bitmap after reading. Multi-GPU:
+ * the bitmaps of the stimulus shards combine by bitwise OR (north star: NCCL
+ * gathers coverage; all_gather + OR, NCCL has no OR reduction). Errors:
+ * E_STATE without the flag or before bind. */
+int rtlsim_coverage(rtlsim_ctx *ctx, uint32_t *bitmap, int clear);
+/* Per-stimulus digest of the current register state, digest[s] (host, N
+ * words) = XOR_k mix(((k + 1 + 2^31) << 32) | R[s][k]) — the register half of
+ * the per-cycle DIGEST, so N x 8 bytes identify every final
+ * register state (the rank-0 gather of §8(e) collects these instead of the
+ * registers themselves). P:L1128-1129: results compared per stimulus. */
+int rtlsim_reg_digest(rtlsim_ctx *ctx, uint64_t *digest);
 
 int rtlsim_stats(const rtlsim_ctx *ctx, rtlsim_stats_t *st);
 /* Kernel launches issued by this ctx since load (for the bench's gpu_launches). */

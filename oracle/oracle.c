@@ -46,12 +46,6 @@ static unsigned nw(unsigned bits) { return (bits + 31u) / 32u; }
 static unsigned umax(unsigned a, unsigned b) { return a > b ? a : b; }
 
 static int getbit(const big_t *x, unsigned i) { return (int)((x->w[i / 32] >> (i % 32)) & 1u); }
-static void setbit(big_t *x, unsigned i, int v) {
-  if (v)
-    x->w[i / 32] |= (1u << (i % 32));
-  else
-    x->w[i / 32] &= ~(1u << (i % 32));
-}
 
 /* zero every bit at position >= bits among the first `words` words (the
  * words above are already zero) */
@@ -65,31 +59,52 @@ static void mask_range(big_t *x, unsigned bits, unsigned words) {
   }
 }
 
-/* zero every bit at position >= bits */
-static void mask_to(big_t *x, unsigned bits) { mask_range(x, bits, BIGW); }
-
 /* x := src (w_src bits) extended to `bits` bits (zero- or sign-extension),
  * or truncated when bits < w_src. Only the first max(nw(w_src), nw(bits))
- * words can be non-zero, so only those are masked. */
+ * words of x are defined (written); every reader below stays inside the
+ * words its own width defines, so no other word is ever cleared or read. */
 static void ext(big_t *x, const uint32_t *src, unsigned w_src, unsigned bits, int sign) {
-  memset(x, 0, sizeof *x);
   const unsigned n = nw(w_src), nb = nw(bits) > n ? nw(bits) : n;
-  for (unsigned i = 0; i < n; i++) x->w[i] = src[i];
+  for (unsigned i = 0; i < nb; i++) x->w[i] = i < n ? src[i] : 0u;
   mask_range(x, w_src, n);
-  if (sign && bits > w_src && getbit(x, w_src - 1))
-    for (unsigned i = w_src; i < bits; i++) setbit(x, i, 1);
+  if (sign && bits > w_src && getbit(x, w_src - 1)) /* set bits w_src .. bits-1 */
+    for (unsigned i = w_src / 32; i < nb; i++)
+      x->w[i] |= (32 * i >= w_src) ? 0xFFFFFFFFu : ~((1u << (w_src % 32)) - 1u);
   mask_range(x, bits, nb);
 }
 
-static int is_zero(const big_t *x) {
-  for (unsigned i = 0; i < BIGW; i++)
+/* r := x >> s on `words`-word values: bit i of r = bit i+s of x (0 above
+ * the x's words). r and x are distinct. */
+static void shr_words(big_t *r, const big_t *x, unsigned words, unsigned s) {
+  const unsigned q = s / 32, k = s % 32;
+  for (unsigned i = 0; i < words; i++) {
+    uint32_t lo = i + q < words ? x->w[i + q] : 0u;
+    uint32_t hi = i + q + 1 < words ? x->w[i + q + 1] : 0u;
+    r->w[i] = k ? (lo >> k) | (hi << (32 - k)) : lo;
+  }
+}
+
+/* r := x << s on `words`-word values: bit i of r = bit i-s of x (0 below
+ * s). r and x are distinct. */
+static void shl_words(big_t *r, const big_t *x, unsigned words, unsigned s) {
+  const unsigned q = s / 32, k = s % 32;
+  for (unsigned i = 0; i < words; i++) {
+    uint32_t hi = i >= q ? x->w[i - q] : 0u;
+    uint32_t lo = i >= q + 1 ? x->w[i - q - 1] : 0u;
+    r->w[i] = k ? (hi << k) | (lo >> (32 - k)) : hi;
+  }
+}
+
+/* x == 0 over its first `words` words */
+static int is_zero(const big_t *x, unsigned words) {
+  for (unsigned i = 0; i < words; i++)
     if (x->w[i]) return 0;
   return 1;
 }
 
-/* unsigned compare of two values (already extended): -1, 0, 1 */
-static int ucmp(const big_t *x, const big_t *y) {
-  for (int i = BIGW - 1; i >= 0; i--) {
+/* unsigned compare of two values (both extended to `words` words): -1, 0, 1 */
+static int ucmp(const big_t *x, const big_t *y, unsigned words) {
+  for (int i = (int)words - 1; i >= 0; i--) {
     if (x->w[i] != y->w[i]) return x->w[i] < y->w[i] ? -1 : 1;
   }
   return 0;
@@ -100,7 +115,7 @@ static int ucmp(const big_t *x, const big_t *y) {
 static uint32_t shamt(const uint32_t *b, unsigned wb) {
   big_t x;
   ext(&x, b, wb, wb, 0);
-  for (unsigned i = 1; i < BIGW; i++)
+  for (unsigned i = 1; i < nw(wb); i++)
     if (x.w[i]) return 0xFFFFFFFFu;
   return x.w[0];
 }
@@ -108,11 +123,11 @@ static uint32_t shamt(const uint32_t *b, unsigned wb) {
 static uint64_t to_u64(const uint32_t *a, unsigned wa) {
   big_t x;
   ext(&x, a, wa, wa, 0);
-  return (uint64_t)x.w[0] | ((uint64_t)x.w[1] << 32);
+  return (uint64_t)x.w[0] | (nw(wa) > 1 ? (uint64_t)x.w[1] << 32 : 0);
 }
 
+/* r's first two words := v (r is cleared by the caller) */
 static void from_u64(big_t *r, uint64_t v) {
-  memset(r, 0, sizeof *r);
   r->w[0] = (uint32_t)v;
   r->w[1] = (uint32_t)(v >> 32);
 }
@@ -126,8 +141,12 @@ int oracle_eval_op(uint32_t opc, uint32_t wd, uint32_t imm, const uint32_t *a, u
                    const uint32_t *b, uint32_t wb, const uint32_t *c, uint32_t wc,
                    uint32_t *result) {
   big_t x, y, r;
-  memset(&r, 0, sizeof r);
   unsigned W = umax(wd, umax(wa, b ? wb : 0));
+  /* words of r any case below can write: every operand width, a CONCAT of
+   * a and b, and two words for the 64-bit MUL/DIVU/MODU results */
+  unsigned RN = nw(umax(umax(W, c ? wc : 0), umax(wa + (b ? wb : 0), 64)));
+  if (RN > BIGW) RN = BIGW;
+  for (unsigned i = 0; i < RN; i++) r.w[i] = 0;
   switch (opc) {
     case ORC_COPY: /* zext(a) mod 2^wd */
       ext(&r, a, wa, wd, 0);
@@ -194,7 +213,7 @@ int oracle_eval_op(uint32_t opc, uint32_t wd, uint32_t imm, const uint32_t *a, u
       if (sg && getbit(&x, wc2 - 1) != getbit(&y, wc2 - 1))
         cmp = getbit(&x, wc2 - 1) ? -1 : 1; /* negative < non-negative */
       else
-        cmp = ucmp(&x, &y); /* same sign: two's complement order = unsigned order */
+        cmp = ucmp(&x, &y, nw(wc2)); /* same sign: two's complement order = unsigned order */
       int t = 0;
       switch (opc) {
         case ORC_EQ: t = cmp == 0; break;
@@ -211,65 +230,62 @@ int oracle_eval_op(uint32_t opc, uint32_t wd, uint32_t imm, const uint32_t *a, u
       unsigned Ws = umax(wd, wa);
       uint32_t s = shamt(b, wb);
       ext(&x, a, wa, Ws, 0);
-      if (s < wd)
-        for (unsigned i = s; i < Ws; i++) setbit(&r, i, getbit(&x, i - s));
+      if (s < wd) shl_words(&r, &x, nw(Ws), s);
       break;
     }
     case ORC_SHRL: { /* b >= W -> 0; else zext_W(a) >> b */
       unsigned Ws = umax(wd, wa);
       uint32_t s = shamt(b, wb);
       ext(&x, a, wa, Ws, 0);
-      if (s < Ws)
-        for (unsigned i = 0; i + s < Ws; i++) setbit(&r, i, getbit(&x, i + s));
+      if (s < Ws) shr_words(&r, &x, nw(Ws), s);
       break;
     }
     case ORC_SHRA: { /* x = sext_{wa->W}(a); b >= W -> all sign; else x >>a b */
+      /* bit i < W of the result is bit i+s of x, or the sign when i+s >= W:
+       * sign-extend a further, to W + min(s, W) bits, and shift right */
       unsigned Ws = umax(wd, wa);
       uint32_t s = shamt(b, wb);
-      ext(&x, a, wa, Ws, 1);
-      int sign = getbit(&x, Ws - 1);
-      for (unsigned i = 0; i < Ws; i++) {
-        int v = (s < Ws && i + s < Ws) ? getbit(&x, i + s) : sign;
-        setbit(&r, i, v);
-      }
+      if (s > Ws) s = Ws;
+      ext(&x, a, wa, Ws + s, 1);
+      shr_words(&r, &x, nw(Ws + s), s);
       break;
     }
     case ORC_MUX: /* a = select (any width), b = then, c = else */
       ext(&x, a, wa, wa, 0);
-      if (!is_zero(&x))
+      if (!is_zero(&x, nw(wa)))
         ext(&r, b, wb, wd, 0);
       else
         ext(&r, c, wc, wd, 0);
       break;
     case ORC_CONCAT: /* ((a << wb) | b) mod 2^wd */
-      ext(&x, a, wa, wa, 0);
+      ext(&x, a, wa, wa + wb, 0);
       ext(&y, b, wb, wb, 0);
-      for (unsigned i = 0; i < wb; i++) setbit(&r, i, getbit(&y, i));
-      for (unsigned i = 0; i < wa; i++) setbit(&r, wb + i, getbit(&x, i));
+      shl_words(&r, &x, nw(wa + wb), wb);
+      for (unsigned i = 0; i < nw(wb); i++) r.w[i] |= y.w[i];
       break;
     case ORC_SLICE: /* (a >> imm) mod 2^wd; imm + wd <= wa is validated */
       if (imm + wd > wa) return -1;
       ext(&x, a, wa, wa, 0);
-      for (unsigned i = 0; i < wd; i++) setbit(&r, i, getbit(&x, imm + i));
+      shr_words(&r, &x, nw(wa), imm);
       break;
     case ORC_REDAND:
     case ORC_REDOR:
-    case ORC_REDXOR: {
+    case ORC_REDXOR: { /* all / any / parity of the wa bits of a */
       ext(&x, a, wa, wa, 0);
-      int acc = opc == ORC_REDAND ? 1 : 0;
-      for (unsigned i = 0; i < wa; i++) {
-        int v = getbit(&x, i);
-        if (opc == ORC_REDAND) acc &= v;
-        else if (opc == ORC_REDOR) acc |= v;
-        else acc ^= v;
+      uint32_t all = 1, any = 0, par = 0;
+      for (unsigned i = 0; i < nw(wa); i++) {
+        uint32_t full = (32 * i + 32 <= wa) ? 0xFFFFFFFFu : (1u << (wa % 32)) - 1u;
+        all &= x.w[i] == full;
+        any |= x.w[i] != 0;
+        for (unsigned k = 0; k < 32; k++) par ^= (x.w[i] >> k) & 1u;
       }
-      r.w[0] = (uint32_t)acc;
+      r.w[0] = opc == ORC_REDAND ? all : opc == ORC_REDOR ? any : par;
       break;
     }
     default:
       return -1;
   }
-  mask_to(&r, wd); /* truncation on assignment */
+  mask_range(&r, wd, RN); /* truncation on assignment */
   for (unsigned i = 0; i < nw(wd); i++) result[i] = r.w[i];
   return 0;
 }

@@ -1081,7 +1081,11 @@ std::string step_function(const Program &G, const std::string &name, uint32_t s0
       for (uint32_t k = G.step_ptr[s * G.L + w]; k < G.step_ptr[s * G.L + w + 1]; k++) emit_desc(e, G, G.desc[k]);
       e.l("cp.async.commit_group");
       e.l(fmt("cp.async.wait_group %u", G.step_wait[s]));
-      e.l("bar.sync 0");
+      // the per-warp code blocks each hold their own copy of the step
+      // barrier, so different warps execute different barrier instructions:
+      // the non-.aligned form is required then; with one block
+      // (L == 1) every warp runs the same instruction
+      e.l(G.L > 1 ? "barrier.sync 0" : "bar.sync 0");
     }
     if (G.L > 1) e.l(fmt("bra.uni %s", end.c_str()));
   }
@@ -1265,11 +1269,22 @@ int jit_build(const Program &G, const std::string &rt_ptx_path, uint32_t smem_by
   out->libs.assign(NP, nullptr);
   std::vector<std::vector<char>> cubins(NP);
   std::vector<std::string> errs(NP);
+  std::vector<char> from_cache(NP, 0);
   std::atomic<uint32_t> next{0};
   std::atomic<size_t> ptx_bytes{0};
   std::atomic<uint32_t> cache_hits{0};
+  // RTLSIM_JIT_CACHE=dir: a private cubin cache. It is used only when it is
+  // a directory owned by this user and not writable by anyone else (cubins
+  // found there are loaded and run in this process); otherwise the
+  // kernels are compiled without a cache.
+  std::string cache_dir;
   if (const char *cdir = getenv("RTLSIM_JIT_CACHE"))
-    if (*cdir) mkdir(cdir, 0777);   // one level; an existing directory is fine
+    if (*cdir) {
+      mkdir(cdir, 0700);   // one level; an existing directory is checked below
+      struct stat sb;
+      if (stat(cdir, &sb) == 0 && S_ISDIR(sb.st_mode) && sb.st_uid == geteuid() && !(sb.st_mode & 022))
+        cache_dir = cdir;
+    }
   auto t0 = std::chrono::steady_clock::now();
   unsigned nth = std::max(1u, std::thread::hardware_concurrency());
   std::vector<std::thread> th;
@@ -1285,9 +1300,9 @@ int jit_build(const Program &G, const std::string &rt_ptx_path, uint32_t smem_by
         }
         // RTLSIM_JIT_CACHE=dir: cubins keyed by a hash of (PTX, options);
         // lets the ranks of one node (bench.py) and repeated loads share work
-        const char *cdir = getenv("RTLSIM_JIT_CACHE");
+        const char *cdir = cache_dir.c_str();
         std::string cpath;
-        if (cdir && *cdir) {
+        if (!cache_dir.empty()) {
           uint64_t h = 1469598103934665603ull;   // FNV-1a
           auto mixin = [&](const std::string &x) {
             for (unsigned char ch : x) h = (h ^ ch) * 1099511628211ull;
@@ -1300,6 +1315,7 @@ int jit_build(const Program &G, const std::string &rt_ptx_path, uint32_t smem_by
             std::vector<char> buf((std::istreambuf_iterator<char>(in)), std::istreambuf_iterator<char>());
             if (!buf.empty()) {
               cubins[q] = std::move(buf);
+              from_cache[q] = 1;
               cache_hits++;
               continue;
             }
@@ -1312,11 +1328,16 @@ int jit_build(const Program &G, const std::string &rt_ptx_path, uint32_t smem_by
           }
         } else if (!cpath.empty()) {
           const std::string tmp = cpath + fmt(".tmp%d.%u", (int)getpid(), q);
+          bool ok;
           {
             std::ofstream o(tmp, std::ios::binary);
             o.write(cubins[q].data(), (std::streamsize)cubins[q].size());
+            o.flush();
+            ok = (bool)o;
           }
-          std::rename(tmp.c_str(), cpath.c_str());
+          // only a complete file is published under the cache name
+          if (ok) ok = std::rename(tmp.c_str(), cpath.c_str()) == 0;
+          if (!ok) std::remove(tmp.c_str());
         }
       }
     });
@@ -1336,6 +1357,15 @@ int jit_build(const Program &G, const std::string &rt_ptx_path, uint32_t smem_by
     out->cubin_bytes += cubins[q].size();
     if (device < 0) continue;
     cudaError_t e = cudaLibraryLoadData(&out->libs[q], cubins[q].data(), nullptr, nullptr, 0, nullptr, nullptr, 0);
+    if (e != cudaSuccess && from_cache[q]) {   // a damaged cached cubin: compile it again
+      cudaGetLastError();
+      std::string cerr;
+      if (compile_ptx(jit_partition_ptx(G, q, rt, tmax, dig, nspec), o3, &cubins[q], &cerr) != 0) {
+        *err = fmt("partition %u: ", q) + cerr;
+        return RTLSIM_E_ARG;
+      }
+      e = cudaLibraryLoadData(&out->libs[q], cubins[q].data(), nullptr, nullptr, 0, nullptr, nullptr, 0);
+    }
     if (e == cudaSuccess) e = cudaLibraryGetKernel(&out->kern[q], out->libs[q], "rtl_jit_part");
     if (e == cudaSuccess)
       e = cudaKernelSetAttributeForDevice(out->kern[q], cudaFuncAttributeMaxDynamicSharedMemorySize,

@@ -317,8 +317,14 @@ __global__ void __launch_bounds__(512, 2) rtl_eval_kernel(const EvalParams p) {
   }
 }
 
-cudaError_t eval_set_smem(uint32_t smem_bytes) {
-  return cudaFuncSetAttribute(rtl_eval_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem_bytes);
+// The attribute is process-wide per kernel: set it to the device's opt-in
+// maximum (not the size of the context loaded last), so a context needing more
+// shared memory than one loaded after it still launches.
+cudaError_t eval_set_smem(uint32_t /*smem_bytes*/) {
+  int dev = 0, optin = 232448;
+  cudaGetDevice(&dev);
+  cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev);
+  return cudaFuncSetAttribute(rtl_eval_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, optin);
 }
 
 cudaError_t launch_eval(const EvalParams &p, uint32_t smem_bytes, cudaStream_t st) {
@@ -478,6 +484,94 @@ cudaError_t launch_regs_export(Arena a, const RegWord *map, uint32_t RW, uint32_
   return cudaGetLastError();
 }
 
+
+// ------------------------------------------------------------- N5 / digest --
+// N5 toggle coverage of one cycle: for register word k (class row m.row),
+// cov[k] |= OR over the real stimuli s < N of (R_c[s][k] ^ R_{c+1}[s][k]).
+// Grid (RW, stimulus chunks): each thread ORs 32-bit words of the two
+// arenas' rows (4 / 2 / 1 stimuli per word for u8 / u16 / u32 rows, 32 for
+// packed bit rows), padding stimuli masked out; a warp OR-reduction, then
+// one atomicOr per warp (ballot / reduce + atomicOr, NS subsystem 4).
+__global__ void toggle_coverage_kernel(Arena cur, Arena nxt, const RegWord *__restrict__ map, uint32_t N,
+                                       uint32_t N_pad, uint32_t *__restrict__ cov) {
+  const uint32_t k = blockIdx.x;
+  const RegWord m = map[k];
+  const uint32_t per = m.cls == CLS_BIT ? 32u : m.cls == CLS_U8 ? 4u : m.cls == CLS_U16 ? 2u : 1u;
+  const uint32_t words = N_pad / per;   // 32-bit words of the row
+  const uint32_t *a, *b;
+  switch (m.cls) {
+    case CLS_BIT: a = cur.bit + (size_t)m.row * (N_pad >> 5); b = nxt.bit + (size_t)m.row * (N_pad >> 5); break;
+    case CLS_U8: a = (const uint32_t *)(cur.u8 + (size_t)m.row * N_pad); b = (const uint32_t *)(nxt.u8 + (size_t)m.row * N_pad); break;
+    case CLS_U16: a = (const uint32_t *)(cur.u16 + (size_t)m.row * N_pad); b = (const uint32_t *)(nxt.u16 + (size_t)m.row * N_pad); break;
+    default: a = cur.u32 + (size_t)m.row * N_pad; b = nxt.u32 + (size_t)m.row * N_pad; break;
+  }
+  uint32_t acc = 0;
+  for (uint32_t i = blockIdx.y * blockDim.x + threadIdx.x; i < words; i += gridDim.y * blockDim.x) {
+    uint32_t t = __ldg(a + i) ^ __ldg(b + i);
+    const uint32_t s0 = i * per;                  // first stimulus of this word
+    if (s0 + per > N) {                           // mask the padding stimuli
+      const uint32_t real = s0 >= N ? 0u : N - s0;
+      const uint32_t bits_per = 32u / per;
+      t &= real * bits_per >= 32u ? 0xFFFFFFFFu : ((1u << (real * bits_per)) - 1u);
+    }
+    if (m.cls == CLS_BIT) t = t ? 1u : 0u;        // a 1-bit register: bit 0 toggled
+    else if (per > 1) {                           // fold the stimulus lanes of the word
+      const uint32_t lb = 32u / per;
+      uint32_t f = 0;
+      for (uint32_t j = 0; j < per; j++) f |= (t >> (j * lb)) & ((1u << lb) - 1u);
+      t = f;
+    }
+    acc |= t;
+  }
+  acc = __reduce_or_sync(0xFFFFFFFFu, acc);
+  if ((threadIdx.x & 31u) == 0 && acc) atomicOr(cov + k, acc);
+}
+
+cudaError_t launch_toggle_coverage(Arena cur, Arena nxt, const RegWord *map, uint32_t RW, uint32_t N,
+                                   uint32_t N_pad, uint32_t *cov, cudaStream_t st) {
+  if (RW == 0 || N == 0) return cudaSuccess;
+  const uint32_t chunks = std::min<uint32_t>(64u, (N_pad + 8191u) / 8192u);
+  toggle_coverage_kernel<<<dim3(RW, chunks), 256, 0, st>>>(cur, nxt, map, N, N_pad, cov);
+  return cudaGetLastError();
+}
+
+__device__ __forceinline__ uint64_t mix64_dev(uint64_t z) {   // splitmix64 finalizer (DIGEST)
+  z ^= z >> 30;
+  z *= 0xBF58476D1CE4E5B9ull;
+  z ^= z >> 27;
+  z *= 0x94D049BB133111EBull;
+  return z ^ (z >> 31);
+}
+
+// Per-stimulus DIGEST of the register state (the register part of the
+// per-cycle digest): dig[s] = XOR_k mix(((k+1+2^31) << 32) | R[s][k]).
+// One thread per stimulus walks the RW words; consecutive threads read
+// consecutive stimuli of a row (coalesced).
+__global__ void reg_digest_kernel(Arena a, const RegWord *__restrict__ map, uint32_t RW, uint32_t N,
+                                  uint32_t N_pad, unsigned long long *__restrict__ dig) {
+  const uint32_t s = blockIdx.x * blockDim.x + threadIdx.x;
+  if (s >= N) return;
+  uint64_t h = 0;
+  for (uint32_t k = 0; k < RW; k++) {
+    const RegWord m = map[k];
+    uint32_t v;
+    switch (m.cls) {
+      case CLS_BIT: v = (a.bit[(size_t)m.row * (N_pad >> 5) + (s >> 5)] >> (s & 31u)) & 1u; break;
+      case CLS_U8: v = a.u8[(size_t)m.row * N_pad + s]; break;
+      case CLS_U16: v = a.u16[(size_t)m.row * N_pad + s]; break;
+      default: v = a.u32[(size_t)m.row * N_pad + s]; break;
+    }
+    h ^= mix64_dev(((uint64_t)(k + 1u + 0x80000000u) << 32) | v);
+  }
+  dig[s] = h;
+}
+
+cudaError_t launch_reg_digest(Arena a, const RegWord *map, uint32_t RW, uint32_t N, uint32_t N_pad,
+                              unsigned long long *dig, cudaStream_t st) {
+  if (N == 0) return cudaSuccess;
+  reg_digest_kernel<<<(N + 255u) / 256u, 256, 0, st>>>(a, map, RW, N, N_pad, dig);
+  return cudaGetLastError();
+}
 
 // ====================================================================== v4 --
 // Run-based evaluator over the lowered micro-op stream (lower.cpp). Same tile

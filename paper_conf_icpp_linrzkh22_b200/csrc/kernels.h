@@ -80,5 +80,11 @@ cudaError_t launch_regs_import(const uint32_t *src, uint64_t src_stride, const R
 // arena -> regs[N][RW]
 cudaError_t launch_regs_export(Arena a, const RegWord *map, uint32_t RW, uint32_t N,
                                uint32_t N_pad, uint32_t *dst, cudaStream_t st);
+// N5 toggle coverage of one cycle (cov[k] |= OR_s R_c ^ R_{c+1}) and the
+// per-stimulus register digest
+cudaError_t launch_toggle_coverage(Arena cur, Arena nxt, const RegWord *map, uint32_t RW, uint32_t N,
+                                   uint32_t N_pad, uint32_t *cov, cudaStream_t st);
+cudaError_t launch_reg_digest(Arena a, const RegWord *map, uint32_t RW, uint32_t N, uint32_t N_pad,
+                              unsigned long long *dig, cudaStream_t st);
 
 }  // namespace rtlsim

@@ -88,6 +88,7 @@ struct rtlsim_ctx {
   Arena d_in[2]{};                    // class-formatted input rows [Tc][rows][N]
   InStride in_stride{};
   RegWord *d_inmap = nullptr;
+  uint32_t *d_cov = nullptr;          // RTLSIM_F_COVERAGE: [RW] toggle bitmap (N5)
   uint32_t *d_out[2]{}, *d_raw[2]{}, *d_outu[2]{};
   unsigned long long *d_dig[2]{}, *d_digu[2]{};
   uint32_t *h_in[2]{}, *h_out[2]{};
@@ -157,6 +158,7 @@ static void free_binding(rtlsim_ctx *ctx) {
     ctx->h_dig[b] = nullptr;
     ctx->ev_used[b] = false;
   }
+  ctx->d_cov = nullptr;
   ctx->src = SRC_NONE;
   ctx->N = ctx->T = ctx->cycle = 0;
   ctx->device_bytes = ctx->static_bytes;
@@ -164,6 +166,7 @@ static void free_binding(rtlsim_ctx *ctx) {
 
 
 constexpr uint32_t kJitMaxLanes = 4;
+constexpr uint64_t kMaxStimuli = 65535ull * 32ull;   // per context: transposes' grid.y bound
 
 // descriptor staging buffers start after the slots, 16-byte aligned
 static uint32_t desc_smem_off(const Program &G) { return (G.smem_words + 3u) & ~3u; }
@@ -389,7 +392,9 @@ static int reset_regs(rtlsim_ctx *ctx) {
 static int bind_common(rtlsim_ctx *ctx, uint64_t N, uint64_t T) {
   if (!ctx) return RTLSIM_E_ARG;
   if (ctx->failed || ctx->host_only) return arg_fail(ctx, RTLSIM_E_STATE, ctx->failed ? ctx->err : "host-only ctx");
-  if (N == 0 || N > (1ull << 31)) return arg_fail(ctx, RTLSIM_E_ARG, "N out of range");
+  // the N2 / N3 / digest transposes put the 32-stimulus tiles in grid.y
+  // (<= 65535 blocks): N <= 65535 * 32 stimuli per context (per GPU shard)
+  if (N == 0 || N > kMaxStimuli) return arg_fail(ctx, RTLSIM_E_ARG, "N out of range (1..2097120 per context)");
   CK(cudaSetDevice(ctx->device));
   CK(cudaStreamSynchronize(ctx->st));
   CK(cudaStreamSynchronize(ctx->st_h2d));
@@ -406,6 +411,10 @@ static int bind_common(rtlsim_ctx *ctx, uint64_t N, uint64_t T) {
   for (int b = 0; b < 2; b++)
     if ((rc = alloc_arena(ctx, &ctx->state[b], G.rows)) != RTLSIM_OK) return rc;
   if ((rc = alloc_arena(ctx, &ctx->xnet, G.xrows)) != RTLSIM_OK) return rc;
+  if ((ctx->opt.flags & RTLSIM_F_COVERAGE) && G.RW) {
+    CK(dalloc(ctx, (void **)&ctx->d_cov, (size_t)G.RW * 4, true));
+    CK(cudaMemsetAsync(ctx->d_cov, 0, (size_t)G.RW * 4, ctx->st));
+  }
   const size_t NP = ctx->N_pad, Tc = ctx->Tc;
   ctx->in_stride.s[CLS_BIT] = (uint64_t)G.in_rows[CLS_BIT] * (NP / 32);
   ctx->in_stride.s[CLS_U8] = (uint64_t)G.in_rows[CLS_U8] * NP;
@@ -533,11 +542,13 @@ static int jit_ensure(rtlsim_ctx *ctx, bool dig) {
 // JIT: tiles per CTA — as many as the shared memory holds (up to the count
 // the kernels were compiled for) that divide the tile count; env override
 // RTLSIM_JIT_TPC for measurements
-static uint32_t jit_tiles_per_cta(rtlsim_ctx *ctx) {
+static uint32_t jit_tiles_per_cta(rtlsim_ctx *ctx, const JitKernels &JK) {
   const uint32_t tiles = ctx->N_pad / 32u;
   int optin = 232448;
   cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, ctx->device);
-  uint32_t m = std::min<uint32_t>(ctx->jit.tmax, (uint32_t)optin / std::max<uint32_t>(ctx->jit_smem, 1u));
+  // the kernel set being launched (the check-mode variant may have been built
+  // with another RTLSIM_JIT_TMAX than the plain one): its .maxntid bound
+  uint32_t m = std::min<uint32_t>(JK.tmax, (uint32_t)optin / std::max<uint32_t>(ctx->jit_smem, 1u));
   if (const char *e = getenv("RTLSIM_JIT_TPC")) m = std::min<uint32_t>(m, (uint32_t)atoi(e));
   m = std::max<uint32_t>(m, 1u);
   while (m > 1 && tiles % m) m--;
@@ -586,7 +597,9 @@ static int launch_chunk(rtlsim_ctx *ctx, int b, uint64_t cycle0, uint32_t nc, bo
     CK(get_event(ctx, &tm.b));
     CK(cudaEventRecord(tm.a, ctx->st));
   }
-  if (!(ctx->opt.flags & (RTLSIM_F_GRAPH | RTLSIM_F_JIT | RTLSIM_F_STREAM))) {
+  // the fused interpreter runs a whole chunk in one launch; coverage needs a
+  // cycle boundary, so it uses the per-(cycle, partition) graph instead
+  if (!(ctx->opt.flags & (RTLSIM_F_GRAPH | RTLSIM_F_JIT | RTLSIM_F_STREAM | RTLSIM_F_COVERAGE))) {
     EvalParams p = eval_params(ctx, b, cycle0, nc, digest);
     CK(evaluator(ctx, p, ctx->st));
     ctx->launches++;
@@ -627,7 +640,7 @@ static int launch_chunk(rtlsim_ctx *ctx, int b, uint64_t cycle0, uint32_t nc, bo
           jp.digest = digest ? (uint64_t)(ctx->d_dig[b] + (size_t)c * ctx->N_pad) : 0;
           jp.wide = (uint64_t)ctx->d_wide;
           jp.N = ctx->N_pad;
-          jp.tpc = jit_tiles_per_cta(ctx);
+          jp.tpc = jit_tiles_per_cta(ctx, JK);
           void *args[] = {&jp};
           e = cudaLaunchKernel((const void *)JK.kern[q], dim3(ctx->N_pad / 32u / jp.tpc),
                                dim3(32u * G.L * jp.tpc), args, ctx->jit_smem * jp.tpc, cap);
@@ -645,6 +658,12 @@ static int launch_chunk(rtlsim_ctx *ctx, int b, uint64_t cycle0, uint32_t nc, bo
         }
         if (e != cudaSuccess) return e;
       }
+      if (ctx->d_cov) {   // N5: toggles of this cycle's register update
+        const uint32_t par = (uint32_t)(((cycle0 & 1ull) + c) & 1ull);
+        cudaError_t e = launch_toggle_coverage(ctx->state[par], ctx->state[par ^ 1u], ctx->d_regmap, G.RW,
+                                               (uint32_t)ctx->N, ctx->N_pad, ctx->d_cov, cap);
+        if (e != cudaSuccess) return e;
+      }
     }
     return cudaSuccess;
   };
@@ -652,7 +671,7 @@ static int launch_chunk(rtlsim_ctx *ctx, int b, uint64_t cycle0, uint32_t nc, bo
     // the paper's stream-based baseline (Table 4): the same per-(cycle,
     // partition) launches issued one by one every chunk, no graph
     CK(issue(ctx->st));
-    ctx->launches += (uint64_t)nc * (G.part_steps.size() - 1);
+    ctx->launches += (uint64_t)nc * (G.part_steps.size() - 1 + (ctx->d_cov ? 1 : 0));
     if (timing) {
       CK(cudaEventRecord(tm.b, ctx->st));
       ctx->timed_pending.push_back(tm);
@@ -679,7 +698,7 @@ static int launch_chunk(rtlsim_ctx *ctx, int b, uint64_t cycle0, uint32_t nc, bo
     it = ctx->graphs.emplace(key, ge).first;
   }
   CK(cudaGraphLaunch(it->second, ctx->st));
-  ctx->launches += (uint64_t)nc * (G.part_steps.size() - 1);
+  ctx->launches += (uint64_t)nc * (G.part_steps.size() - 1 + (ctx->d_cov ? 1 : 0));
   if (timing) {
     CK(cudaEventRecord(tm.b, ctx->st));
     ctx->timed_pending.push_back(tm);
@@ -715,6 +734,18 @@ static int run_impl(rtlsim_ctx *ctx, uint64_t cycles, const Dest &dst, bool dige
 
   const uint64_t nchunks = (cycles + ctx->Tc - 1) / ctx->Tc;
   std::vector<uint32_t> nc_of(nchunks);
+  // A producer / consumer abort ends the run after the chunks already
+  // simulated: the work queued for them completes, and the cycle cursor and
+  // the register state stay consistent at the end of the last simulated
+  // chunk (which can be one chunk past the one a consumer refused).
+  uint64_t simulated = 0;
+  auto aborted = [&](const char *why) -> int {
+    cudaStreamSynchronize(ctx->st_h2d);
+    cudaStreamSynchronize(ctx->st);
+    cudaStreamSynchronize(ctx->st_d2h);
+    ctx->cycle += simulated;
+    return arg_fail(ctx, RTLSIM_E_ARG, why);
+  };
   // host-side completion of chunk k (pageable outputs / consumer)
   auto finish_host = [&](uint64_t k) -> int {
     const int b = (int)(k & 1);
@@ -731,7 +762,7 @@ static int run_impl(rtlsim_ctx *ctx, uint64_t cycles, const Dest &dst, bool dige
         memcpy(dst.dig_host + s * dst.cycles + c0, ctx->h_dig[b] + s * (uint64_t)nc, (size_t)nc * 8);
     if (dst.cons) {
       if (dst.cons(dst.user, ctx->cycle0_run + c0, nc, ctx->h_out[b], digest ? (const uint64_t *)ctx->h_dig[b] : nullptr))
-        return arg_fail(ctx, RTLSIM_E_ARG, "consumer aborted");
+        return aborted("consumer aborted");
     }
     return RTLSIM_OK;
   };
@@ -763,7 +794,7 @@ static int run_impl(rtlsim_ctx *ctx, uint64_t cycles, const Dest &dst, bool dige
               memcpy(ctx->h_in[b] + s * (uint64_t)nc * IW, ctx->stim + (s * ctx->T + abs_c) * IW,
                      (size_t)nc * IW * 4);
           } else if (ctx->prod(ctx->prod_user, abs_c, nc, ctx->h_in[b])) {
-            return arg_fail(ctx, RTLSIM_E_ARG, "producer aborted");
+            return aborted("producer aborted");
           }
           hsrc = ctx->h_in[b];
           hpitch = (uint64_t)nc * IW;
@@ -785,6 +816,7 @@ static int run_impl(rtlsim_ctx *ctx, uint64_t cycles, const Dest &dst, bool dige
     if (ctx->ev_used[b]) CK(cudaStreamWaitEvent(ctx->st, ctx->ev_drain_done[b], 0));
     int rc = launch_chunk(ctx, b, abs_c, nc, digest);
     if (rc) return rc;
+    simulated += nc;
     CK(cudaEventRecord(ctx->ev_comp_done[b], ctx->st));
     if (serial) CK(cudaStreamSynchronize(ctx->st));
     // ---- C: drain (side stream)
@@ -930,6 +962,36 @@ extern "C" int rtlsim_reset(rtlsim_ctx *ctx) {
   CK(cudaSetDevice(ctx->device));
   int rc = reset_regs(ctx);
   if (rc) return rc;
+  CK(cudaStreamSynchronize(ctx->st));
+  return RTLSIM_OK;
+}
+
+extern "C" int rtlsim_coverage(rtlsim_ctx *ctx, uint32_t *bitmap, int clear) {
+  if (!ctx || !bitmap) return RTLSIM_E_ARG;
+  if (ctx->failed) return arg_fail(ctx, RTLSIM_E_STATE, ctx->err);
+  if (!(ctx->opt.flags & RTLSIM_F_COVERAGE)) return arg_fail(ctx, RTLSIM_E_STATE, "loaded without RTLSIM_F_COVERAGE");
+  if (ctx->src == SRC_NONE) return arg_fail(ctx, RTLSIM_E_STATE, "coverage before bind");
+  Program &G = ctx->prog;
+  if (!G.RW) return RTLSIM_OK;
+  CK(cudaSetDevice(ctx->device));
+  CK(cudaMemcpyAsync(bitmap, ctx->d_cov, (size_t)G.RW * 4, cudaMemcpyDeviceToHost, ctx->st));
+  if (clear) CK(cudaMemsetAsync(ctx->d_cov, 0, (size_t)G.RW * 4, ctx->st));
+  CK(cudaStreamSynchronize(ctx->st));
+  return RTLSIM_OK;
+}
+
+extern "C" int rtlsim_reg_digest(rtlsim_ctx *ctx, uint64_t *digest) {
+  if (!ctx || !digest) return RTLSIM_E_ARG;
+  if (ctx->failed) return arg_fail(ctx, RTLSIM_E_STATE, ctx->err);
+  if (ctx->src == SRC_NONE) return arg_fail(ctx, RTLSIM_E_STATE, "reg_digest before bind");
+  Program &G = ctx->prog;
+  CK(cudaSetDevice(ctx->device));
+  unsigned long long *tmp = nullptr;
+  CK(cudaMallocAsync((void **)&tmp, (size_t)ctx->N * 8, ctx->st));
+  CK(launch_reg_digest(ctx->state[ctx->cycle & 1], ctx->d_regmap, G.RW, (uint32_t)ctx->N, ctx->N_pad, tmp, ctx->st));
+  ctx->launches++;
+  CK(cudaMemcpyAsync(digest, tmp, (size_t)ctx->N * 8, cudaMemcpyDeviceToHost, ctx->st));
+  CK(cudaFreeAsync(tmp, ctx->st));
   CK(cudaStreamSynchronize(ctx->st));
   return RTLSIM_OK;
 }

@@ -23,10 +23,11 @@ STATUS = {0: "OK", -1: "E_ARG", -2: "E_IR", -3: "E_COMB_LOOP", -4: "E_UNSUPPORTE
           -6: "E_CUDA", -7: "E_STATE", -8: "E_RANGE"}
 F_DIGEST, F_NO_PIPELINE, F_GRAPH, F_HOST_ONLY, F_TIMING, F_JIT, F_V4, F_STREAM = 0x1, 0x2, 0x4, 0x8, 0x10, 0x20, 0x40, 0x80
 F_NO_DCE = 0x100
+F_COVERAGE = 0x200
 
 EXPORTS = ["rtlsim_load", "rtlsim_bind", "rtlsim_bind_device", "rtlsim_bind_stream", "rtlsim_run",
            "rtlsim_run_device", "rtlsim_run_stream", "rtlsim_sync", "rtlsim_get_regs", "rtlsim_set_regs",
-           "rtlsim_reset", "rtlsim_stats", "rtlsim_launch_count", "rtlsim_last_error", "rtlsim_free"]
+           "rtlsim_reset", "rtlsim_coverage", "rtlsim_reg_digest", "rtlsim_stats", "rtlsim_launch_count", "rtlsim_last_error", "rtlsim_free"]
 
 
 class RtlsimError(RuntimeError):
@@ -104,6 +105,8 @@ def lib():
         L.rtlsim_get_regs.argtypes = [_P, _P]
         L.rtlsim_set_regs.argtypes = [_P, _P]
         L.rtlsim_reset.argtypes = [_P]
+        L.rtlsim_coverage.argtypes = [_P, _P, c_int]
+        L.rtlsim_reg_digest.argtypes = [_P, _P]
         L.rtlsim_stats.argtypes = [_P, ctypes.POINTER(Stats)]
         L.rtlsim_launch_count.argtypes = [_P]
         L.rtlsim_launch_count.restype = u64
@@ -201,6 +204,14 @@ def rtlsim_reset(ctx):
     _check(lib().rtlsim_reset(ctx), ctx)
 
 
+def rtlsim_coverage(ctx, bitmap, clear=False):
+    _check(lib().rtlsim_coverage(ctx, _ptr(bitmap), 1 if clear else 0), ctx)
+
+
+def rtlsim_reg_digest(ctx, digest):
+    _check(lib().rtlsim_reg_digest(ctx, _ptr(digest)), ctx)
+
+
 def rtlsim_stats(ctx) -> dict:
     st = Stats()
     _check(lib().rtlsim_stats(ctx, ctypes.byref(st)), ctx)
@@ -255,6 +266,39 @@ class Simulator:
         rtlsim_bind_device(self.ctx, stim_dev, N, T)
         self.N, self.T = N, T
 
+    def bind_stream(self, N: int, T: int, produce):
+        """Producer binding: ``produce(c0, nc)`` returns the stimulus words
+        [N][nc][IW] of cycles c0..c0+nc-1 (or None to abort the run)."""
+        IW = self.IW
+
+        def _cb(_user, c0, nc, dst):
+            v = produce(int(c0), int(nc))
+            if v is None:
+                return 1
+            n = N * int(nc) * IW
+            if n:
+                np.ctypeslib.as_array(dst, shape=(n,))[:] = np.asarray(v, np.uint32).reshape(-1)
+            return 0
+
+        cb = PRODUCER(_cb)
+        self._keep = cb            # the library calls it during every run
+        rtlsim_bind_stream(self.ctx, N, T, cb)
+        self.N, self.T = N, T
+
+    def run_stream(self, cycles: int, consume):
+        """Consumer run: ``consume(c0, out[N][nc][OW], digest[N][nc] or None)``
+        is called per chunk in cycle order; a false return aborts the run."""
+        N, OW = self.N, self.OW
+
+        def _cb(_user, c0, nc, out, dig):
+            nc = int(nc)
+            o = np.ctypeslib.as_array(out, shape=(N * nc * OW,)).reshape(N, nc, OW).copy() if N * nc * OW else \
+                np.zeros((N, nc, OW), np.uint32)
+            d = np.ctypeslib.as_array(dig, shape=(N * nc,)).reshape(N, nc).copy() if dig else None
+            return 0 if consume(int(c0), o, d) else 1
+
+        rtlsim_run_stream(self.ctx, cycles, CONSUMER(_cb))
+
     def run(self, cycles: int, out=True, regs=True, digest=False):
         o = np.zeros((self.N, cycles, self.OW), np.uint32) if out else None
         r = np.zeros((self.N, self.RW), np.uint32) if regs else None
@@ -278,6 +322,16 @@ class Simulator:
 
     def reset(self):
         rtlsim_reset(self.ctx)
+
+    def coverage(self, clear=False) -> np.ndarray:
+        b = np.zeros(self.RW, np.uint32)
+        rtlsim_coverage(self.ctx, b, clear)
+        return b
+
+    def reg_digest(self) -> np.ndarray:
+        d = np.zeros(self.N, np.uint64)
+        rtlsim_reg_digest(self.ctx, d)
+        return d
 
     def launch_count(self) -> int:
         return rtlsim_launch_count(self.ctx)

@@ -107,3 +107,24 @@ def stimulus_torch(ir: I.IR, seed: int, s0: int, n: int, c0: int, nc: int, devic
         w = w & m.view(1, 1, -1)
     w = torch.where(w >= (1 << 31), w - (1 << 32), w)
     return w.to(torch.int32)
+
+
+def parity_sample(N: int, n: int, boundaries=(), seed: int = SAMPLE_SEED) -> np.ndarray:
+    """Deterministic parity sample of ``n`` stimulus indices in [0, N)
+    (SURVEY §8(c) parity policy): the warp/tile edges 0, 1, 31, 32, 33, 63,
+    64, 127, 128, 255, 256, 1023, 1024, N/2 +- 1 and N-2, N-1, every multiple
+    of each given boundary (shard / pipeline-chunk size) +- 1, then seeded
+    uniform indices until ``n`` distinct ones (all of [0, N) when n >= N).
+    Input plumbing only: shared by tools/make_golden.py and the GPU tests."""
+    if n >= N:
+        return np.arange(N, dtype=np.int64)
+    idx = {0, 1, 31, 32, 33, 63, 64, 127, 128, 255, 256, 1023, 1024,
+           N // 2 - 1, N // 2, N // 2 + 1, N - 2, N - 1}
+    for b in boundaries:
+        for m in range(b, N, b):
+            idx |= {m - 1, m, m + 1}
+    idx = {i for i in idx if 0 <= i < N}
+    rng = np.random.default_rng(seed & 0xFFFFFFFF)
+    while len(idx) < n:
+        idx |= set(int(x) for x in rng.integers(0, N, size=n - len(idx)))
+    return np.array(sorted(idx), dtype=np.int64)

@@ -7,7 +7,7 @@ ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 if ROOT not in sys.path:
     sys.path.insert(0, ROOT)
 # JIT cubins keyed by a hash of their PTX (load time only; shared with bench.py)
-os.environ.setdefault("RTLSIM_JIT_CACHE", "/tmp/rtlsim_jit_cache")
+os.environ.setdefault("RTLSIM_JIT_CACHE", f"/tmp/rtlsim_jit_cache-{os.getuid()}")
 
 
 def pytest_configure(config):

@@ -1,5 +1,5 @@
 """Quick perf probe: eval-kernel time per cycle on the shaped configs."""
-import sys, time, json
+import os, sys, time, json
 import numpy as np
 import torch
 sys.path.insert(0, '.')
@@ -14,8 +14,8 @@ for cid in cfgs:
     t0 = time.time()
     ir = designs.tiny_dut() if cid == 1 else shaped.generate(cid)
     tg = time.time() - t0
-    N = NS[cid]
-    Tc = 8 if cid == 4 else 32
+    N = int(os.environ.get('N', NS[cid]))
+    Tc = int(os.environ.get('TC', 4 if cid == 4 else 16))
     T = Tc * 4
     t0 = time.time()
     import os
@@ -38,7 +38,7 @@ for cid in cfgs:
     s1 = sim.stats()
     ems = s1['eval_ms'] - s0['eval_ms']
     stc = 3 * Tc * N
-    print(json.dumps({"cfg": cid, "env": {k: os.environ.get(k) for k in ("JIT","LANES","SMEM_KB","RTLSIM_JIT_OPT")}, "gen_s": round(tg,1), "load_s": round(tl,2), "L": st['op_lanes'], "smem_KB": st['smem_words']*4/1024,
+    print(json.dumps({"cfg": cid, "env": {k: os.environ.get(k) for k in ("JIT","LANES","SMEM_KB","RTLSIM_JIT_OPT","RTLSIM_JIT_TMAX","RTLSIM_JIT_TPC","N")}, "tpc_max_smem": 232448 // max(1, st["smem_words"]*4), "jit_s": s1["jit_compile_s"], "cubin": s1["jit_cubin_bytes"], "tpc_used": None, "gen_s": round(tg,1), "load_s": round(tl,2), "L": st['op_lanes'], "smem_KB": st['smem_words']*4/1024,
           "steps": st['n_steps'], "desc": st['n_desc'], "b_floor": st['b_floor'], "b_state": st['b_state'],
           "ms_per_cycle_total": ms / (3*Tc), "ms_per_cycle_eval": ems / (3*Tc),
           "stim_cyc_per_s": stc / (ms/1e3), "eval_GBps_floor": st['b_floor'] * stc / (ems/1e3) / 1e9}))
