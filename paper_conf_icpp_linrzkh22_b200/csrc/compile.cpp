@@ -1059,18 +1059,83 @@ int compile_program(const rtlsim_ir *ir, uint32_t op_lanes, uint32_t smem_limit_
   G.step_ptr.reserve((size_t)G.n_steps * L + 1);
   G.desc.reserve(total);
   G.bit_ptr.reserve(G.n_steps + 1);
-  for (auto &st : all_steps) {
+  // Lane affinity (JIT schedules, RTLSIM_AFFINITY != 0): an op goes to the
+  // op-lane that produced its operands in the last two steps when that lane
+  // is not overloaded, so the JIT forwards them in registers instead of a
+  // shared-memory round trip (the consumer is in the same warp).
+  const bool affinity = fold_conv && (!getenv("RTLSIM_AFFINITY") || atoi(getenv("RTLSIM_AFFINITY")) != 0);
+  std::unordered_map<uint32_t, std::pair<uint32_t, int32_t>> writer;   // slot row -> (lane, step)
+  auto rows_of = [&](uint32_t off, uint32_t lay, uint32_t w, std::vector<uint32_t> &out) {
+    if (lay == LC_IMM || w == 0) return;
+    if (lay == LC_U32)
+      for (uint32_t i = 0; i < nwords(w); i++) out.push_back(off + 32 * i);
+    else out.push_back(off);
+  };
+  auto operands = [&](const Desc &d, std::vector<uint32_t> &src, std::vector<uint32_t> &dst) {
+    const uint32_t code = d.x & 0xFFu;
+    if (code < 32u) {
+      const uint32_t la = (d.x >> 8) & 7u, lb = (d.x >> 11) & 7u, lc = (d.x >> 14) & 7u, ld = (d.x >> 17) & 7u;
+      rows_of(d.y >> 16, la, 32, src);
+      if ((d.w >> 11) & 1u) rows_of(d.z & 0xFFFFu, lb, 32, src);
+      if ((d.w >> 12) & 1u) rows_of(d.z >> 16, lc, 32, src);
+      rows_of(d.y & 0xFFFFu, ld, 32, dst);
+    } else if (code == CODE_WIDE) {
+      const WideRec &w = G.wide[d.y];
+      rows_of(w.a, w.lays & 0xFFu, w.wa, src);
+      rows_of(w.b, (w.lays >> 8) & 0xFFu, w.wb, src);
+      rows_of(w.c, (w.lays >> 16) & 0xFFu, w.wc, src);
+      rows_of(w.d, w.wd <= 32 ? value_layout(w.wd, false) : LC_U32, w.wd, dst);
+    } else if (code == CODE_ST_REG || code == CODE_ST_X || code == CODE_ST_OUT) {
+      const uint32_t nw = (d.x >> 12) & 63u, lay = (d.x >> 18) & 7u;
+      rows_of(d.y, lay, lay == LC_U32 ? 32 * nw : 32, src);
+    } else if (code == CODE_ST_REGC) {
+      const uint32_t lay = (d.x >> 18) & 7u, sw = d.x >> 21;
+      rows_of(d.y, lay, sw, src);
+    } else if (code == CODE_LD_CONST) {
+      const uint32_t nw = (d.x >> 12) & 63u;
+      if (!((d.x >> 18) & 1u)) rows_of(d.y, LC_U32, 32 * nw, dst);
+    }
+  };
+  uint32_t part_q = 0;
+  std::vector<uint32_t> srcv, dstv;
+  for (size_t si = 0; si < all_steps.size(); si++) {
+    auto &st = all_steps[si];
+    while (part_q + 1 < G.part_steps.size() && si >= G.part_steps[part_q + 1]) {
+      part_q++;
+      writer.clear();   // a partition kernel starts with no live registers
+    }
     G.bit_ptr.push_back((uint32_t)G.bitdesc.size());
     G.bitdesc.insert(G.bitdesc.end(), st.bits.begin(), st.bits.end());
-    // longest-processing-time-first onto the least loaded lane
+    // longest-processing-time-first onto the least loaded lane (or the
+    // producer's lane, within a slack)
     std::stable_sort(st.lane.begin(), st.lane.end(),
                      [](const std::pair<Desc, uint32_t> &x, const std::pair<Desc, uint32_t> &y) {
                        return x.second > y.second;
                      });
     std::vector<std::vector<Desc>> lanes(L);
     std::vector<uint64_t> load(L, 0);
+    uint64_t step_cost = 0;
+    for (auto &sd : st.lane) step_cost += sd.second;
+    const uint64_t slack = std::max<uint64_t>(8, step_cost / L / 6);
+    std::vector<uint32_t> score(L);
     for (auto &sd : st.lane) {
       uint32_t best = (uint32_t)(std::min_element(load.begin(), load.end()) - load.begin());
+      srcv.clear();
+      dstv.clear();
+      if (affinity && L > 1) {
+        operands(sd.first, srcv, dstv);
+        std::fill(score.begin(), score.end(), 0u);
+        for (uint32_t r : srcv) {
+          auto it = writer.find(r);
+          if (it != writer.end() && (int32_t)si - it->second.second <= 2) score[it->second.first]++;
+        }
+        const uint64_t lim = load[best] + slack;
+        uint32_t pick = best;
+        for (uint32_t l = 0; l < L; l++)
+          if (load[l] <= lim && (score[l] > score[pick] || (score[l] == score[pick] && load[l] < load[pick]))) pick = l;
+        best = pick;
+        for (uint32_t r : dstv) writer[r] = {best, (int32_t)si};
+      }
       lanes[best].push_back(sd.first);
       load[best] += sd.second;
     }

@@ -12,6 +12,7 @@
 #include <nvPTXCompiler.h>
 
 #include <algorithm>
+#include <array>
 #include <atomic>
 #include <chrono>
 #include <cstdarg>
@@ -47,11 +48,22 @@ std::string fmt(const char *f, ...) {
 }
 
 // context values passed from the kernel to every step function
-const char *kCtx32[] = {"smb", "lane", "wl", "N"};
+const char *kCtx32[] = {"smb", "lane", "wl", "N", "tbar"};
 const char *kCtx64[] = {"tb_c0", "tb_c1", "tb_c2", "tb_c3", "tb_n0", "tb_n1", "tb_n2", "tb_n3",
                         "tb_x0", "tb_x1", "tb_x2", "tb_x3", "tb_i0", "tb_i1", "tb_i2", "tb_i3",
                         "outb", "dig", "wide", "smg"};
-constexpr int kN32 = 4, kN64 = 20;
+constexpr int kN32 = 5, kN64 = 20;
+
+// Step barrier (RTLSIM_JIT_TBAR, read per build): 0 = one CTA-wide barrier
+// per step (all K tiles x L op-lanes); 1 = a named barrier per tile (id
+// 1 + tile, 32 L threads), so the tiles of a CTA do not wait for each other
+// (with L == 1 a tile is one warp and the step edge is only a warp barrier);
+// 2 = the CTA-wide barrier in its non-.aligned form (A/B, see the step loop).
+// Measured on config 3 (profiles/r02_sweep_b.log): 1 is no faster than 0.
+int jit_tbar() {
+  const char *e = getenv("RTLSIM_JIT_TBAR");
+  return e ? atoi(e) : 0;
+}
 
 // Shared-memory slot keys for register forwarding: (space, word offset).
 enum : uint64_t { SP_W = 1, SP_H = 2, SP_B = 3, SP_S = 4 };   // [%rw] [%rh] [%rb] [%smb]
@@ -107,7 +119,27 @@ struct Em {
   struct Fwd {
     std::string reg;
     int32_t step;
+    uint64_t op;               // op counter at the write (register-budget forwarding)
   };
+  uint64_t opn = 0;            // descriptors emitted so far in this pass
+  uint64_t fwd_ops = UINT64_MAX;   // forward only within this many ops (register budget)
+  // ---- slot compaction (one op-lane): every value written to a slot is an
+  // instance living from its defining step to its last shared-memory read;
+  // only instances read back from shared memory (or written opaquely by
+  // cp.async / the generic path) get space, allocated between the probe pass
+  // and the final pass; the final pass emits the compacted offsets.
+  struct Inst {
+    uint32_t off, words;       // original slot words [off, off + words)
+    int32_t s0, s1;            // defining step, last shared-memory read step
+    bool need;                 // read from shared memory or written opaquely
+    bool opq;                  // written opaquely (cp.async load / generic path)
+    uint32_t nb;               // compacted offset (final pass)
+  };
+  bool compact = false;
+  std::vector<Inst> *inst = nullptr;        // shared by the probe and final passes
+  uint32_t ninst = 0;                       // instances begun in this pass
+  std::unordered_map<uint64_t, uint32_t> cur;   // row key -> current instance
+  std::vector<WideRec> *wrec = nullptr;     // generic-path records with compacted offsets
   std::unordered_map<uint64_t, Fwd> fwd;
   uint32_t nr = 0, nrd = 0, np = 0, nlab = 0;
   // N_pad the code is specialised for (0: generic, row stride from %N at run
@@ -163,6 +195,45 @@ std::string gaddr(Em &e, const char *sreg, uint32_t row, const char *base) {
   return off_str(a, ((int64_t)row - wrow) * stride);
 }
 
+// words of one row (the unit a slot key addresses) per space
+inline uint32_t sp_row_words(uint64_t sp) { return sp == SP_W ? 32u : sp == SP_H ? 16u : sp == SP_B ? 8u : 1u; }
+
+// A value of `rows` rows (row keys off, off + stride, ...) is about to be
+// written: start its instance (compaction). Safe at the start of a
+// descriptor: the schedule never gives a value the slot of an operand that is
+// still live in the same step.
+void begin_value(Em &e, uint64_t sp, uint32_t off, uint32_t rows, bool opaque = false) {
+  if (!e.compact || e.dry) return;
+  const uint32_t stride = sp == SP_W ? 32u : 1u;
+  const uint32_t id = e.ninst++;
+  if (e.probe) {
+    if (e.inst->size() <= id) e.inst->resize(id + 1);
+    (*e.inst)[id] = Em::Inst{off, stride * (rows - 1) + sp_row_words(sp), e.step, e.step, opaque, opaque, 0};
+  }
+  for (uint32_t i = 0; i < rows; i++) e.cur[skey(sp, off + stride * i)] = id;
+}
+// the instance holding row key (sp, off), or -1 (never written: keep the offset)
+int64_t inst_of(Em &e, uint64_t sp, uint32_t off) {
+  if (!e.compact || e.dry) return -1;
+  auto it = e.cur.find(skey(sp, off));
+  return it == e.cur.end() ? -1 : (int64_t)it->second;
+}
+// a shared-memory read of row (sp, off): extends the instance (probe pass)
+void inst_read(Em &e, uint64_t sp, uint32_t off) {
+  const int64_t id = inst_of(e, sp, off);
+  if (id < 0 || !e.probe) return;
+  Em::Inst &I = (*e.inst)[(size_t)id];
+  I.need = true;
+  I.s1 = std::max(I.s1, e.step);
+}
+// the word offset to emit for row (sp, off)
+uint32_t xoff(Em &e, uint64_t sp, uint32_t off) {
+  const int64_t id = inst_of(e, sp, off);
+  if (id < 0 || e.probe) return off;
+  const Em::Inst &I = (*e.inst)[(size_t)id];
+  return I.nb + (off - I.off);
+}
+
 const char *kSpBase[5] = {"", "%rw", "%rh", "%rb", "%smb"};
 const char *kSpTy[5] = {"", "u32", "u16", "u8", "u32"};
 
@@ -172,33 +243,39 @@ std::string lds(Em &e, uint64_t sp, uint32_t off) {
   if (!e.dry && e.fwd_max > 0) {
     auto it = e.fwd.find(k);
     if (it != e.fwd.end()) {
-      if (e.step - it->second.step <= e.fwd_max && !e.log->other(k, e.warp, it->second.step, e.step))
+      if (e.step - it->second.step <= e.fwd_max && e.opn - it->second.op <= e.fwd_ops &&
+          !e.log->other(k, e.warp, it->second.step, e.step))
         return it->second.reg;
       e.fwd.erase(it);
     }
   }
   std::string r = e.R();
-  e.l(fmt("ld.shared.%s %s, [%s+%u]", kSpTy[sp], r.c_str(), kSpBase[sp], off * 4));
+  e.l(fmt("ld.shared.%s %s, [%s+%u]", kSpTy[sp], r.c_str(), kSpBase[sp], xoff(e, sp, off) * 4));
   if (e.probe) e.log->rd[k].push_back(e.step);
+  inst_read(e, sp, off);
   // a read-created entry is only as good as the read itself: a write by
   // another warp in this same step is not ordered with it, so the validity
   // window starts one step earlier
-  if (!e.dry) e.fwd[k] = Em::Fwd{r, e.step - 1};
+  if (!e.dry) e.fwd[k] = Em::Fwd{r, e.step - 1, e.opn};
   return r;
 }
 // slot write from a register
 void sts(Em &e, uint64_t sp, uint32_t off, const std::string &r) {
   const uint64_t k = skey(sp, off);
-  if (!(e.dse && e.log->dead_store(k, e.step, e.to_end)))
-    e.l(fmt("st.shared.%s [%s+%u], %s", kSpTy[sp], kSpBase[sp], off * 4, r.c_str()));
+  const int64_t id = inst_of(e, sp, off);
+  const bool unread = id >= 0 && !e.probe && !(*e.inst)[(size_t)id].need;   // compacted away
+  if (!unread && !(e.dse && e.log->dead_store(k, e.step, e.to_end)))
+    e.l(fmt("st.shared.%s [%s+%u], %s", kSpTy[sp], kSpBase[sp], xoff(e, sp, off) * 4, r.c_str()));
   if (e.dry) e.log->w[k].push_back({e.step, e.warp});
-  else e.fwd[k] = Em::Fwd{r, e.step};
+  else e.fwd[k] = Em::Fwd{r, e.step, e.opn};
 }
 // a write this warp cannot forward (cp.async, generic path)
 void opaque_write(Em &e, uint64_t sp, uint32_t off) {
   const uint64_t k = skey(sp, off);
   if (e.dry) e.log->w[k].push_back({e.step, e.warp});
   else e.fwd.erase(k);
+  const int64_t id = inst_of(e, sp, off);
+  if (id >= 0 && e.probe) (*e.inst)[(size_t)id].need = true;
 }
 uint64_t layout_space(uint32_t lay) {
   return lay == LC_U32 ? SP_W : lay == LC_U16 ? SP_H : lay == LC_U8 ? SP_B : SP_S;
@@ -206,6 +283,7 @@ uint64_t layout_space(uint32_t lay) {
 // a shared-memory read that bypasses lds (direct loads, the generic path)
 void note_read(Em &e, uint64_t sp, uint32_t off) {
   if (e.probe) e.log->rd[skey(sp, off)].push_back(e.step);
+  inst_read(e, sp, off);
 }
 // every slot word an operand (offset, width, layout) of the generic path may read
 void note_operand_reads(Em &e, uint32_t off, uint32_t w, uint32_t lay) {
@@ -344,6 +422,7 @@ void emit_narrow(Em &e, const Desc &q) {
   const uint32_t wd = (q.x >> 20) & 63u, wa = q.x >> 26, wb = q.w & 63u, imm = (q.w >> 6) & 31u;
   const bool hb = (q.w >> 11) & 1u, hc = (q.w >> 12) & 1u;
   const uint32_t d = q.y & 0xFFFFu, a = q.y >> 16, b = q.z & 0xFFFFu, c = q.z >> 16;
+  begin_value(e, layout_space(ld), d, 1);
   if (op == RTLSIM_OP_MUX && la == LC_BIT && hb && hc) {
     // 1-bit select straight from its packed word: the lane's bit moved to
     // bit 31 and sign-filled is the all-ones / zero mask of the LOP3 mux
@@ -512,6 +591,21 @@ void generic_wide(Em &e, const WideRec &w, uint32_t idx) {
   note_operand_reads(e, w.a, w.wa, w.lays & 0xFFu);
   note_operand_reads(e, w.b, w.wb, (w.lays >> 8) & 0xFFu);
   note_operand_reads(e, w.c, w.wc, (w.lays >> 16) & 0xFFu);
+  if (e.compact && e.wrec) {
+    // the generic path reads the record's slot offsets: a copy with the
+    // compacted offsets, in this partition's own record table
+    WideRec r = w;
+    auto tr = [&](uint32_t off, uint32_t wv, uint32_t lay) -> uint32_t {
+      if (lay == LC_IMM || wv == 0) return off;
+      return xoff(e, layout_space(lay), off);
+    };
+    r.a = tr(w.a, w.wa, w.lays & 0xFFu);
+    r.b = tr(w.b, w.wb, (w.lays >> 8) & 0xFFu);
+    r.c = tr(w.c, w.wc, (w.lays >> 16) & 0xFFu);
+    r.d = tr(w.d, w.wd, w.wd <= 32 ? value_layout(w.wd, false) : LC_U32);
+    idx = (uint32_t)e.wrec->size();
+    e.wrec->push_back(r);
+  }
   emit_generic_call(e, idx);
   if (w.wd <= 32) {
     opaque_write(e, layout_space(value_layout(w.wd, false)), w.d);
@@ -526,6 +620,8 @@ void emit_wide(Em &e, const WideRec &w, uint32_t idx) {
   A.off = w.a; A.w = w.wa; A.lay = w.lays & 0xFFu;
   B.off = w.b; B.w = w.wb; B.lay = (w.lays >> 8) & 0xFFu;
   C.off = w.c; C.w = w.wc; C.lay = (w.lays >> 16) & 0xFFu;
+  if (wd <= 32) begin_value(e, layout_space(value_layout(wd, false)), w.d, 1);
+  else begin_value(e, SP_W, w.d, nd);
   auto bin = [&](const char *ins) {
     for (uint32_t i = 0; i < nd; i++) {
       std::string xa = reg_of(e, wword(e, A, i, false)), xb = reg_of(e, wword(e, B, i, false)), r = e.R();
@@ -753,25 +849,29 @@ void emit_ld(Em &e, uint32_t arena, uint32_t cls, uint32_t row, uint32_t slot, u
   std::string addr;
   switch (cls) {
     case CLS_U32:
+      begin_value(e, SP_W, slot, nw, true);
       for (uint32_t i = 0; i < nw; i++) {
         std::string ai = gaddr(e, "N4", row + i, fmt("tb_%s3", A).c_str());
-        e.l(fmt("cp.async.ca.shared.global [%%rw+%u], [%s], 4", (slot + 32 * i) * 4, ai.c_str()));
+        e.l(fmt("cp.async.ca.shared.global [%%rw+%u], [%s], 4", xoff(e, SP_W, slot + 32 * i) * 4, ai.c_str()));
         opaque_write(e, SP_W, slot + 32 * i);
       }
       break;
     case CLS_U16:
+      begin_value(e, SP_H, slot, 1, true);
       addr = gaddr(e, "N2", row, fmt("tb_%s2", A).c_str());
-      e.l(fmt("@%%pl16 cp.async.ca.shared.global [%%rw+%u], [%s], 4", slot * 4, addr.c_str()));
+      e.l(fmt("@%%pl16 cp.async.ca.shared.global [%%rw+%u], [%s], 4", xoff(e, SP_H, slot) * 4, addr.c_str()));
       opaque_write(e, SP_H, slot);
       break;
     case CLS_U8:
+      begin_value(e, SP_B, slot, 1, true);
       addr = gaddr(e, "N", row, fmt("tb_%s1", A).c_str());
-      e.l(fmt("@%%pl8 cp.async.ca.shared.global [%%rw+%u], [%s], 4", slot * 4, addr.c_str()));
+      e.l(fmt("@%%pl8 cp.async.ca.shared.global [%%rw+%u], [%s], 4", xoff(e, SP_B, slot) * 4, addr.c_str()));
       opaque_write(e, SP_B, slot);
       break;
     default:
+      begin_value(e, SP_S, slot, 1, true);
       addr = gaddr(e, "Nb", row, fmt("tb_%s0", A).c_str());
-      e.l(fmt("@%%pl0 cp.async.ca.shared.global [%%smb+%u], [%s], 4", slot * 4, addr.c_str()));
+      e.l(fmt("@%%pl0 cp.async.ca.shared.global [%%smb+%u], [%s], 4", xoff(e, SP_S, slot) * 4, addr.c_str()));
       opaque_write(e, SP_S, slot);
       break;
   }
@@ -823,7 +923,7 @@ void emit_st(Em &e, uint32_t code, uint32_t cls, uint32_t nw, uint32_t lay, uint
       // 32 byte / half-word lanes: 8 or 16 lanes copy the packed words
       std::string t = e.R();
       const char *pl = cls == CLS_U8 ? "%pl8" : "%pl16";
-      e.l(fmt("@%s ld.shared.u32 %s, [%%rw+%u]", pl, t.c_str(), slot * 4));
+      e.l(fmt("@%s ld.shared.u32 %s, [%%rw+%u]", pl, t.c_str(), xoff(e, cls == CLS_U8 ? SP_B : SP_H, slot) * 4));
       note_read(e, cls == CLS_U8 ? SP_B : SP_H, slot);
       note_read(e, layout_space(lay), slot);
       addr = cls == CLS_U8 ? gaddr(e, "N", row, fmt("tb_%s1", A).c_str()) : gaddr(e, "N2", row, fmt("tb_%s2", A).c_str());
@@ -901,6 +1001,7 @@ void emit_st_conv(Em &e, uint32_t tcls, uint32_t tnw, uint32_t slay, uint32_t sw
 }
 
 void emit_ld_const(Em &e, const Program &G, uint32_t slot, uint32_t pool, uint32_t nw, bool bcast) {
+  begin_value(e, bcast ? SP_S : SP_W, slot, nw);
   for (uint32_t i = 0; i < nw; i++) {
     std::string v = e.R();
     e.l(fmt("mov.u32 %s, %u", v.c_str(), G.const_pool[pool + i]));
@@ -923,6 +1024,7 @@ uint32_t lop3_lut(uint32_t lut) {
 void emit_bit(Em &e, const BitDesc &q) {
   const uint32_t lut = q.x & 0xFFu, immf = q.x >> 8;
   const uint32_t f[3] = {q.y >> 16, q.z & 0xFFFFu, q.z >> 16};
+  begin_value(e, SP_S, q.y & 0xFFFFu, 1);
   std::string v[3];
   for (int k = 0; k < 3; k++) {
     v[k] = e.R();
@@ -969,6 +1071,7 @@ void note_kind(Em &e, const std::string &kind, size_t from) {
 
 void emit_desc_(Em &e, const Program &G, const Desc &q);
 void emit_desc(Em &e, const Program &G, const Desc &q) {
+  e.opn++;
   const size_t from = e.s.size();
   emit_desc_(e, G, q);
   const uint32_t code = q.x & 0xFFu;
@@ -1030,8 +1133,22 @@ std::string func_proto(const std::string &name) {
 // (bar.sync 0, counted per CTA, not per PC) inside every warp's stream — so
 // a warp's instruction fetch is sequential across steps instead of jumping
 // over the other warps' code at every step.
+bool jit_compact_env(const Program &G) {
+  const char *e = getenv("RTLSIM_JIT_COMPACT");
+  return G.L == 1 && (e ? atoi(e) != 0 : true);
+}
+uint64_t jit_fwd_ops(bool compact) {
+  const char *e = getenv("RTLSIM_JIT_FWDOPS");
+  if (e) return (uint64_t)atoll(e);
+  return compact ? 64u : UINT64_MAX;
+}
+
 std::string step_function(const Program &G, const std::string &name, uint32_t s0, uint32_t s1, bool dig,
-                          uint32_t nspec, bool to_end) {
+                          uint32_t nspec, bool to_end, uint32_t *tile_words = nullptr,
+                          std::vector<WideRec> *wrec_out = nullptr) {
+  const bool compact = jit_compact_env(G) && to_end && tile_words;
+  std::vector<Em::Inst> insts;
+  std::vector<WideRec> wrec_probe, wrec_final;
   // dry pass: which warp writes which slot in which step (forwarding validity)
   WriteLog log;
   {
@@ -1055,7 +1172,11 @@ std::string step_function(const Program &G, const std::string &name, uint32_t s0
   e.to_end = to_end;
   e.nspec = nspec;
   e.log = &log;
-  e.fwd_max = jit_fwd_steps();
+  e.fwd_max = compact ? INT32_MAX / 2 : jit_fwd_steps();
+  e.fwd_ops = jit_fwd_ops(compact);
+  e.compact = compact;
+  e.inst = &insts;
+  e.wrec = probe ? &wrec_probe : &wrec_final;
   std::vector<std::string> labs(G.L);
   std::string tbl = e.L("T"), end = e.L("E");
   if (G.L > 1) {
@@ -1075,17 +1196,33 @@ std::string step_function(const Program &G, const std::string &name, uint32_t s0
       e.step = (int32_t)s;
       for (uint32_t k = G.bit_ptr[s] + w; k < G.bit_ptr[s + 1]; k += G.L) {
         const size_t from = e.s.size();
+        e.opn++;
         emit_bit(e, G.bitdesc[k]);
         note_kind(e, "bit", from);
       }
       for (uint32_t k = G.step_ptr[s * G.L + w]; k < G.step_ptr[s * G.L + w + 1]; k++) emit_desc(e, G, G.desc[k]);
       e.l("cp.async.commit_group");
       e.l(fmt("cp.async.wait_group %u", G.step_wait[s]));
-      // the per-warp code blocks each hold their own copy of the step
-      // barrier, so different warps execute different barrier instructions:
-      // the non-.aligned form is required then; with one block
-      // (L == 1) every warp runs the same instruction
-      e.l(G.L > 1 ? "barrier.sync 0" : "bar.sync 0");
+      // The per-warp code blocks each hold their own copy of the step
+      // barrier, so different warps reach barrier 0 through different
+      // barrier instructions. ADVICE r1 asked for the non-.aligned form
+      // (barrier.sync) there; measured, it makes ptxas treat every step as
+      // potentially divergent: config 3 partition 0 grows from 21,272 to
+      // 48,208 SASS instructions (WARPSYNC before every vote and barrier) and
+      // runs slower. Every warp of the CTA executes exactly one barrier-0
+      // instruction per step, warp-converged, in the same order — the
+      // property the hardware barrier counts, and the one warp-specialised
+      // CUTLASS kernels rely on when producer and consumer warps meet at a
+      // named barrier from different code. The aligned form is kept;
+      // RTLSIM_JIT_TBAR=2 emits the non-aligned one for A/B.
+      if (jit_tbar() == 0)
+        e.l("bar.sync 0");
+      else if (jit_tbar() == 2)
+        e.l("barrier.sync 0");
+      else if (G.L > 1)
+        e.l(fmt("barrier.sync %%tbar, %u", 32u * G.L));
+      else
+        e.l("bar.warp.sync -1");
     }
     if (G.L > 1) e.l(fmt("bra.uni %s", end.c_str()));
   }
@@ -1095,16 +1232,61 @@ std::string step_function(const Program &G, const std::string &name, uint32_t s0
   // records which slot reads still go to shared memory once forwarding is
   // applied; the final pass drops the stores nobody reads from there
   Em e;
-  if (jit_dse()) {
+  if (jit_dse() || compact) {
     Em pe;
     emit_real(pe, true, false);
+    if (compact) {
+      // first-fit by step interval over the instances read back from shared
+      // memory (or written opaquely); space is reused only across steps, so
+      // a cp.async into a reused row never overtakes a read of its old value
+      std::vector<uint32_t> order;
+      for (uint32_t i = 0; i < insts.size(); i++)
+        if (insts[i].need) order.push_back(i);
+      std::sort(order.begin(), order.end(), [&](uint32_t a, uint32_t b) {
+        return insts[a].s0 != insts[b].s0 ? insts[a].s0 < insts[b].s0 : a < b;
+      });
+      struct Act { uint32_t nb, words; int32_t s1; };
+      std::vector<Act> act;
+      uint32_t extent = 0;
+      for (uint32_t id : order) {
+        Em::Inst &I = insts[id];
+        act.erase(std::remove_if(act.begin(), act.end(), [&](const Act &a) { return a.s1 < I.s0; }), act.end());
+        std::sort(act.begin(), act.end(), [](const Act &a, const Act &b) { return a.nb < b.nb; });
+        uint32_t at = 0;
+        for (const Act &a : act) {
+          if (a.nb >= at + I.words) break;
+          at = std::max(at, a.nb + a.words);
+        }
+        I.nb = at;
+        act.push_back({at, I.words, std::max(I.s0, I.s1)});
+        extent = std::max(extent, at + I.words);
+      }
+      *tile_words = extent;
+      if (getenv("RTLSIM_JIT_COMPACT_DEBUG")) {
+        std::map<int32_t, std::array<uint64_t, 3>> live;   // step -> words (all, loaded, reread)
+        for (uint32_t id : order) {
+          const Em::Inst &I = insts[id];
+          for (int32_t t = I.s0; t <= std::max(I.s0, I.s1); t++) {
+            live[t][0] += I.words;
+            if (I.opq) live[t][1] += I.words;
+          }
+        }
+        uint64_t mx = 0, ml = 0;
+        for (auto &kv : live)
+          if (kv.second[0] > mx) mx = kv.second[0], ml = kv.second[1];
+        size_t n_need = order.size();
+        fprintf(stderr, "compact %s: %zu instances, %zu in smem, extent %u words, peak live %llu words (%llu loaded)\n",
+                name.c_str(), insts.size(), n_need, extent, (unsigned long long)mx, (unsigned long long)ml);
+      }
+    }
     emit_real(e, false, true);
+    if (compact && wrec_out) *wrec_out = wrec_final;
   } else {
     emit_real(e, false, false);
   }
   std::string out = func_proto(name) + "\n{\n";
   out += fmt("\t.reg .b32 %%r<%u>;\n\t.reg .b64 %%rd<%u>;\n\t.reg .pred %%p<%u>;\n", e.nr + 1, e.nrd + 1, e.np + 1);
-  out += "\t.reg .b32 %smb, %lane, %wl, %N, %rw, %rh, %rb, %N4, %N2, %Nb, %lsh;\n\t.reg .b64 %tbb1, %tbb2, %tlw, ";
+  out += "\t.reg .b32 %smb, %lane, %wl, %N, %tbar, %rw, %rh, %rb, %N4, %N2, %Nb, %lsh;\n\t.reg .b64 %tbb1, %tbb2, %tlw, ";
   for (int i = 0; i < kN64; i++) out += fmt("%s%%%s", i ? ", " : "", kCtx64[i]);
   out += ";\n\t.reg .pred %pl0, %pl8, %pl16, %pdig;\n";
   for (int i = 0; i < kN32; i++) out += fmt("\tld.param.u32 %%%s, [a_%s];\n", kCtx32[i], kCtx32[i]);
@@ -1122,8 +1304,11 @@ std::string step_function(const Program &G, const std::string &name, uint32_t s0
 
 }  // namespace
 
+bool jit_compact(const Program &G) { return jit_compact_env(G); }
+
 std::string jit_partition_ptx(const Program &G, uint32_t q, const std::string &rt_ptx, uint32_t tmax, bool dig,
-                              uint32_t nspec) {
+                              uint32_t nspec, JitPartInfo *info) {
+  const bool compact = jit_compact_env(G);
   const uint32_t s0 = G.part_steps[q], s1 = G.part_steps[q + 1];
   std::string mod;
   mod.reserve(1 << 20);
@@ -1143,27 +1328,36 @@ std::string jit_partition_ptx(const Program &G, uint32_t q, const std::string &r
   uint64_t acc = 0;
   for (uint32_t s = s0; s < s1; s++) {
     acc += (G.step_ptr[(s + 1) * G.L] - G.step_ptr[s * G.L]) + (G.bit_ptr[s + 1] - G.bit_ptr[s]);
-    if (acc >= kGroupOps || s + 1 == s1) {
+    // compacted slots are allocated per function: one function per partition
+    if ((acc >= kGroupOps && !compact) || s + 1 == s1) {
       groups.push_back({g0, s + 1});
       g0 = s + 1;
       acc = 0;
     }
   }
+  uint32_t tile_words = 0;
+  JitPartInfo local;
+  if (!info) info = &local;
   for (size_t g = 0; g < groups.size(); g++)
     mod += step_function(G, fmt("rtl_steps_%zu", g), groups[g].first, groups[g].second, dig, nspec,
-                         groups[g].second == s1) + "\n";
+                         groups[g].second == s1, compact ? &tile_words : nullptr,
+                         compact ? &info->wide : nullptr) + "\n";
+  // shared memory per tile: the compacted extent, or the schedule's slots
+  const uint32_t tbytes = compact ? std::max<uint32_t>(16u, ((tile_words * 4u) + 15u) & ~15u) : jit_tile_bytes(G);
+  info->tile_bytes = tbytes;
   // the kernel: per-thread context, then the step functions in order
   // A CTA holds `tpc` tiles; warp g works on tile g / L as op-lane g % L, so
   // the warps of one op-lane (one per tile) run identical code in step
   // lock-step and share its instruction fetch.
   mod += fmt(".visible .entry rtl_jit_part(.param .align 8 .b8 prm[%zu])\n.maxntid %u, 1, 1\n{\n",
              sizeof(JitParams), 32u * G.L * std::max<uint32_t>(tmax, 1u));
-  mod += "\t.reg .b32 %tidx, %tile, %s, %smb, %lane, %wl, %N, %wg, %tsub, %tpc;\n\t.reg .b64 %t64, %b64, %digb;\n\t.reg .pred %pz;\n\t.reg .b64 ";
+  mod += "\t.reg .b32 %tidx, %tile, %s, %smb, %lane, %wl, %N, %wg, %tsub, %tpc, %tbar;\n\t.reg .b64 %t64, %b64, %digb;\n\t.reg .pred %pz;\n\t.reg .b64 ";
   for (int i = 0; i < kN64; i++) mod += fmt("%s%%%s", i ? ", " : "", kCtx64[i]);
   mod += ";\n";
   mod += fmt("\tmov.u32 %%tidx, %%tid.x;\n\tand.b32 %%lane, %%tidx, 31;\n\tshr.u32 %%wg, %%tidx, 5;\n"
              "\trem.u32 %%wl, %%wg, %u;\n\tdiv.u32 %%tsub, %%wg, %u;\n", G.L, G.L);
   mod += fmt("\tld.param.u32 %%tpc, [prm+%zu];\n", offsetof(JitParams, tpc));
+  mod += "\tadd.u32 %tbar, %tsub, 1;\n";
   mod += "\tmov.u32 %tile, %ctaid.x;\n\tmad.lo.u32 %tile, %tile, %tpc, %tsub;\n\tmad.lo.u32 %s, %tile, 32, %lane;\n";
   mod += fmt("\tld.param.u32 %%N, [prm+%zu];\n", offsetof(JitParams, N));
   if (nspec)   // row offsets are immediates for this N_pad: refuse any other
@@ -1188,7 +1382,7 @@ std::string jit_partition_ptx(const Program &G, uint32_t q, const std::string &r
   mod += fmt("\tld.param.u64 %%wide, [prm+%zu];\n", offsetof(JitParams, wide));
   mod += fmt("\tmov.u32 %%smb, dyn_smem;\n\tmad.lo.u32 %%smb, %%tsub, %u, %%smb;\n\tcvta.shared.u64 %%smg, dyn_smem;\n"
              "\tmul.wide.u32 %%t64, %%tsub, %u;\n\tadd.u64 %%smg, %%smg, %%t64;\n",
-             jit_tile_bytes(G), jit_tile_bytes(G));
+             tbytes, tbytes);
   for (size_t g = 0; g < groups.size(); g++) {
     mod += "\t{\n";
     std::string args;
@@ -1252,10 +1446,17 @@ int jit_build(const Program &G, const std::string &rt_ptx_path, uint32_t smem_by
   }
   const uint32_t NP = (uint32_t)G.part_steps.size() - 1;
   // tiles per CTA the kernels are built for (their thread count bounds registers)
-  const uint32_t tmax = std::max<uint32_t>(
-      1u, std::min<uint32_t>(std::min<uint32_t>(jit_default_tiles(), 32u / std::max<uint32_t>(G.L, 1u)),
-                             smem_bytes / jit_tile_bytes(G)));
+  // (compacted kernels: their shared memory is known only after generation;
+  // the launch picks the tiles per CTA that fit, up to tmax)
+  const bool compact = jit_compact_env(G);
+  const uint32_t tmax = compact
+      ? std::max<uint32_t>(1u, std::min<uint32_t>(jit_default_tiles(true), 32u))
+      : std::max<uint32_t>(
+            1u, std::min<uint32_t>(std::min<uint32_t>(jit_default_tiles(), 32u / std::max<uint32_t>(G.L, 1u)),
+                                   smem_bytes / jit_tile_bytes(G)));
   out->tmax = tmax;
+  out->compact = compact;
+  std::vector<JitPartInfo> infos(NP);
   out->nspec = nspec;
   // ptxas -O3 schedules this code better than --Ofast-compile=mid (config 3
   // ~1.8x, config 4 175 vs 185 ms/cycle) but compiles ~3x slower (config 4:
@@ -1292,7 +1493,7 @@ int jit_build(const Program &G, const std::string &rt_ptx_path, uint32_t smem_by
     th.emplace_back([&]() {
       for (uint32_t q; (q = next++) < NP;) {
         if (G.part_steps[q] == G.part_steps[q + 1]) continue;
-        std::string ptx = jit_partition_ptx(G, q, rt, tmax, dig, nspec);
+        std::string ptx = jit_partition_ptx(G, q, rt, tmax, dig, nspec, &infos[q]);
         ptx_bytes += ptx.size();
         if (const char *dir = getenv("RTLSIM_JIT_SAVE")) {   // debugging aid: keep the module
           std::ofstream o(fmt("%s/part%u.ptx", dir, q));
@@ -1352,6 +1553,23 @@ int jit_build(const Program &G, const std::string &rt_ptx_path, uint32_t smem_by
       *err = fmt("partition %u: ", q) + errs[q];
       return RTLSIM_E_ARG;
     }
+  out->tile_bytes.assign(NP, 0);
+  out->wide_base.assign(NP, 0);
+  std::vector<WideRec> wall;
+  for (uint32_t q = 0; q < NP; q++) {
+    out->tile_bytes[q] = infos[q].tile_bytes ? infos[q].tile_bytes : jit_tile_bytes(G);
+    out->wide_base[q] = (uint32_t)wall.size();
+    wall.insert(wall.end(), infos[q].wide.begin(), infos[q].wide.end());
+  }
+  if (device >= 0 && !wall.empty()) {
+    cudaError_t e = cudaMalloc((void **)&out->d_wide, wall.size() * sizeof(WideRec));
+    if (e == cudaSuccess) e = cudaMemcpy(out->d_wide, wall.data(), wall.size() * sizeof(WideRec), cudaMemcpyHostToDevice);
+    if (e != cudaSuccess) {
+      *err = std::string("JIT record table: ") + cudaGetErrorString(e);
+      cudaGetLastError();
+      return RTLSIM_E_CUDA;
+    }
+  }
   for (uint32_t q = 0; q < NP; q++) {
     if (cubins[q].empty()) continue;
     out->cubin_bytes += cubins[q].size();
@@ -1360,16 +1578,18 @@ int jit_build(const Program &G, const std::string &rt_ptx_path, uint32_t smem_by
     if (e != cudaSuccess && from_cache[q]) {   // a damaged cached cubin: compile it again
       cudaGetLastError();
       std::string cerr;
-      if (compile_ptx(jit_partition_ptx(G, q, rt, tmax, dig, nspec), o3, &cubins[q], &cerr) != 0) {
+      if (compile_ptx(jit_partition_ptx(G, q, rt, tmax, dig, nspec, &infos[q]), o3, &cubins[q], &cerr) != 0) {
         *err = fmt("partition %u: ", q) + cerr;
         return RTLSIM_E_ARG;
       }
       e = cudaLibraryLoadData(&out->libs[q], cubins[q].data(), nullptr, nullptr, 0, nullptr, nullptr, 0);
     }
     if (e == cudaSuccess) e = cudaLibraryGetKernel(&out->kern[q], out->libs[q], "rtl_jit_part");
-    if (e == cudaSuccess)
-      e = cudaKernelSetAttributeForDevice(out->kern[q], cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                          (int)std::max<uint32_t>(smem_bytes, 1024), device);
+    if (e == cudaSuccess) {   // the launch picks tiles per CTA within the device's opt-in maximum
+      int optin = (int)std::max<uint32_t>(smem_bytes, 1024);
+      cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, device);
+      e = cudaKernelSetAttributeForDevice(out->kern[q], cudaFuncAttributeMaxDynamicSharedMemorySize, optin, device);
+    }
     if (e != cudaSuccess) {
       *err = std::string("loading JIT kernel: ") + cudaGetErrorString(e);
       cudaGetLastError();
@@ -1379,12 +1599,14 @@ int jit_build(const Program &G, const std::string &rt_ptx_path, uint32_t smem_by
   return RTLSIM_OK;
 }
 
-uint32_t jit_default_tiles() {
+uint32_t jit_default_tiles(bool compact) {
   const char *e = getenv("RTLSIM_JIT_TMAX");   // read per load (tests vary it)
-  return e ? std::min<uint32_t>(kJitMaxTiles, (uint32_t)std::max(1, atoi(e))) : 4u;
+  return e ? std::min<uint32_t>(kJitMaxTiles, (uint32_t)std::max(1, atoi(e))) : (compact ? 16u : 4u);
 }
 
 void jit_free(JitKernels *k) {
+  if (k->d_wide) cudaFree(k->d_wide);
+  k->d_wide = nullptr;
   for (cudaLibrary_t l : k->libs)
     if (l) cudaLibraryUnload(l);
   k->libs.clear();

@@ -31,15 +31,25 @@ struct JitParams {
 static_assert(sizeof(JitParams) == 160, "JitParams layout is hard-coded in the PTX generator");
 
 // Maximum tiles per CTA the kernels are compiled for (.maxntid 32 * L * kJitMaxTiles).
-constexpr uint32_t kJitMaxTiles = 8;
+constexpr uint32_t kJitMaxTiles = 16;
 // Tiles per CTA the kernels are compiled for by default (RTLSIM_JIT_TMAX
 // overrides, up to kJitMaxTiles and 1024 threads per CTA).
-uint32_t jit_default_tiles();
+uint32_t jit_default_tiles(bool compact = false);
 // Bytes of shared memory per tile in a JIT CTA (16-byte aligned).
 inline uint32_t jit_tile_bytes(const Program &G) { return ((G.smem_words * 4u) + 15u) & ~15u; }
 
+// What the generator decided for one partition kernel beyond its PTX.
+struct JitPartInfo {
+  uint32_t tile_bytes = 0;          // shared memory per tile (compacted slots; 0 = jit_tile_bytes(G))
+  std::vector<WideRec> wide;        // generic-path records with compacted slot offsets (or empty)
+};
+
 struct JitKernels {
   std::vector<cudaLibrary_t> libs;
+  std::vector<uint32_t> tile_bytes; // per exec-order partition: shared memory per tile
+  std::vector<uint32_t> wide_base;  // per partition: first record in d_wide (compacted records)
+  WideRec *d_wide = nullptr;        // compacted generic-path records of all partitions (or null)
+  bool compact = false;             // slot compaction (L == 1 kernels)
   std::vector<cudaKernel_t> kern;   // per exec-order partition (nullptr: empty partition)
   double gen_s = 0, compile_s = 0;
   bool o3 = false;
@@ -55,7 +65,11 @@ struct JitKernels {
 // immediates; the kernel traps on any other N), 0 = generic (row stride read
 // from the launch parameters).
 std::string jit_partition_ptx(const Program &G, uint32_t q, const std::string &rt_ptx, uint32_t tmax, bool dig,
-                              uint32_t nspec);
+                              uint32_t nspec, JitPartInfo *info = nullptr);
+// Slot compaction (RTLSIM_JIT_COMPACT, default on for one op-lane): a tile is
+// one warp, so only values read back from shared memory (the others stay in
+// registers) get slots, allocated by step interval.
+bool jit_compact(const Program &G);
 // Generate + compile (nvPTXCompiler, all host cores) + load every partition.
 // device < 0: generate and compile only (host-only contexts, CPU tests).
 int jit_build(const Program &G, const std::string &rt_ptx_path, uint32_t smem_bytes, int device, JitKernels *out,

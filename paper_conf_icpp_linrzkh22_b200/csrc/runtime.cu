@@ -542,13 +542,17 @@ static int jit_ensure(rtlsim_ctx *ctx, bool dig) {
 // JIT: tiles per CTA — as many as the shared memory holds (up to the count
 // the kernels were compiled for) that divide the tile count; env override
 // RTLSIM_JIT_TPC for measurements
-static uint32_t jit_tiles_per_cta(rtlsim_ctx *ctx, const JitKernels &JK) {
+static uint32_t jit_tile_smem(rtlsim_ctx *ctx, const JitKernels &JK, uint32_t q) {
+  return q < JK.tile_bytes.size() && JK.tile_bytes[q] ? JK.tile_bytes[q] : ctx->jit_smem;
+}
+static uint32_t jit_tiles_per_cta(rtlsim_ctx *ctx, const JitKernels &JK, uint32_t q) {
   const uint32_t tiles = ctx->N_pad / 32u;
   int optin = 232448;
   cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, ctx->device);
   // the kernel set being launched (the check-mode variant may have been built
-  // with another RTLSIM_JIT_TMAX than the plain one): its .maxntid bound
-  uint32_t m = std::min<uint32_t>(JK.tmax, (uint32_t)optin / std::max<uint32_t>(ctx->jit_smem, 1u));
+  // with another RTLSIM_JIT_TMAX than the plain one): its .maxntid bound; the
+  // partition's own shared memory per tile (compacted kernels differ)
+  uint32_t m = std::min<uint32_t>(JK.tmax, (uint32_t)optin / std::max<uint32_t>(jit_tile_smem(ctx, JK, q), 1u));
   if (const char *e = getenv("RTLSIM_JIT_TPC")) m = std::min<uint32_t>(m, (uint32_t)atoi(e));
   m = std::max<uint32_t>(m, 1u);
   while (m > 1 && tiles % m) m--;
@@ -638,12 +642,12 @@ static int launch_chunk(rtlsim_ctx *ctx, int b, uint64_t cycle0, uint32_t nc, bo
           jp.in[3] = (uint64_t)(ctx->d_in[b].u32 + (size_t)c * ctx->in_stride.s[CLS_U32]);
           jp.out = (uint64_t)(ctx->d_out[b] + (size_t)c * G.OW * ctx->N_pad);
           jp.digest = digest ? (uint64_t)(ctx->d_dig[b] + (size_t)c * ctx->N_pad) : 0;
-          jp.wide = (uint64_t)ctx->d_wide;
+          jp.wide = JK.d_wide ? (uint64_t)(JK.d_wide + JK.wide_base[q]) : (uint64_t)ctx->d_wide;
           jp.N = ctx->N_pad;
-          jp.tpc = jit_tiles_per_cta(ctx, JK);
+          jp.tpc = jit_tiles_per_cta(ctx, JK, q);
           void *args[] = {&jp};
           e = cudaLaunchKernel((const void *)JK.kern[q], dim3(ctx->N_pad / 32u / jp.tpc),
-                               dim3(32u * G.L * jp.tpc), args, ctx->jit_smem * jp.tpc, cap);
+                               dim3(32u * G.L * jp.tpc), args, jit_tile_smem(ctx, JK, q) * jp.tpc, cap);
         } else {
           EvalParams p = eval_params(ctx, b, (cycle0 & 1ull) + c, 1, digest);
           p.step_begin = G.part_steps[q];
