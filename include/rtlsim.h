@@ -68,7 +68,9 @@ enum rtlsim_opcode {
   RTLSIM_OP_MUX = 25,   /* a = select (any width, != 0), b = then, c = else  */
   RTLSIM_OP_CONCAT = 26,/* {a, b}: (a << wb) | b                             */
   RTLSIM_OP_SLICE = 27, /* a[imm + wd - 1 : imm]; imm + wd <= wa             */
-  RTLSIM_OP_REDAND = 28, RTLSIM_OP_REDOR = 29, RTLSIM_OP_REDXOR = 30
+  RTLSIM_OP_REDAND = 28, RTLSIM_OP_REDOR = 29, RTLSIM_OP_REDXOR = 30,
+  RTLSIM_OP_MEMRD = 31  /* ARRSEL read: dst := MEM[imm][V[a]], 0 when V[a] >=
+                           depth; wd = the memory's width (reading 12) */
 };
 #define RTLSIM_NONE 0xFFFFFFFFu
 #define RTLSIM_MAX_WIDTH 1024
@@ -100,6 +102,25 @@ typedef struct {
   uint32_t n_outputs;
   const uint32_t *output_sig;  /* [n_outputs] any signals: output word order  */
   uint32_t n_partitions;       /* ops[i].part < n_partitions; partition DAG acyclic */
+  /* Memories (§3.1.1, Fig 5: ARRSEL, an array variable indexed at
+   * run time, v1[v2[2]]; reading 12). All zero / NULL: none.
+   * Memory m: mem_depth[m] entries of mem_width[m] bits, initial contents
+   * mem_init (every memory's entries in order, ceil(w/32) words each; NULL =
+   * all zero), the same for every stimulus. Reads: RTLSIM_OP_MEMRD ops (the
+   * memory as it was at the start of the cycle). Write port p =
+   * mem_wport[4p..4p+3] = {memory, address signal, data signal, enable
+   * signal}: at the clock edge, with every register, if V[en] != 0 and
+   * V[addr] < depth, entry V[addr] := V[data] zero-extended / truncated to the
+   * memory width; ports apply in index order (a later port wins). Memory
+   * state is per stimulus, laid out [entry word][N] in HBM. Supported with
+   * RTLSIM_F_JIT (other backends: E_UNSUPPORTED); read and write addresses
+   * at most 32 bits wide. */
+  uint32_t n_mems;
+  const uint16_t *mem_width;   /* [n_mems] 1..1024                             */
+  const uint32_t *mem_depth;   /* [n_mems] >= 1                                */
+  const uint32_t *mem_init;    /* [sum depth * ceil(w/32)] or NULL             */
+  uint32_t n_wports;
+  const uint32_t *mem_wport;   /* [n_wports * 4]                               */
 } rtlsim_ir;
 
 /* Option flags */
@@ -175,6 +196,14 @@ typedef struct {
                                 exceed the smem budget (options.smem_limit) */
   uint64_t n_live_ops;       /* ops evaluated per cycle (n_ops minus dead logic) */
   uint64_t live_word_ops;    /* word_ops of the live ops                       */
+  uint64_t jit_sass_instructions; /* RTLSIM_F_JIT: SASS instructions of all partition
+                                kernels; straight-line code, so each is issued by
+                                one warp per 32-stimulus tile per cycle:
+                                / n_live_ops = warp-instructions per live op */
+  uint32_t jit_tiles_per_cta;  /* RTLSIM_F_JIT: tiles per CTA of the largest launch
+                                (warps of one op-lane that share each fetched
+                                instruction)                                  */
+  uint32_t pad0;
 } rtlsim_stats_t;
 
 typedef struct rtlsim_ctx rtlsim_ctx;
@@ -238,6 +267,10 @@ int rtlsim_reset(rtlsim_ctx *ctx);
  * gathers coverage; all_gather + OR, NCCL has no OR reduction). Errors:
  * E_STATE without the flag or before bind. */
 int rtlsim_coverage(rtlsim_ctx *ctx, uint32_t *bitmap, int clear);
+/* Memory contents mems[N][MW] (host; MW = sum over memories of depth x
+ * ceil(width/32) words, memories and entries in IR order) after the last
+ * simulated cycle. E_STATE before bind. */
+int rtlsim_get_mems(rtlsim_ctx *ctx, uint32_t *mems);
 /* Per-stimulus digest of the current register state, digest[s] (host, N
  * words) = XOR_k mix(((k + 1 + 2^31) << 32) | R[s][k]) — the register half of
  * the per-cycle DIGEST, so N x 8 bytes identify every final

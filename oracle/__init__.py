@@ -60,6 +60,13 @@ def lib():
         for f in ("oracle_iw", "oracle_ow", "oracle_rw"):
             getattr(L, f).restype = u32
             getattr(L, f).argtypes = [P]
+        L.oracle_design_set_mems.restype = ctypes.c_int
+        L.oracle_design_set_mems.argtypes = [P, u32, P, P, P, u32, P, ctypes.c_char_p, ctypes.c_int]
+        L.oracle_mw.restype = u64
+        L.oracle_mw.argtypes = [P]
+        L.oracle_simulate_mem.restype = ctypes.c_int
+        L.oracle_simulate_mem.argtypes = [P, u64, u64, P, P, P, P, P, P, ctypes.c_int, ctypes.c_char_p,
+                                          ctypes.c_int]
         _lib = L
     return _lib
 
@@ -86,14 +93,22 @@ class Design:
             raise ValueError("oracle rejected IR: " + err.value.decode())
         self.h = h
         self.IW, self.OW, self.RW = L.oracle_iw(h), L.oracle_ow(h), L.oracle_rw(h)
+        if getattr(ir, "n_mems", 0) or getattr(ir, "mem_wport", np.zeros((0, 4))).size:
+            self._keep += [ir.mem_width, ir.mem_depth, ir.mem_init, ir.mem_wport]
+            rc = L.oracle_design_set_mems(h, ir.n_mems, _p(ir.mem_width), _p(ir.mem_depth), _p(ir.mem_init),
+                                          int(ir.mem_wport.shape[0]), _p(ir.mem_wport), err, 256)
+            if rc:
+                raise ValueError("oracle rejected memories: " + err.value.decode())
+        self.MW = int(L.oracle_mw(h))
 
     def __del__(self):
         if getattr(self, "h", None):
             lib().oracle_design_free(self.h)
             self.h = None
 
-    def simulate(self, stim, regs_in=None, out=True, regs=True, digest=False, threads=1):
-        """stim [N][T][IW] u32 -> dict(out [N][T][OW], regs [N][RW], digest [N][T])."""
+    def simulate(self, stim, regs_in=None, out=True, regs=True, digest=False, threads=1, mems=False):
+        """stim [N][T][IW] u32 -> dict(out [N][T][OW], regs [N][RW], digest [N][T],
+        mems [N][MW] final memory words when mems=True)."""
         stim = np.ascontiguousarray(stim, dtype=np.uint32)
         N, T = int(stim.shape[0]), int(stim.shape[1])
         assert stim.shape[2] == self.IW, (stim.shape, self.IW)
@@ -101,12 +116,13 @@ class Design:
         r = np.zeros((N, self.RW), np.uint32) if regs else None
         dg = np.zeros((N, T), np.uint64) if digest else None
         rin = None if regs_in is None else np.ascontiguousarray(regs_in, dtype=np.uint32)
+        m = np.zeros((N, self.MW), np.uint32) if mems and self.MW else None
         err = ctypes.create_string_buffer(256)
-        rc = lib().oracle_simulate(self.h, N, T, _p(stim), _p(rin), _p(o), _p(r), _p(dg),
-                                   int(threads), err, 256)
+        rc = lib().oracle_simulate_mem(self.h, N, T, _p(stim), _p(rin), _p(o), _p(r), _p(dg), _p(m),
+                                       int(threads), err, 256)
         if rc:
             raise RuntimeError(err.value.decode())
-        return {"out": o, "regs": r, "digest": dg}
+        return {"out": o, "regs": r, "digest": dg, "mems": m}
 
 
 def simulate(ir, stim, **kw):

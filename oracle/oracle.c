@@ -40,6 +40,12 @@ struct oracle_design {
   uint64_t *off; /* word offset of each signal in a value vector */
   uint64_t total_words;
   uint32_t iw, ow, rw;
+  /* memories (oracle_design_set_mems) */
+  uint32_t n_mems, n_wports;
+  uint16_t *mem_width;
+  uint32_t *mem_depth, *mem_init, *wports;
+  uint64_t *mem_off; /* word offset of each memory in a memory vector */
+  uint64_t mw;       /* words of all memories */
 };
 
 static unsigned nw(unsigned bits) { return (bits + 31u) / 32u; }
@@ -307,7 +313,7 @@ static void seterr(char *err, int errlen, const char *msg, long v) {
 static int op_arity(unsigned opc) {
   switch (opc) {
     case ORC_COPY: case ORC_SEXT: case ORC_NOT: case ORC_NEG: case ORC_SLICE:
-    case ORC_REDAND: case ORC_REDOR: case ORC_REDXOR:
+    case ORC_REDAND: case ORC_REDOR: case ORC_REDXOR: case ORC_MEMRD:
       return 1;
     case ORC_MUX:
       return 3;
@@ -318,6 +324,7 @@ static int op_arity(unsigned opc) {
 
 void oracle_design_free(oracle_design *d) {
   if (!d) return;
+  free(d->mem_width); free(d->mem_depth); free(d->mem_init); free(d->wports); free(d->mem_off);
   free(d->width); free(d->kind); free(d->ops); free(d->reg_q); free(d->reg_d);
   free(d->reg_init); free(d->const_sig); free(d->const_words); free(d->input_sig);
   free(d->output_sig); free(d->off); free(d);
@@ -408,6 +415,57 @@ fail:
   return NULL;
 }
 
+int oracle_design_set_mems(oracle_design *d, uint32_t n_mems, const uint16_t *width, const uint32_t *depth,
+                           const uint32_t *init, uint32_t n_wports, const uint32_t *wports, char *err,
+                           int errlen) {
+  if (!d || (n_mems && (!width || !depth)) || (n_wports && !wports)) {
+    seterr(err, errlen, "bad memory arguments", 0);
+    return -1;
+  }
+  uint64_t mw = 0;
+  for (uint32_t m = 0; m < n_mems; m++) {
+    if (width[m] < 1 || width[m] > 1024 || depth[m] < 1) { seterr(err, errlen, "bad memory shape", m); return -1; }
+    mw += (uint64_t)depth[m] * nw(width[m]);
+  }
+  for (uint32_t p = 0; p < n_wports; p++) {
+    const uint32_t *w = wports + 4 * p;
+    if (w[0] >= n_mems || w[1] >= d->n_signals || w[2] >= d->n_signals || w[3] >= d->n_signals) {
+      seterr(err, errlen, "bad write port", p);
+      return -1;
+    }
+  }
+  for (uint32_t i = 0; i < d->n_ops; i++) {
+    const oracle_op *o = &d->ops[i];
+    if (o->opcode == ORC_MEMRD && (o->imm >= n_mems || d->width[o->dst] != width[o->imm])) {
+      seterr(err, errlen, "MEMRD: no such memory or width differs", i);
+      return -1;
+    }
+  }
+  free(d->mem_width); free(d->mem_depth); free(d->mem_init); free(d->wports); free(d->mem_off);
+  d->n_mems = n_mems;
+  d->n_wports = n_wports;
+  DUP(d->mem_width, width, n_mems, uint16_t);
+  DUP(d->mem_depth, depth, n_mems, uint32_t);
+  DUP(d->mem_init, init, mw, uint32_t);
+  if (!init) memset(d->mem_init, 0, sizeof(uint32_t) * (size_t)mw);
+  const size_t nwp = 4 * (size_t)n_wports;
+  DUP(d->wports, wports, nwp, uint32_t);
+  d->mem_off = (uint64_t *)malloc(sizeof(uint64_t) * ((size_t)n_mems + 1));
+  uint64_t pos = 0;
+  for (uint32_t m = 0; m < n_mems; m++) {
+    d->mem_off[m] = pos;
+    pos += (uint64_t)depth[m] * nw(width[m]);
+  }
+  d->mem_off[n_mems] = pos;
+  d->mw = mw;
+  return 0;
+}
+
+uint64_t oracle_mw(const oracle_design *d) { return d->mw; }
+
+/* value of a (width wa) as an index: UINT32_MAX when it does not fit 32 bits */
+static uint32_t as_index(const uint32_t *a, unsigned wa) { return shamt(a, wa); }
+
 uint32_t oracle_iw(const oracle_design *d) { return d->iw; }
 uint32_t oracle_ow(const oracle_design *d) { return d->ow; }
 uint32_t oracle_rw(const oracle_design *d) { return d->rw; }
@@ -418,6 +476,7 @@ typedef struct {
   const uint32_t *stim, *regs_in;
   uint32_t *out, *regs_out;
   uint64_t *digest;
+  uint32_t *mem_out;
   int rc;
 } job_t;
 
@@ -428,10 +487,12 @@ static void *run_block(void *arg) {
   uint32_t *V = (uint32_t *)calloc(d->total_words + 1, sizeof(uint32_t));
   uint32_t *R = (uint32_t *)calloc(d->rw + 1, sizeof(uint32_t));
   uint32_t *Rn = (uint32_t *)calloc(d->rw + 1, sizeof(uint32_t));
+  uint32_t *M = (uint32_t *)calloc(d->mw + 1, sizeof(uint32_t));
   j->rc = 0;
   for (uint64_t s = j->s0; s < j->s1; s++) {
-    /* R := reg_init, or the caller's per-stimulus state */
+    /* R := reg_init, or the caller's per-stimulus state; M := memory init */
     memcpy(R, j->regs_in ? j->regs_in + s * d->rw : d->reg_init, sizeof(uint32_t) * d->rw);
+    if (d->mw) memcpy(M, d->mem_init, sizeof(uint32_t) * d->mw);
     for (uint64_t c = 0; c < j->T; c++) {
       /* V[inputs] := stim[s][c] & mask(width) */
       const uint32_t *st = j->stim + (s * j->T + c) * d->iw;
@@ -468,6 +529,15 @@ static void *run_block(void *arg) {
         uint32_t wa = d->width[o->a];
         uint32_t wb = ar >= 2 ? d->width[o->b] : 0;
         uint32_t wc = ar >= 3 ? d->width[o->c] : 0;
+        if (o->opcode == ORC_MEMRD) {
+          /* ARRSEL read: entry V[a] of memory imm as it was at the start of
+           * the cycle; an index >= depth reads 0 (reading 12) */
+          if (o->imm >= d->n_mems) { j->rc = -1; goto done; }
+          const uint32_t m = o->imm, n = nw(d->mem_width[m]), idx = as_index(pa, wa);
+          for (unsigned t = 0; t < n; t++)
+            V[d->off[o->dst] + t] = idx < d->mem_depth[m] ? M[d->mem_off[m] + (uint64_t)idx * n + t] : 0u;
+          continue;
+        }
         if (oracle_eval_op(o->opcode, d->width[o->dst], o->imm, pa, wa, pb, wb, pc, wc,
                            V + d->off[o->dst]) != 0) {
           j->rc = -1;
@@ -499,18 +569,38 @@ static void *run_block(void *arg) {
         }
       }
       if (j->digest) j->digest[s * j->T + c] = dig;
+      /* memory write ports at the clock edge, in port order (a later port
+       * wins); their signals are the pre-edge values of this cycle */
+      for (uint32_t p = 0; p < d->n_wports; p++) {
+        const uint32_t *w = d->wports + 4 * p;
+        const uint32_t m = w[0], n = nw(d->mem_width[m]);
+        big_t en, data;
+        ext(&en, V + d->off[w[3]], d->width[w[3]], d->width[w[3]], 0);
+        if (is_zero(&en, nw(d->width[w[3]]))) continue;
+        const uint32_t idx = as_index(V + d->off[w[1]], d->width[w[1]]);
+        if (idx >= d->mem_depth[m]) continue;
+        ext(&data, V + d->off[w[2]], d->width[w[2]], d->mem_width[m], 0);
+        for (unsigned t = 0; t < n; t++) M[d->mem_off[m] + (uint64_t)idx * n + t] = data.w[t];
+      }
       memcpy(R, Rn, sizeof(uint32_t) * d->rw);
     }
     if (j->regs_out) memcpy(j->regs_out + s * d->rw, R, sizeof(uint32_t) * d->rw);
+    if (j->mem_out && d->mw) memcpy(j->mem_out + s * d->mw, M, sizeof(uint32_t) * d->mw);
   }
 done:
-  free(V); free(R); free(Rn);
+  free(V); free(R); free(Rn); free(M);
   return NULL;
 }
 
 int oracle_simulate(const oracle_design *d, uint64_t N, uint64_t T, const uint32_t *stim,
                     const uint32_t *regs_in, uint32_t *out, uint32_t *regs_out,
                     uint64_t *digest, int n_threads, char *err, int errlen) {
+  return oracle_simulate_mem(d, N, T, stim, regs_in, out, regs_out, digest, NULL, n_threads, err, errlen);
+}
+
+int oracle_simulate_mem(const oracle_design *d, uint64_t N, uint64_t T, const uint32_t *stim,
+                        const uint32_t *regs_in, uint32_t *out, uint32_t *regs_out, uint64_t *digest,
+                        uint32_t *mem_out, int n_threads, char *err, int errlen) {
   if (!d || (N && T && d->iw && !stim)) { seterr(err, errlen, "bad arguments", 0); return -1; }
   if (n_threads < 1) n_threads = 1;
   if ((uint64_t)n_threads > N) n_threads = N ? (int)N : 1;
@@ -519,7 +609,7 @@ int oracle_simulate(const oracle_design *d, uint64_t N, uint64_t T, const uint32
   for (int t = 0; t < n_threads; t++) {
     job_t *j = &jobs[t];
     j->d = d; j->T = T; j->stim = stim; j->regs_in = regs_in;
-    j->out = out; j->regs_out = regs_out; j->digest = digest;
+    j->out = out; j->regs_out = regs_out; j->digest = digest; j->mem_out = mem_out;
     j->s0 = N * (uint64_t)t / (uint64_t)n_threads;
     j->s1 = N * (uint64_t)(t + 1) / (uint64_t)n_threads;
   }
@@ -532,7 +622,7 @@ int oracle_simulate(const oracle_design *d, uint64_t N, uint64_t T, const uint32
   }
   for (int t = 0; t < n_threads; t++)
     if (jobs[t].rc) rc = -1;
-  if (rc) seterr(err, errlen, "unsupported operation (MUL/DIV > 64 bits or bad SLICE)", 0);
+  if (rc) seterr(err, errlen, "unsupported operation (MUL/DIV > 64 bits, bad SLICE or MEMRD without memory)", 0);
   free(jobs); free(th);
   return rc;
 }

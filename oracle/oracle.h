@@ -46,7 +46,8 @@ enum {
   ORC_LTS = 18, ORC_LES = 19, ORC_GTS = 20, ORC_GES = 21,
   ORC_SHL = 22, ORC_SHRL = 23, ORC_SHRA = 24, ORC_MUX = 25, ORC_CONCAT = 26,
   ORC_SLICE = 27, ORC_REDAND = 28, ORC_REDOR = 29, ORC_REDXOR = 30,
-  ORC_N_OPCODES = 31
+  ORC_MEMRD = 31, /* dst := MEM[imm][V[a]] (0 when V[a] >= depth): ARRSEL read */
+  ORC_N_OPCODES = 32
 };
 enum { ORC_INPUT = 0, ORC_REG = 1, ORC_COMB = 2, ORC_CONST = 3 };
 
@@ -69,6 +70,28 @@ oracle_design *oracle_design_new(uint32_t n_signals, const uint16_t *width, cons
                                  uint32_t n_outputs, const uint32_t *output_sig,
                                  char *err, int errlen);
 void oracle_design_free(oracle_design *d);
+
+/* Memories (§3.1.1, Fig 5: ARRSEL — an array variable indexed by a
+ * run-time value, v1[v2[2]]; reading 12). Memory m has depth[m]
+ * entries of width[m] bits (ceil(width/32) words each), initial contents
+ * init[] (all memories, entry-major, the same for every stimulus). Reads are
+ * the ORC_MEMRD op (combinational, see oracle_eval_op's caller). Write port
+ * p = {mem, addr, data, en} (signals): at the clock edge, after outputs are
+ * sampled and register next-states computed from the pre-edge values, every
+ * port with V[en] != 0 and V[addr] < depth writes zext/trunc(V[data]) to
+ * entry V[addr]; ports apply in index order (a later port wins). Reads in a
+ * cycle see the memory as it was at the start of the cycle (non-blocking,
+ * like registers). Returns 0, or -1 with err on bad arguments. */
+int oracle_design_set_mems(oracle_design *d, uint32_t n_mems, const uint16_t *width, const uint32_t *depth,
+                           const uint32_t *init, uint32_t n_wports, const uint32_t *wports /* [n][4] */,
+                           char *err, int errlen);
+/* Words of all memories of one stimulus (sum depth * ceil(width/32)). */
+uint64_t oracle_mw(const oracle_design *d);
+/* Like oracle_simulate, plus the final memory contents mem_out [N][MW] (may
+ * be NULL). */
+int oracle_simulate_mem(const oracle_design *d, uint64_t N, uint64_t T, const uint32_t *stim,
+                        const uint32_t *regs_in, uint32_t *out, uint32_t *regs_out, uint64_t *digest,
+                        uint32_t *mem_out, int n_threads, char *err, int errlen);
 uint32_t oracle_iw(const oracle_design *d);
 uint32_t oracle_ow(const oracle_design *d);
 uint32_t oracle_rw(const oracle_design *d);

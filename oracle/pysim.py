@@ -37,7 +37,18 @@ def simulate(ir: I.IR, stim: np.ndarray, regs_in=None):
         k += n
     ops = [(I.OPNAMES[int(o["opcode"])], int(o["dst"]), int(o["a"]), int(o["b"]), int(o["c"]),
             int(o["imm"])) for o in ir.ops]
+    # memories (reading 12): entry lists, read by MEMRD, written at
+    # the clock edge by the ports in order
+    n_mems = getattr(ir, "n_mems", 0)
+    mem_init, k = [], 0
+    for m in range(n_mems):
+        wm, dm = int(ir.mem_width[m]), int(ir.mem_depth[m])
+        n = I.nwords(wm)
+        mem_init.append([_val(ir.mem_init[k + n * e:k + n * (e + 1)], wm) for e in range(dm)])
+        k += n * dm
+    mems_out = []
     for s in range(N):
+        M = [list(x) for x in mem_init]
         if regs_in is None:
             R = list(init)
         else:
@@ -56,6 +67,9 @@ def simulate(ir: I.IR, stim: np.ndarray, regs_in=None):
             for q, v in zip(ir.reg_q, R):
                 V[int(q)] = v
             for name, d, a, b, cc, imm in ops:
+                if name == "MEMRD":
+                    V[d] = M[imm][V[a]] if V[a] < len(M[imm]) else 0
+                    continue
                 V[d] = ops_ref.evaluate(
                     name, width[d], V[a], width[a],
                     V.get(b, 0) if b != I.NONE else 0, width[b] if b != I.NONE else 0,
@@ -65,8 +79,16 @@ def simulate(ir: I.IR, stim: np.ndarray, regs_in=None):
                 row += I.int_to_words(V[int(o)], width[o])
             outs[s, c] = row
             R = [V[int(d)] & ops_ref.mask(width[q]) for q, d in zip(ir.reg_q, ir.reg_d)]
+            for m, a, dd, en in (ir.mem_wport if n_mems else []):
+                m, a, dd, en = int(m), int(a), int(dd), int(en)
+                if V[en] != 0 and V[a] < len(M[m]):
+                    M[m][V[a]] = V[dd] & ops_ref.mask(int(ir.mem_width[m]))
+        mems_out.append([w for m in range(n_mems) for v in M[m]
+                         for w in I.int_to_words(v, int(ir.mem_width[m]))])
         row = []
         for q, v in zip(ir.reg_q, R):
             row += I.int_to_words(v, width[q])
         regs[s] = row
+    if n_mems:
+        return outs, regs, np.asarray(mems_out, np.uint32).reshape(N, -1)
     return outs, regs

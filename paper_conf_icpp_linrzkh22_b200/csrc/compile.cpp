@@ -43,6 +43,7 @@ static int arity(uint32_t opc) {
   switch (opc) {
     case RTLSIM_OP_COPY: case RTLSIM_OP_SEXT: case RTLSIM_OP_NOT: case RTLSIM_OP_NEG:
     case RTLSIM_OP_SLICE: case RTLSIM_OP_REDAND: case RTLSIM_OP_REDOR: case RTLSIM_OP_REDXOR:
+    case RTLSIM_OP_MEMRD:
       return 1;
     case RTLSIM_OP_MUX:
       return 3;
@@ -235,7 +236,12 @@ int compile_program(const rtlsim_ir *ir, uint32_t op_lanes, uint32_t smem_limit_
   for (uint32_t i = 0; i < G.n_ops; i++) {
     const rtlsim_op &o = G.ops[i];
     const std::string at = "op " + std::to_string(i) + ": ";
-    if (o.opcode > RTLSIM_OP_REDXOR) return fail(err, RTLSIM_E_IR, at + "bad opcode");
+    if (o.opcode > RTLSIM_OP_MEMRD) return fail(err, RTLSIM_E_IR, at + "bad opcode");
+    if (o.opcode == RTLSIM_OP_MEMRD) {
+      if (o.imm >= ir->n_mems || !ir->mem_width || ir->mem_width[o.imm] != G.width[o.dst] || o.a >= n)
+        return fail(err, RTLSIM_E_IR, at + "MEMRD: no such memory or width differs");
+      if (G.width[o.a] > 32) return fail(err, RTLSIM_E_UNSUPPORTED, at + "MEMRD address wider than 32 bits");
+    }
     if (o.dst >= n || G.kind[o.dst] != RTLSIM_COMB) return fail(err, RTLSIM_E_IR, at + "dst must be a COMB signal");
     if (def[o.dst] != -1) return fail(err, RTLSIM_E_IR, at + "multiple drivers");
     def[o.dst] = (int32_t)i;
@@ -253,6 +259,47 @@ int compile_program(const rtlsim_ir *ir, uint32_t op_lanes, uint32_t smem_limit_
   }
   for (uint32_t s = 0; s < n; s++)
     if (G.kind[s] == RTLSIM_COMB && def[s] < 0) return fail(err, RTLSIM_E_IR, "undriven COMB signal " + std::to_string(s));
+  // memories: arena rows [entry word][N] (u32), write-port signals stored to
+  // the port arena every cycle (applied after the cycle's partitions)
+  if (ir->n_mems && (!ir->mem_width || !ir->mem_depth)) return fail(err, RTLSIM_E_ARG, "NULL memory arrays");
+  if (ir->n_wports && !ir->mem_wport) return fail(err, RTLSIM_E_ARG, "NULL write ports");
+  for (uint32_t m = 0; m < ir->n_mems; m++) {
+    const uint32_t w = ir->mem_width[m], dpt = ir->mem_depth[m];
+    if (w < 1 || w > RTLSIM_MAX_WIDTH || dpt < 1) return fail(err, RTLSIM_E_IR, "memory " + std::to_string(m) + ": bad shape");
+    if ((uint64_t)G.MR + (uint64_t)dpt * nwords(w) >= (1ull << 31))
+      return fail(err, RTLSIM_E_UNSUPPORTED, "memories larger than 2^31 words per stimulus");
+    G.mem_width.push_back((uint16_t)w);
+    G.mem_depth.push_back(dpt);
+    G.mem_row0.push_back(G.MR);
+    G.MR += dpt * nwords(w);
+  }
+  G.mem_init.assign(G.MR, 0u);
+  if (ir->mem_init) std::copy(ir->mem_init, ir->mem_init + G.MR, G.mem_init.begin());
+  for (uint32_t m = 0; m < G.mem_width.size(); m++)   // canonical entries: bits >= width are zero
+    if (G.mem_width[m] & 31u)
+      for (uint32_t e = 0; e < G.mem_depth[m]; e++)
+        G.mem_init[G.mem_row0[m] + e * nwords(G.mem_width[m]) + nwords(G.mem_width[m]) - 1] &=
+            (1u << (G.mem_width[m] & 31u)) - 1u;
+  for (uint32_t p = 0; p < ir->n_wports; p++) {
+    const uint32_t *w = ir->mem_wport + 4 * p;
+    if (w[0] >= ir->n_mems || w[1] >= n || w[2] >= n || w[3] >= n)
+      return fail(err, RTLSIM_E_IR, "write port " + std::to_string(p) + ": bad memory or signal");
+    if (G.width[w[1]] > 32) return fail(err, RTLSIM_E_UNSUPPORTED, "write port address wider than 32 bits");
+    Program::WPort wp{};
+    wp.mem = w[0];
+    auto port_word = [&](uint32_t sig) {
+      G.port_sig.push_back(sig);
+      G.port_word.push_back(G.PW);
+      G.PW += nwords(G.width[sig]);
+      return G.port_word.back();
+    };
+    wp.addr_word = port_word(w[1]);
+    wp.data_word = port_word(w[2]);
+    wp.data_width = G.width[w[2]];
+    wp.en_word = port_word(w[3]);
+    wp.en_width = G.width[w[3]];
+    G.wports.push_back(wp);
+  }
 
   // ------------------------------------------------ topological op order --
   std::vector<uint32_t> topo;
@@ -294,6 +341,7 @@ int compile_program(const rtlsim_ir *ir, uint32_t op_lanes, uint32_t smem_limit_
     std::vector<char> need(n, 0);
     for (uint32_t r = 0; r < ir->n_regs; r++) need[G.reg_d[r]] = 1;
     for (uint32_t o = 0; o < ir->n_outputs; o++) need[G.output_sig[o]] = 1;
+    for (uint32_t s : G.port_sig) need[s] = 1;   // memory write ports observe their signals
     for (auto it = topo.rbegin(); it != topo.rend(); ++it) {
       const rtlsim_op &o = G.ops[*it];
       live[*it] = need[o.dst];
@@ -397,8 +445,9 @@ int compile_program(const rtlsim_ir *ir, uint32_t op_lanes, uint32_t smem_limit_
   // ----------------------------------------------- per-partition schedule --
   std::vector<std::vector<uint32_t>> part_ops(NP);
   for (uint32_t i : topo) part_ops[G.ops[i].part].push_back(i);
-  std::vector<std::vector<uint32_t>> reg_sinks(NP), out_sinks(NP);
+  std::vector<std::vector<uint32_t>> reg_sinks(NP), out_sinks(NP), port_sinks(NP);
   for (uint32_t r = 0; r < ir->n_regs; r++) reg_sinks[owner_of_sig(G.reg_d[r])].push_back(r);
+  for (uint32_t k = 0; k < G.port_sig.size(); k++) port_sinks[owner_of_sig(G.port_sig[k])].push_back(k);
   for (uint32_t o = 0; o < ir->n_outputs; o++) out_sinks[owner_of_sig(G.output_sig[o])].push_back(o);
   std::vector<uint32_t> out_word(ir->n_outputs);
   for (uint32_t o = 0, w = 0; o < ir->n_outputs; o++) {
@@ -417,6 +466,7 @@ int compile_program(const rtlsim_ir *ir, uint32_t op_lanes, uint32_t smem_limit_
     }
     for (uint32_t r = 0; r < ir->n_regs; r++) used[G.reg_d[r]] = 1;
     for (uint32_t o = 0; o < ir->n_outputs; o++) used[G.output_sig[o]] = 1;
+    for (uint32_t s : G.port_sig) used[s] = 1;
     for (uint32_t i : topo) {
       uint32_t d = G.ops[i].dst;
       if (!used[d]) dump_words = std::max(dump_words, slot_words(value_layout(G.width[d], false), G.width[d]));
@@ -637,6 +687,7 @@ int compile_program(const rtlsim_ir *ir, uint32_t op_lanes, uint32_t smem_limit_
     };
     for (uint32_t r : reg_sinks[p]) add_sink(CODE_ST_REG, G.reg_d[r], G.width[G.reg_q[r]], r);
     for (uint32_t o : out_sinks[p]) add_sink(CODE_ST_OUT, G.output_sig[o], G.width[G.output_sig[o]], o);
+    for (uint32_t k : port_sinks[p]) add_sink(CODE_ST_PORT, G.port_sig[k], G.width[G.port_sig[k]], k);
     for (uint32_t i : ops_p)
       if (is_xnet[G.ops[i].dst] || (spilled.count(G.ops[i].dst) && spill_uses.count(G.ops[i].dst)))
         add_sink(CODE_ST_X, G.ops[i].dst, G.width[G.ops[i].dst], G.ops[i].dst);
@@ -909,7 +960,7 @@ int compile_program(const rtlsim_ir *ir, uint32_t op_lanes, uint32_t smem_limit_
     // compute op -> bit-sliced, narrow or wide descriptor
     auto emit_compute = [&](uint32_t opc, int32_t vd, int ar, const int32_t *src, uint32_t imm, int32_t step) {
       const Value &D = vals[vd];
-      bool allbit = D.width == 1, narrow = D.width <= 32;
+      bool allbit = D.width == 1 && opc != RTLSIM_OP_MEMRD, narrow = D.width <= 32;
       for (int k = 0; k < ar; k++) {
         const Value &v = vals[src[k]];
         allbit = allbit && v.width == 1;
@@ -946,7 +997,7 @@ int compile_program(const rtlsim_ir *ir, uint32_t op_lanes, uint32_t smem_limit_
         d.x = opc | (lay[0] << 8) | (lay[1] << 11) | (lay[2] << 14) | (D.layout << 17) | (D.width << 20) |
               (wsrc[0] << 26);
         d.y = D.slot | (off[0] << 16);
-        d.z = off[1] | (off[2] << 16);
+        d.z = opc == RTLSIM_OP_MEMRD ? imm : off[1] | (off[2] << 16);   // MEMRD: the memory
         d.w = wsrc[1] | (imm << 6) | ((ar >= 2 ? 1u : 0u) << 11) | ((ar >= 3 ? 1u : 0u) << 12) |
               (fast_handler(opc, ar, lay, D.layout, wsrc, D.width) << 13);
         G.n_narrow++;
@@ -980,7 +1031,7 @@ int compile_program(const rtlsim_ir *ir, uint32_t op_lanes, uint32_t smem_limit_
       const uint32_t i = ops_p[j];
       const rtlsim_op &o = G.ops[i];
       emit_compute(o.opcode, vid(o.dst), arity(o.opcode), op_vals[j].data(),
-                   o.opcode == RTLSIM_OP_SLICE ? o.imm : 0u, op_step[i]);
+                   (o.opcode == RTLSIM_OP_SLICE || o.opcode == RTLSIM_OP_MEMRD) ? o.imm : 0u, op_step[i]);
     }
     for (const Synth &sy : synth) {
       const int32_t src = flex_src(sy.src_sig);
@@ -999,6 +1050,9 @@ int compile_program(const rtlsim_ir *ir, uint32_t op_lanes, uint32_t smem_limit_
         bytes_state += lane_bytes(ri.width);
       } else if (sk.code == CODE_ST_OUT) {
         d.z = out_word[sk.idx];
+        bytes_state += 4.0 * nwords(w);
+      } else if (sk.code == CODE_ST_PORT) {
+        d.z = G.port_word[sk.idx];
         bytes_state += 4.0 * nwords(w);
       } else {
         d.z = row_of_x(sk.idx);
@@ -1085,7 +1139,7 @@ int compile_program(const rtlsim_ir *ir, uint32_t op_lanes, uint32_t smem_limit_
       rows_of(w.b, (w.lays >> 8) & 0xFFu, w.wb, src);
       rows_of(w.c, (w.lays >> 16) & 0xFFu, w.wc, src);
       rows_of(w.d, w.wd <= 32 ? value_layout(w.wd, false) : LC_U32, w.wd, dst);
-    } else if (code == CODE_ST_REG || code == CODE_ST_X || code == CODE_ST_OUT) {
+    } else if (code == CODE_ST_REG || code == CODE_ST_X || code == CODE_ST_OUT || code == CODE_ST_PORT) {
       const uint32_t nw = (d.x >> 12) & 63u, lay = (d.x >> 18) & 7u;
       rows_of(d.y, lay, lay == LC_U32 ? 32 * nw : 32, src);
     } else if (code == CODE_ST_REGC) {

@@ -51,8 +51,8 @@ std::string fmt(const char *f, ...) {
 const char *kCtx32[] = {"smb", "lane", "wl", "N", "tbar"};
 const char *kCtx64[] = {"tb_c0", "tb_c1", "tb_c2", "tb_c3", "tb_n0", "tb_n1", "tb_n2", "tb_n3",
                         "tb_x0", "tb_x1", "tb_x2", "tb_x3", "tb_i0", "tb_i1", "tb_i2", "tb_i3",
-                        "outb", "dig", "wide", "smg"};
-constexpr int kN32 = 5, kN64 = 20;
+                        "outb", "dig", "wide", "smg", "bitl", "memb", "portb"};
+constexpr int kN32 = 5, kN64 = 23;
 
 // Step barrier (RTLSIM_JIT_TBAR, read per build): 0 = one CTA-wide barrier
 // per step (all K tiles x L op-lanes); 1 = a named barrier per tile (id
@@ -140,6 +140,7 @@ struct Em {
   uint32_t ninst = 0;                       // instances begun in this pass
   std::unordered_map<uint64_t, uint32_t> cur;   // row key -> current instance
   std::vector<WideRec> *wrec = nullptr;     // generic-path records with compacted offsets
+  std::vector<uint32_t> *bittab = nullptr;  // bit-op batch table (uint4 per op)
   std::unordered_map<uint64_t, Fwd> fwd;
   uint32_t nr = 0, nrd = 0, np = 0, nlab = 0;
   // N_pad the code is specialised for (0: generic, row stride from %N at run
@@ -415,6 +416,33 @@ std::string reg_of(Em &e, const std::string &v) {
   return v;
 }
 
+// -------------------------------------------------------- memories --
+// word t of entry idx (a register holding the lane's canonical index) of
+// memory m: 0 when idx >= depth. Memory rows are [row][N_pad] u32; %memb is
+// this stimulus' column. The rows differ per lane, so the load is a gather.
+thread_local const Program *t_prog = nullptr;   // the program being emitted (memory shapes)
+std::string emit_mem_read(Em &e, const std::string &idx, uint32_t m, uint32_t t) {
+  const Program &G = *t_prog;
+  const uint32_t nw = nwords(G.mem_width[m]), row = G.mem_row0[m] + t;
+  std::string p = e.P(), off = e.RD(), a = e.RD(), v = e.R();
+  e.l(fmt("setp.lt.u32 %s, %s, %u", p.c_str(), idx.c_str(), G.mem_depth[m]));
+  if (e.nspec) {
+    const uint64_t n4 = 4ull * e.nspec;
+    e.l(fmt("mul.wide.u32 %s, %s, %llu", off.c_str(), idx.c_str(), (unsigned long long)(n4 * nw)));
+    e.l(fmt("add.s64 %s, %s, %llu", a.c_str(), off.c_str(), (unsigned long long)(n4 * row)));
+  } else {
+    std::string k = e.R(), r = e.R();
+    e.l(fmt("mul.lo.u32 %s, %%N4, %u", k.c_str(), nw));
+    e.l(fmt("mul.wide.u32 %s, %s, %s", off.c_str(), idx.c_str(), k.c_str()));
+    e.l(fmt("mul.wide.u32 %s, %%N4, %u", a.c_str(), row));
+    e.l(fmt("add.s64 %s, %s, %s", a.c_str(), a.c_str(), off.c_str()));
+  }
+  e.l(fmt("add.s64 %s, %s, %%memb", a.c_str(), a.c_str()));
+  e.l(fmt("mov.u32 %s, 0", v.c_str()));
+  e.l(fmt("@%s ld.global.u32 %s, [%s]", p.c_str(), v.c_str(), a.c_str()));
+  return v;
+}
+
 // -------------------------------------------------------- narrow ops --
 void emit_narrow(Em &e, const Desc &q) {
   const uint32_t op = q.x & 0xFFu;
@@ -423,6 +451,12 @@ void emit_narrow(Em &e, const Desc &q) {
   const bool hb = (q.w >> 11) & 1u, hc = (q.w >> 12) & 1u;
   const uint32_t d = q.y & 0xFFFFu, a = q.y >> 16, b = q.z & 0xFFFFu, c = q.z >> 16;
   begin_value(e, layout_space(ld), d, 1);
+  if (op == RTLSIM_OP_MEMRD) {   // ARRSEL read: entry V[a] of memory q.z (reading 12)
+    std::string idx = fetch_narrow(e, la, a, wa);
+    std::string v = emit_mem_read(e, idx, q.z, 0);
+    store_narrow(e, ld, d, v);
+    return;
+  }
   if (op == RTLSIM_OP_MUX && la == LC_BIT && hb && hc) {
     // 1-bit select straight from its packed word: the lane's bit moved to
     // bit 31 and sign-filled is the all-ones / zero mask of the LOP3 mux
@@ -622,6 +656,11 @@ void emit_wide(Em &e, const WideRec &w, uint32_t idx) {
   C.off = w.c; C.w = w.wc; C.lay = (w.lays >> 16) & 0xFFu;
   if (wd <= 32) begin_value(e, layout_space(value_layout(wd, false)), w.d, 1);
   else begin_value(e, SP_W, w.d, nd);
+  if (op == RTLSIM_OP_MEMRD) {   // ARRSEL read of a wide entry (reading 12)
+    std::string idx = reg_of(e, wword(e, A, 0, false));
+    for (uint32_t i = 0; i < nd; i++) wstore(e, w.d, wd, i, emit_mem_read(e, idx, w.imm, i));
+    return;
+  }
   auto bin = [&](const char *ins) {
     for (uint32_t i = 0; i < nd; i++) {
       std::string xa = reg_of(e, wword(e, A, i, false)), xb = reg_of(e, wword(e, B, i, false)), r = e.R();
@@ -893,6 +932,14 @@ void emit_dig(Em &e, uint32_t key, const std::string &v) {
 void emit_st(Em &e, uint32_t code, uint32_t cls, uint32_t nw, uint32_t lay, uint32_t slot, uint32_t row,
              uint32_t aux) {
   const bool dg = code == CODE_ST_REG;
+  if (code == CODE_ST_PORT) {   // write-port words of this cycle (applied after the cycle)
+    for (uint32_t i = 0; i < nw; i++) {
+      std::string v = lay == LC_U32 ? lds(e, SP_W, slot + 32 * i) : fetch_narrow(e, lay, slot, 32);
+      std::string addr = gaddr(e, "N4", row + i, "portb");
+      e.l(fmt("st.global.u32 [%s], %s", addr.c_str(), v.c_str()));
+    }
+    return;
+  }
   if (code == CODE_ST_OUT) {
     for (uint32_t i = 0; i < nw; i++) {
       std::string v;
@@ -1042,6 +1089,72 @@ void emit_bit(Em &e, const BitDesc &q) {
   sts(e, SP_S, q.y & 0xFFFFu, r);
 }
 
+// Lane-parallel bit ops (RTLSIM_JIT_BITBATCH=k, default 0 = off): the 1-bit
+// ops of one warp's step that share one truth table (immediates folded in),
+// in groups of >= k; lane i evaluates op i of the group on the packed words
+// (32 stimuli each), its four operand / result slot addresses read from a
+// per-partition table (one LDG.128 per lane): up to 32 ops in ~11 warp
+// instructions instead of ~4-5 each (every lane computing the same word).
+// Measured off by default: config 3 steps hold ~28 bit ops over 4 warps and
+// ~6 truth tables, so groups average 3.3 ops, and batched results can no
+// longer be forwarded in registers (total SASS +2 %).
+uint32_t jit_bitbatch() {
+  const char *e = getenv("RTLSIM_JIT_BITBATCH");
+  return e ? (uint32_t)atoi(e) : 0u;
+}
+// truth table with the immediate operands substituted (they become unused)
+uint32_t bit_fold_lut(const BitDesc &q) {
+  uint32_t lut = q.x & 0xFFu;
+  const uint32_t immf = q.x >> 8;
+  const uint32_t f[3] = {q.y >> 16, q.z & 0xFFFFu, q.z >> 16};
+  for (uint32_t k = 0; k < 3; k++) {
+    if (!(immf & (1u << k))) continue;
+    uint32_t n = 0;
+    for (uint32_t j = 0; j < 8; j++) {
+      const uint32_t src = (j & ~(1u << k)) | ((f[k] & 1u) << k);
+      n |= ((lut >> src) & 1u) << j;
+    }
+    lut = n;
+  }
+  return lut;
+}
+bool lut_uses(uint32_t lut, uint32_t k) {
+  for (uint32_t idx = 0; idx < 8; idx++)
+    if (((lut >> idx) & 1u) != ((lut >> (idx ^ (1u << k))) & 1u)) return true;
+  return false;
+}
+void emit_bit_batch(Em &e, const std::vector<BitDesc> &ops, uint32_t lut) {
+  const uint32_t n = (uint32_t)ops.size();
+  for (const BitDesc &q : ops) begin_value(e, SP_S, q.y & 0xFFFFu, 1, true);
+  const uint32_t base = e.bittab ? (uint32_t)(e.bittab->size() / 4) : 0;
+  for (const BitDesc &q : ops) {
+    const uint32_t d = q.y & 0xFFFFu;
+    const uint32_t f[3] = {q.y >> 16, q.z & 0xFFFFu, q.z >> 16};
+    uint32_t ent[4];
+    for (uint32_t k = 0; k < 3; k++) {
+      if (lut_uses(lut, k)) {
+        note_read(e, SP_S, f[k]);
+        ent[k] = xoff(e, SP_S, f[k]) * 4;
+      } else {
+        ent[k] = xoff(e, SP_S, d) * 4;   // ignored input: the lane's own result word
+      }
+    }
+    ent[3] = xoff(e, SP_S, d) * 4;
+    if (e.bittab && !e.dry) e.bittab->insert(e.bittab->end(), ent, ent + 4);
+  }
+  std::string p = e.P(), t[4], a[4], v[3], r = e.R();
+  for (int k = 0; k < 4; k++) { t[k] = e.R(); a[k] = e.R(); }
+  for (int k = 0; k < 3; k++) v[k] = e.R();
+  e.l(fmt("setp.lt.u32 %s, %%lane, %u", p.c_str(), n));
+  e.l(fmt("@%s ld.global.nc.v4.u32 {%s, %s, %s, %s}, [%%bitl+%u]", p.c_str(), t[0].c_str(), t[1].c_str(),
+          t[2].c_str(), t[3].c_str(), base * 16));
+  for (int k = 0; k < 4; k++) e.l(fmt("add.u32 %s, %s, %%smb", a[k].c_str(), t[k].c_str()));
+  for (int k = 0; k < 3; k++) e.l(fmt("@%s ld.shared.u32 %s, [%s]", p.c_str(), v[k].c_str(), a[k].c_str()));
+  e.l(fmt("lop3.b32 %s, %s, %s, %s, 0x%02x", r.c_str(), v[0].c_str(), v[1].c_str(), v[2].c_str(), lop3_lut(lut)));
+  e.l(fmt("@%s st.shared.u32 [%s], %s", p.c_str(), a[3].c_str(), r.c_str()));
+  for (const BitDesc &q : ops) opaque_write(e, SP_S, q.y & 0xFFFFu);
+}
+
 // RTLSIM_JIT_STATS: PTX instruction lines per descriptor kind (stderr at exit)
 struct EmitStats {
   std::mutex mu;
@@ -1097,7 +1210,7 @@ void emit_desc_(Em &e, const Program &G, const Desc &q) {
     case CODE_LD_X: emit_ld(e, 2, cls, q.z, q.y, nw); break;
     case CODE_LD_IN: emit_ld(e, 3, cls, q.z, q.y, nw); break;
     case CODE_LD_CONST: emit_ld_const(e, G, q.y, q.z, nw, ((q.x >> 18) & 1u) != 0); break;
-    case CODE_ST_REG: case CODE_ST_X: case CODE_ST_OUT:
+    case CODE_ST_REG: case CODE_ST_X: case CODE_ST_OUT: case CODE_ST_PORT:
       emit_st(e, code, cls, nw, (q.x >> 18) & 7u, q.y, q.z, q.w);
       break;
     case CODE_ST_REGC:
@@ -1145,10 +1258,12 @@ uint64_t jit_fwd_ops(bool compact) {
 
 std::string step_function(const Program &G, const std::string &name, uint32_t s0, uint32_t s1, bool dig,
                           uint32_t nspec, bool to_end, uint32_t *tile_words = nullptr,
-                          std::vector<WideRec> *wrec_out = nullptr) {
+                          std::vector<WideRec> *wrec_out = nullptr, std::vector<uint32_t> *bittab_out = nullptr) {
+  t_prog = &G;
   const bool compact = jit_compact_env(G) && to_end && tile_words;
   std::vector<Em::Inst> insts;
   std::vector<WideRec> wrec_probe, wrec_final;
+  std::vector<uint32_t> bit_probe;
   // dry pass: which warp writes which slot in which step (forwarding validity)
   WriteLog log;
   {
@@ -1177,6 +1292,7 @@ std::string step_function(const Program &G, const std::string &name, uint32_t s0
   e.compact = compact;
   e.inst = &insts;
   e.wrec = probe ? &wrec_probe : &wrec_final;
+  e.bittab = probe ? &bit_probe : bittab_out;
   std::vector<std::string> labs(G.L);
   std::string tbl = e.L("T"), end = e.L("E");
   if (G.L > 1) {
@@ -1194,11 +1310,36 @@ std::string step_function(const Program &G, const std::string &name, uint32_t s0
     e.warp = w;
     for (uint32_t s = s0; s < s1; s++) {
       e.step = (int32_t)s;
-      for (uint32_t k = G.bit_ptr[s] + w; k < G.bit_ptr[s + 1]; k += G.L) {
-        const size_t from = e.s.size();
-        e.opn++;
-        emit_bit(e, G.bitdesc[k]);
-        note_kind(e, "bit", from);
+      {
+        // this warp's bit ops of the step: groups sharing a truth table
+        // (immediates folded in) of >= RTLSIM_JIT_BITBATCH ops run
+        // lane-parallel, the rest one by one
+        const uint32_t bb = jit_bitbatch();
+        std::map<uint32_t, std::vector<BitDesc>> groups;
+        std::vector<BitDesc> single;
+        for (uint32_t k = G.bit_ptr[s] + w; k < G.bit_ptr[s + 1]; k += G.L) {
+          if (bb) groups[bit_fold_lut(G.bitdesc[k])].push_back(G.bitdesc[k]);
+          else single.push_back(G.bitdesc[k]);
+        }
+        for (auto &g : groups) {
+          if (g.second.size() < bb) {
+            single.insert(single.end(), g.second.begin(), g.second.end());
+            continue;
+          }
+          for (size_t i = 0; i < g.second.size(); i += 32) {
+            std::vector<BitDesc> part(g.second.begin() + i, g.second.begin() + std::min(g.second.size(), i + 32));
+            const size_t from = e.s.size();
+            e.opn += part.size();
+            emit_bit_batch(e, part, g.first);
+            note_kind(e, "bitbatch", from);
+          }
+        }
+        for (const BitDesc &q : single) {
+          const size_t from = e.s.size();
+          e.opn++;
+          emit_bit(e, q);
+          note_kind(e, "bit", from);
+        }
       }
       for (uint32_t k = G.step_ptr[s * G.L + w]; k < G.step_ptr[s * G.L + w + 1]; k++) emit_desc(e, G, G.desc[k]);
       e.l("cp.async.commit_group");
@@ -1341,7 +1482,7 @@ std::string jit_partition_ptx(const Program &G, uint32_t q, const std::string &r
   for (size_t g = 0; g < groups.size(); g++)
     mod += step_function(G, fmt("rtl_steps_%zu", g), groups[g].first, groups[g].second, dig, nspec,
                          groups[g].second == s1, compact ? &tile_words : nullptr,
-                         compact ? &info->wide : nullptr) + "\n";
+                         compact ? &info->wide : nullptr, &info->bittab) + "\n";
   // shared memory per tile: the compacted extent, or the schedule's slots
   const uint32_t tbytes = compact ? std::max<uint32_t>(16u, ((tile_words * 4u) + 15u) & ~15u) : jit_tile_bytes(G);
   info->tile_bytes = tbytes;
@@ -1380,6 +1521,12 @@ std::string jit_partition_ptx(const Program &G, uint32_t q, const std::string &r
              "\tsetp.eq.u64 %%pz, %%digb, 0;\n\tselp.b64 %%dig, 0, %%t64, %%pz;\n",
              offsetof(JitParams, digest));
   mod += fmt("\tld.param.u64 %%wide, [prm+%zu];\n", offsetof(JitParams, wide));
+  mod += fmt("\tld.param.u64 %%b64, [prm+%zu];\n\tmul.wide.u32 %%t64, %%lane, 16;\n\tadd.u64 %%bitl, %%b64, %%t64;\n",
+             offsetof(JitParams, bittab));
+  // memory / write-port arenas: this stimulus' column ([row][N_pad] u32)
+  mod += fmt("\tld.param.u64 %%b64, [prm+%zu];\n\tmul.wide.u32 %%t64, %%s, 4;\n\tadd.u64 %%memb, %%b64, %%t64;\n",
+             offsetof(JitParams, mem));
+  mod += fmt("\tld.param.u64 %%b64, [prm+%zu];\n\tadd.u64 %%portb, %%b64, %%t64;\n", offsetof(JitParams, port));
   mod += fmt("\tmov.u32 %%smb, dyn_smem;\n\tmad.lo.u32 %%smb, %%tsub, %u, %%smb;\n\tcvta.shared.u64 %%smg, dyn_smem;\n"
              "\tmul.wide.u32 %%t64, %%tsub, %u;\n\tadd.u64 %%smg, %%smg, %%t64;\n",
              tbytes, tbytes);
@@ -1399,6 +1546,27 @@ std::string jit_partition_ptx(const Program &G, uint32_t q, const std::string &r
   }
   mod += "\tret;\n}\n";
   return mod;
+}
+
+// SASS instructions in a cubin: the sizes of its .text.* sections (ELF64) /
+// 16 bytes per Blackwell instruction
+static uint64_t cubin_sass_instructions(const std::vector<char> &b) {
+  if (b.size() < 64 || memcmp(b.data(), "\x7f" "ELF", 4) != 0 || b[4] != 2) return 0;
+  auto u16 = [&](size_t o) { uint16_t v; memcpy(&v, b.data() + o, 2); return v; };
+  auto u32 = [&](size_t o) { uint32_t v; memcpy(&v, b.data() + o, 4); return v; };
+  auto u64 = [&](size_t o) { uint64_t v; memcpy(&v, b.data() + o, 8); return v; };
+  const uint64_t shoff = u64(0x28);
+  const uint16_t shentsize = u16(0x3A), shnum = u16(0x3C), shstrndx = u16(0x3E);
+  if (shoff + (uint64_t)shnum * shentsize > b.size() || shstrndx >= shnum) return 0;
+  const uint64_t stroff = u64(shoff + (uint64_t)shstrndx * shentsize + 0x18);
+  uint64_t total = 0;
+  for (uint16_t i = 0; i < shnum; i++) {
+    const size_t h = shoff + (size_t)i * shentsize;
+    const uint64_t name = stroff + u32(h);
+    if (name + 6 > b.size()) continue;
+    if (strncmp(b.data() + name, ".text.", 6) == 0) total += u64(h + 0x20);
+  }
+  return total / 16;
 }
 
 static int compile_ptx(const std::string &ptx, bool o3, std::vector<char> *cubin, std::string *err) {
@@ -1561,6 +1729,21 @@ int jit_build(const Program &G, const std::string &rt_ptx_path, uint32_t smem_by
     out->wide_base[q] = (uint32_t)wall.size();
     wall.insert(wall.end(), infos[q].wide.begin(), infos[q].wide.end());
   }
+  std::vector<uint32_t> ball;
+  out->bit_base.assign(NP, 0);
+  for (uint32_t q = 0; q < NP; q++) {
+    out->bit_base[q] = (uint32_t)(ball.size() / 4);
+    ball.insert(ball.end(), infos[q].bittab.begin(), infos[q].bittab.end());
+  }
+  if (device >= 0 && !ball.empty()) {
+    cudaError_t e = cudaMalloc((void **)&out->d_bittab, ball.size() * 4);
+    if (e == cudaSuccess) e = cudaMemcpy(out->d_bittab, ball.data(), ball.size() * 4, cudaMemcpyHostToDevice);
+    if (e != cudaSuccess) {
+      *err = std::string("JIT bit-op table: ") + cudaGetErrorString(e);
+      cudaGetLastError();
+      return RTLSIM_E_CUDA;
+    }
+  }
   if (device >= 0 && !wall.empty()) {
     cudaError_t e = cudaMalloc((void **)&out->d_wide, wall.size() * sizeof(WideRec));
     if (e == cudaSuccess) e = cudaMemcpy(out->d_wide, wall.data(), wall.size() * sizeof(WideRec), cudaMemcpyHostToDevice);
@@ -1573,6 +1756,7 @@ int jit_build(const Program &G, const std::string &rt_ptx_path, uint32_t smem_by
   for (uint32_t q = 0; q < NP; q++) {
     if (cubins[q].empty()) continue;
     out->cubin_bytes += cubins[q].size();
+    out->sass_instructions += cubin_sass_instructions(cubins[q]);
     if (device < 0) continue;
     cudaError_t e = cudaLibraryLoadData(&out->libs[q], cubins[q].data(), nullptr, nullptr, 0, nullptr, nullptr, 0);
     if (e != cudaSuccess && from_cache[q]) {   // a damaged cached cubin: compile it again
@@ -1607,6 +1791,8 @@ uint32_t jit_default_tiles(bool compact) {
 void jit_free(JitKernels *k) {
   if (k->d_wide) cudaFree(k->d_wide);
   k->d_wide = nullptr;
+  if (k->d_bittab) cudaFree(k->d_bittab);
+  k->d_bittab = nullptr;
   for (cudaLibrary_t l : k->libs)
     if (l) cudaLibraryUnload(l);
   k->libs.clear();

@@ -27,8 +27,11 @@ struct JitParams {
   uint64_t wide;                             // WideRec array (generic path)
   uint32_t N;                                // N_pad
   uint32_t tpc;                              // 32-stimulus tiles per CTA (warps of equal op-lane share code)
+  uint64_t bittab;                           // this partition's bit-op batch table (uint4 per op) or 0
+  uint64_t mem;                              // memory arena [MR][N_pad] u32 (MEMRD) or 0
+  uint64_t port;                             // write-port arena [PW][N_pad] u32 (CODE_ST_PORT) or 0
 };
-static_assert(sizeof(JitParams) == 160, "JitParams layout is hard-coded in the PTX generator");
+static_assert(sizeof(JitParams) == 184, "JitParams layout is read through offsetof in the PTX generator");
 
 // Maximum tiles per CTA the kernels are compiled for (.maxntid 32 * L * kJitMaxTiles).
 constexpr uint32_t kJitMaxTiles = 16;
@@ -42,6 +45,7 @@ inline uint32_t jit_tile_bytes(const Program &G) { return ((G.smem_words * 4u) +
 struct JitPartInfo {
   uint32_t tile_bytes = 0;          // shared memory per tile (compacted slots; 0 = jit_tile_bytes(G))
   std::vector<WideRec> wide;        // generic-path records with compacted slot offsets (or empty)
+  std::vector<uint32_t> bittab;     // lane-parallel bit-op batches: {a, b, c, d} smem byte offsets per op
 };
 
 struct JitKernels {
@@ -49,6 +53,8 @@ struct JitKernels {
   std::vector<uint32_t> tile_bytes; // per exec-order partition: shared memory per tile
   std::vector<uint32_t> wide_base;  // per partition: first record in d_wide (compacted records)
   WideRec *d_wide = nullptr;        // compacted generic-path records of all partitions (or null)
+  std::vector<uint32_t> bit_base;   // per partition: first uint4 of its bit-op table in d_bittab
+  uint32_t *d_bittab = nullptr;     // bit-op batch tables of all partitions (or null)
   bool compact = false;             // slot compaction (L == 1 kernels)
   std::vector<cudaKernel_t> kern;   // per exec-order partition (nullptr: empty partition)
   double gen_s = 0, compile_s = 0;
@@ -56,6 +62,7 @@ struct JitKernels {
   uint32_t tmax = 1;                // tiles per CTA the kernels were built for
   uint32_t nspec = 0;               // N_pad the row offsets were specialised for (0: generic)
   size_t ptx_bytes = 0, cubin_bytes = 0;
+  uint64_t sass_instructions = 0;   // .text of every partition kernel (each executed once per tile-cycle)
   uint32_t cache_hits = 0;          // partitions served from RTLSIM_JIT_CACHE
 };
 

@@ -14,6 +14,7 @@
 // N2/N3: stimulus / output transposes between the user layout [N][T][W]
 // (stimulus-major) and the device layout [T][W][N] (coalesced per warp).
 // N4: register init / import / export.
+#include <algorithm>
 #include <cstdint>
 
 #include "device_ops.cuh"
@@ -570,6 +571,69 @@ cudaError_t launch_reg_digest(Arena a, const RegWord *map, uint32_t RW, uint32_t
                               unsigned long long *dig, cudaStream_t st) {
   if (N == 0) return cudaSuccess;
   reg_digest_kernel<<<(N + 255u) / 256u, 256, 0, st>>>(a, map, RW, N, N_pad, dig);
+  return cudaGetLastError();
+}
+
+// ------------------------------------------------------------ memories --
+// Memory write ports at the clock edge (reading 12): after the
+// cycle's partitions stored every port's (address, data, enable) words in the
+// port arena, one thread per stimulus applies the ports in order (a later port
+// wins): entry V[addr] := V[data] zero-extended / truncated to the memory
+// width when V[en] != 0 and V[addr] < depth. Memory rows are [row][N_pad] u32.
+__global__ void mem_commit_kernel(uint32_t *__restrict__ mem, const uint32_t *__restrict__ port,
+                                  const MemPortDev *__restrict__ ports, uint32_t n_ports, uint32_t N,
+                                  uint32_t N_pad) {
+  const uint32_t s = blockIdx.x * blockDim.x + threadIdx.x;
+  if (s >= N) return;
+  for (uint32_t p = 0; p < n_ports; p++) {
+    const MemPortDev P = ports[p];
+    uint32_t en = 0;
+    for (uint32_t t = 0; t < (P.en_width + 31u) / 32u; t++) en |= port[(size_t)(P.en_word + t) * N_pad + s];
+    if (!en) continue;
+    const uint32_t idx = port[(size_t)P.addr_word * N_pad + s];
+    if (idx >= P.depth) continue;
+    const uint32_t nwm = (P.width + 31u) / 32u, nwd = (P.data_width + 31u) / 32u;
+    for (uint32_t t = 0; t < nwm; t++) {
+      uint32_t v = t < nwd ? port[(size_t)(P.data_word + t) * N_pad + s] : 0u;
+      if (t == nwm - 1 && (P.width & 31u)) v &= (1u << (P.width & 31u)) - 1u;
+      mem[(size_t)(P.row0 + idx * nwm + t) * N_pad + s] = v;
+    }
+  }
+}
+
+cudaError_t launch_mem_commit(uint32_t *mem, const uint32_t *port, const MemPortDev *ports, uint32_t n_ports,
+                              uint32_t N, uint32_t N_pad, cudaStream_t st) {
+  if (!n_ports || !N) return cudaSuccess;
+  mem_commit_kernel<<<(N + 255u) / 256u, 256, 0, st>>>(mem, port, ports, n_ports, N, N_pad);
+  return cudaGetLastError();
+}
+
+// memory rows <- their initial values (the same for every stimulus)
+__global__ void mem_init_kernel(uint32_t *__restrict__ mem, const uint32_t *__restrict__ init, uint32_t N_pad) {
+  const uint32_t r = blockIdx.y;
+  const uint32_t v = init[r];
+  for (uint32_t s = blockIdx.x * blockDim.x + threadIdx.x; s < N_pad; s += gridDim.x * blockDim.x)
+    mem[(size_t)r * N_pad + s] = v;
+}
+
+cudaError_t launch_mem_init(uint32_t *mem, const uint32_t *init, uint32_t MR, uint32_t N_pad, cudaStream_t st) {
+  if (!MR) return cudaSuccess;
+  mem_init_kernel<<<dim3(std::min<uint32_t>(64u, (N_pad + 255u) / 256u), MR), 256, 0, st>>>(mem, init, N_pad);
+  return cudaGetLastError();
+}
+
+// memory rows [MR][N_pad] -> dst [N][MR]
+__global__ void mem_export_kernel(const uint32_t *__restrict__ mem, uint32_t MR, uint32_t N, uint32_t N_pad,
+                                  uint32_t *__restrict__ dst) {
+  const uint32_t r = blockIdx.y;
+  for (uint32_t s = blockIdx.x * blockDim.x + threadIdx.x; s < N; s += gridDim.x * blockDim.x)
+    dst[(size_t)s * MR + r] = mem[(size_t)r * N_pad + s];
+}
+
+cudaError_t launch_mem_export(const uint32_t *mem, uint32_t MR, uint32_t N, uint32_t N_pad, uint32_t *dst,
+                              cudaStream_t st) {
+  if (!MR || !N) return cudaSuccess;
+  mem_export_kernel<<<dim3(std::min<uint32_t>(64u, (N + 255u) / 256u), MR), 256, 0, st>>>(mem, MR, N, N_pad, dst);
   return cudaGetLastError();
 }
 

@@ -84,6 +84,15 @@ cudaError_t launch_regs_export(Arena a, const RegWord *map, uint32_t RW, uint32_
 // per-stimulus register digest
 cudaError_t launch_toggle_coverage(Arena cur, Arena nxt, const RegWord *map, uint32_t RW, uint32_t N,
                                    uint32_t N_pad, uint32_t *cov, cudaStream_t st);
+// memories (JIT backend): write-port commit after each cycle, init, export
+struct MemPortDev {
+  uint32_t row0, depth, width, addr_word, data_word, data_width, en_word, en_width;
+};
+cudaError_t launch_mem_commit(uint32_t *mem, const uint32_t *port, const MemPortDev *ports, uint32_t n_ports,
+                              uint32_t N, uint32_t N_pad, cudaStream_t st);
+cudaError_t launch_mem_init(uint32_t *mem, const uint32_t *init, uint32_t MR, uint32_t N_pad, cudaStream_t st);
+cudaError_t launch_mem_export(const uint32_t *mem, uint32_t MR, uint32_t N, uint32_t N_pad, uint32_t *dst,
+                              cudaStream_t st);
 cudaError_t launch_reg_digest(Arena a, const RegWord *map, uint32_t RW, uint32_t N, uint32_t N_pad,
                               unsigned long long *dig, cudaStream_t st);
 

@@ -48,6 +48,7 @@ enum : uint32_t {
   CODE_ST_REG = 96,     // state_next[cls][row z ..] <- slot y ; w = register word index
   CODE_ST_X = 97,       // xnet[cls][row z ..] <- slot y
   CODE_ST_OUT = 98,     // out_chunk[c][word z ..] <- slot y
+  CODE_ST_PORT = 100,   // JIT only: memory write-port word z <- slot y (port arena [PW][N])
   CODE_ST_REGC = 99,    // JIT only: state_next <- slot y converted from the source's
                         // width / layout (x >> 21) to the register's (z >> 20); z & 0xFFFFF = row
 };
@@ -203,6 +204,18 @@ struct Program {
   std::vector<uint32_t> uptr;           // [n_steps * L + 1] offsets into ustream
   uint32_t zero_off = 0;                // word offset of the 32-word zero row
   uint64_t u_class_count[U_NCLASS] = {};
+  // ---- memories (ARRSEL, reading 12; JIT backend only)
+  std::vector<uint16_t> mem_width;
+  std::vector<uint32_t> mem_depth, mem_row0;  // first u32 row of each memory in the memory arena
+  std::vector<uint32_t> mem_init;             // MR words: row r's initial value (all stimuli)
+  uint32_t MR = 0;                            // memory arena rows (u32, [MR][N]) = words per stimulus
+  struct WPort {
+    uint32_t mem, addr_word, data_word, data_width, en_word, en_width;   // words in the port arena
+  };
+  std::vector<WPort> wports;                  // in port order (a later port wins)
+  std::vector<uint32_t> port_sig;             // signals stored to the port arena each cycle
+  std::vector<uint32_t> port_word;            // their first word
+  uint32_t PW = 0;                            // port arena words per stimulus
   // ---- stats
   uint64_t word_ops = 0, n_bitops = 0, n_wide = 0, n_narrow = 0, n_ld = 0, n_st = 0;
   double b_floor = 0, b_state = 0, b_part = 0, b_spill = 0;

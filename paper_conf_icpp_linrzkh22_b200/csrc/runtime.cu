@@ -89,6 +89,10 @@ struct rtlsim_ctx {
   InStride in_stride{};
   RegWord *d_inmap = nullptr;
   uint32_t *d_cov = nullptr;          // RTLSIM_F_COVERAGE: [RW] toggle bitmap (N5)
+  uint32_t *d_mem = nullptr;          // memories: [MR][N_pad] u32 (per-stimulus entries)
+  uint32_t *d_port = nullptr;         // write-port words of the current cycle [PW][N_pad]
+  MemPortDev *d_ports = nullptr;      // port descriptors (static)
+  uint32_t *d_meminit = nullptr;      // [MR] initial row values (static)
   uint32_t *d_out[2]{}, *d_raw[2]{}, *d_outu[2]{};
   unsigned long long *d_dig[2]{}, *d_digu[2]{};
   uint32_t *h_in[2]{}, *h_out[2]{};
@@ -158,7 +162,7 @@ static void free_binding(rtlsim_ctx *ctx) {
     ctx->h_dig[b] = nullptr;
     ctx->ev_used[b] = false;
   }
-  ctx->d_cov = nullptr;
+  ctx->d_cov = ctx->d_mem = ctx->d_port = nullptr;
   ctx->src = SRC_NONE;
   ctx->N = ctx->T = ctx->cycle = 0;
   ctx->device_bytes = ctx->static_bytes;
@@ -221,6 +225,12 @@ extern "C" int rtlsim_load(const rtlsim_ir *ir, const rtlsim_options *opt, rtlsi
     g_load_error = err;
     delete ctx;
     return rc;
+  }
+  if ((ctx->prog.MR || !ctx->prog.wports.empty()) && !(ctx->opt.flags & RTLSIM_F_JIT)) {
+    // memories (ARRSEL reads, write ports) are generated code only
+    g_load_error = "memories (MEMRD / write ports) need RTLSIM_F_JIT";
+    delete ctx;
+    return RTLSIM_E_UNSUPPORTED;
   }
   const bool legacy = (ctx->opt.flags & RTLSIM_F_V4) == 0;
   if ((ctx->opt.flags & RTLSIM_F_JIT) && !ctx->opt.smem_limit &&
@@ -334,6 +344,14 @@ extern "C" int rtlsim_load(const rtlsim_ir *ir, const rtlsim_options *opt, rtlsi
   if (e == cudaSuccess) e = up((void **)&ctx->d_mask, G.in_mask.data(), G.in_mask.size() * 4);
   if (e == cudaSuccess) e = up((void **)&ctx->d_regmap, regmap.data(), regmap.size() * sizeof(RegWord));
   if (e == cudaSuccess) e = up((void **)&ctx->d_reginit, G.reg_init.data(), G.reg_init.size() * 4);
+  if (!G.wports.empty() || G.MR) {
+    std::vector<MemPortDev> mp;
+    for (const Program::WPort &w : G.wports)
+      mp.push_back(MemPortDev{G.mem_row0[w.mem], G.mem_depth[w.mem], G.mem_width[w.mem], w.addr_word, w.data_word,
+                              w.data_width, w.en_word, w.en_width});
+    if (e == cudaSuccess) e = up((void **)&ctx->d_ports, mp.data(), mp.size() * sizeof(MemPortDev));
+    if (e == cudaSuccess) e = up((void **)&ctx->d_meminit, G.mem_init.data(), G.mem_init.size() * 4);
+  }
   if (e == cudaSuccess) e = eval_set_smem(std::max<uint32_t>(ctx->smem_bytes, 1024));
   if (e == cudaSuccess) {
     if (ctx->opt.cuda_stream) {
@@ -382,6 +400,10 @@ static int alloc_arena(rtlsim_ctx *ctx, Arena *a, const uint32_t rows[4]) {
 
 static int reset_regs(rtlsim_ctx *ctx) {
   Program &G = ctx->prog;
+  if (G.MR && ctx->d_mem) {   // memories back to their initial contents
+    CK(launch_mem_init(ctx->d_mem, ctx->d_meminit, G.MR, ctx->N_pad, ctx->st));
+    ctx->launches++;
+  }
   CK(launch_regs_import(ctx->d_reginit, 0, ctx->d_regmap, G.RW, (uint32_t)ctx->N, ctx->N_pad, ctx->state[0],
                         ctx->st));
   ctx->launches++;
@@ -411,6 +433,8 @@ static int bind_common(rtlsim_ctx *ctx, uint64_t N, uint64_t T) {
   for (int b = 0; b < 2; b++)
     if ((rc = alloc_arena(ctx, &ctx->state[b], G.rows)) != RTLSIM_OK) return rc;
   if ((rc = alloc_arena(ctx, &ctx->xnet, G.xrows)) != RTLSIM_OK) return rc;
+  if (G.MR) CK(dalloc(ctx, (void **)&ctx->d_mem, (size_t)G.MR * ctx->N_pad * 4, true));
+  if (G.PW) CK(dalloc(ctx, (void **)&ctx->d_port, (size_t)G.PW * ctx->N_pad * 4, true));
   if ((ctx->opt.flags & RTLSIM_F_COVERAGE) && G.RW) {
     CK(dalloc(ctx, (void **)&ctx->d_cov, (size_t)G.RW * 4, true));
     CK(cudaMemsetAsync(ctx->d_cov, 0, (size_t)G.RW * 4, ctx->st));
@@ -644,6 +668,9 @@ static int launch_chunk(rtlsim_ctx *ctx, int b, uint64_t cycle0, uint32_t nc, bo
           jp.digest = digest ? (uint64_t)(ctx->d_dig[b] + (size_t)c * ctx->N_pad) : 0;
           jp.wide = JK.d_wide ? (uint64_t)(JK.d_wide + JK.wide_base[q]) : (uint64_t)ctx->d_wide;
           jp.N = ctx->N_pad;
+          jp.bittab = JK.d_bittab ? (uint64_t)(JK.d_bittab + 4ull * JK.bit_base[q]) : 0;
+          jp.mem = (uint64_t)ctx->d_mem;
+          jp.port = (uint64_t)ctx->d_port;
           jp.tpc = jit_tiles_per_cta(ctx, JK, q);
           void *args[] = {&jp};
           e = cudaLaunchKernel((const void *)JK.kern[q], dim3(ctx->N_pad / 32u / jp.tpc),
@@ -662,6 +689,11 @@ static int launch_chunk(rtlsim_ctx *ctx, int b, uint64_t cycle0, uint32_t nc, bo
         }
         if (e != cudaSuccess) return e;
       }
+      if (!G.wports.empty()) {   // memory write ports at the clock edge, after every partition
+        cudaError_t e = launch_mem_commit(ctx->d_mem, ctx->d_port, ctx->d_ports, (uint32_t)G.wports.size(),
+                                          (uint32_t)ctx->N, ctx->N_pad, cap);
+        if (e != cudaSuccess) return e;
+      }
       if (ctx->d_cov) {   // N5: toggles of this cycle's register update
         const uint32_t par = (uint32_t)(((cycle0 & 1ull) + c) & 1ull);
         cudaError_t e = launch_toggle_coverage(ctx->state[par], ctx->state[par ^ 1u], ctx->d_regmap, G.RW,
@@ -675,7 +707,7 @@ static int launch_chunk(rtlsim_ctx *ctx, int b, uint64_t cycle0, uint32_t nc, bo
     // the paper's stream-based baseline (Table 4): the same per-(cycle,
     // partition) launches issued one by one every chunk, no graph
     CK(issue(ctx->st));
-    ctx->launches += (uint64_t)nc * (G.part_steps.size() - 1 + (ctx->d_cov ? 1 : 0));
+    ctx->launches += (uint64_t)nc * (G.part_steps.size() - 1 + (ctx->d_cov ? 1 : 0) + (G.wports.empty() ? 0 : 1));
     if (timing) {
       CK(cudaEventRecord(tm.b, ctx->st));
       ctx->timed_pending.push_back(tm);
@@ -702,7 +734,7 @@ static int launch_chunk(rtlsim_ctx *ctx, int b, uint64_t cycle0, uint32_t nc, bo
     it = ctx->graphs.emplace(key, ge).first;
   }
   CK(cudaGraphLaunch(it->second, ctx->st));
-  ctx->launches += (uint64_t)nc * (G.part_steps.size() - 1 + (ctx->d_cov ? 1 : 0));
+  ctx->launches += (uint64_t)nc * (G.part_steps.size() - 1 + (ctx->d_cov ? 1 : 0) + (G.wports.empty() ? 0 : 1));
   if (timing) {
     CK(cudaEventRecord(tm.b, ctx->st));
     ctx->timed_pending.push_back(tm);
@@ -984,6 +1016,23 @@ extern "C" int rtlsim_coverage(rtlsim_ctx *ctx, uint32_t *bitmap, int clear) {
   return RTLSIM_OK;
 }
 
+extern "C" int rtlsim_get_mems(rtlsim_ctx *ctx, uint32_t *mems) {
+  if (!ctx || !mems) return RTLSIM_E_ARG;
+  if (ctx->failed) return arg_fail(ctx, RTLSIM_E_STATE, ctx->err);
+  if (ctx->src == SRC_NONE) return arg_fail(ctx, RTLSIM_E_STATE, "get_mems before bind");
+  Program &G = ctx->prog;
+  if (!G.MR) return RTLSIM_OK;
+  CK(cudaSetDevice(ctx->device));
+  uint32_t *tmp = nullptr;
+  CK(cudaMallocAsync((void **)&tmp, (size_t)ctx->N * G.MR * 4, ctx->st));
+  CK(launch_mem_export(ctx->d_mem, G.MR, (uint32_t)ctx->N, ctx->N_pad, tmp, ctx->st));
+  ctx->launches++;
+  CK(cudaMemcpyAsync(mems, tmp, (size_t)ctx->N * G.MR * 4, cudaMemcpyDeviceToHost, ctx->st));
+  CK(cudaFreeAsync(tmp, ctx->st));
+  CK(cudaStreamSynchronize(ctx->st));
+  return RTLSIM_OK;
+}
+
 extern "C" int rtlsim_reg_digest(rtlsim_ctx *ctx, uint64_t *digest) {
   if (!ctx || !digest) return RTLSIM_E_ARG;
   if (ctx->failed) return arg_fail(ctx, RTLSIM_E_STATE, ctx->err);
@@ -1038,6 +1087,11 @@ extern "C" int rtlsim_stats(const rtlsim_ctx *cctx, rtlsim_stats_t *st) {
   st->eval_stim_cycles = ctx->eval_stim_cycles;
   st->jit_compile_s = ctx->jit.compile_s;
   st->jit_cubin_bytes = ctx->jit.cubin_bytes;
+  st->jit_sass_instructions = ctx->jit.sass_instructions;
+  st->jit_tiles_per_cta = 0;
+  if (!ctx->jit.kern.empty() && ctx->N_pad)
+    for (uint32_t q = 0; q < ctx->jit.kern.size(); q++)
+      if (ctx->jit.kern[q]) st->jit_tiles_per_cta = std::max(st->jit_tiles_per_cta, jit_tiles_per_cta(ctx, ctx->jit, q));
   st->n_bitops = G.n_bitops; st->n_narrow = G.n_narrow; st->n_wide = G.n_wide;
   st->n_ld = G.n_ld; st->n_st = G.n_st;
   return RTLSIM_OK;

@@ -27,7 +27,7 @@ F_COVERAGE = 0x200
 
 EXPORTS = ["rtlsim_load", "rtlsim_bind", "rtlsim_bind_device", "rtlsim_bind_stream", "rtlsim_run",
            "rtlsim_run_device", "rtlsim_run_stream", "rtlsim_sync", "rtlsim_get_regs", "rtlsim_set_regs",
-           "rtlsim_reset", "rtlsim_coverage", "rtlsim_reg_digest", "rtlsim_stats", "rtlsim_launch_count", "rtlsim_last_error", "rtlsim_free"]
+           "rtlsim_reset", "rtlsim_coverage", "rtlsim_reg_digest", "rtlsim_get_mems", "rtlsim_stats", "rtlsim_launch_count", "rtlsim_last_error", "rtlsim_free"]
 
 
 class RtlsimError(RuntimeError):
@@ -51,7 +51,9 @@ class IRStruct(ctypes.Structure):
                 ("n_consts", ctypes.c_uint32), ("const_sig", _P), ("const_words", _P),
                 ("n_inputs", ctypes.c_uint32), ("input_sig", _P),
                 ("n_outputs", ctypes.c_uint32), ("output_sig", _P),
-                ("n_partitions", ctypes.c_uint32)]
+                ("n_partitions", ctypes.c_uint32),
+                ("n_mems", ctypes.c_uint32), ("mem_width", _P), ("mem_depth", _P), ("mem_init", _P),
+                ("n_wports", ctypes.c_uint32), ("mem_wport", _P)]
 
 
 class Options(ctypes.Structure):
@@ -74,7 +76,9 @@ class Stats(ctypes.Structure):
                 ("jit_compile_s", ctypes.c_double), ("jit_cubin_bytes", ctypes.c_uint64),
                 ("n_bitops", ctypes.c_uint64), ("n_narrow", ctypes.c_uint64), ("n_wide", ctypes.c_uint64),
                 ("n_ld", ctypes.c_uint64), ("n_st", ctypes.c_uint64), ("b_spill", ctypes.c_double),
-                ("n_live_ops", ctypes.c_uint64), ("live_word_ops", ctypes.c_uint64)]
+                ("n_live_ops", ctypes.c_uint64), ("live_word_ops", ctypes.c_uint64),
+                ("jit_sass_instructions", ctypes.c_uint64), ("jit_tiles_per_cta", ctypes.c_uint32),
+                ("pad0", ctypes.c_uint32)]
 
 
 PRODUCER = ctypes.CFUNCTYPE(ctypes.c_int, ctypes.c_void_p, ctypes.c_uint64, ctypes.c_uint64,
@@ -107,6 +111,7 @@ def lib():
         L.rtlsim_reset.argtypes = [_P]
         L.rtlsim_coverage.argtypes = [_P, _P, c_int]
         L.rtlsim_reg_digest.argtypes = [_P, _P]
+        L.rtlsim_get_mems.argtypes = [_P, _P]
         L.rtlsim_stats.argtypes = [_P, ctypes.POINTER(Stats)]
         L.rtlsim_launch_count.argtypes = [_P]
         L.rtlsim_launch_count.restype = u64
@@ -152,6 +157,12 @@ def make_ir_struct(ir):
     s.n_outputs = ir.output_sig.size
     s.output_sig = _ptr(ir.output_sig)
     s.n_partitions = int(ir.n_partitions)
+    n_mems = int(getattr(ir, "n_mems", 0))
+    if n_mems or getattr(ir, "mem_wport", np.zeros((0, 4))).size:
+        s.n_mems = n_mems
+        s.mem_width, s.mem_depth, s.mem_init = _ptr(ir.mem_width), _ptr(ir.mem_depth), _ptr(ir.mem_init)
+        s.n_wports = int(ir.mem_wport.shape[0])
+        s.mem_wport = _ptr(ir.mem_wport)
     return s
 
 
@@ -206,6 +217,10 @@ def rtlsim_reset(ctx):
 
 def rtlsim_coverage(ctx, bitmap, clear=False):
     _check(lib().rtlsim_coverage(ctx, _ptr(bitmap), 1 if clear else 0), ctx)
+
+
+def rtlsim_get_mems(ctx, mems):
+    _check(lib().rtlsim_get_mems(ctx, _ptr(mems)), ctx)
 
 
 def rtlsim_reg_digest(ctx, digest):
@@ -327,6 +342,11 @@ class Simulator:
         b = np.zeros(self.RW, np.uint32)
         rtlsim_coverage(self.ctx, b, clear)
         return b
+
+    def get_mems(self) -> np.ndarray:
+        m = np.zeros((self.N, int(getattr(self.ir, "MW", 0))), np.uint32)
+        rtlsim_get_mems(self.ctx, m)
+        return m
 
     def reg_digest(self) -> np.ndarray:
         d = np.zeros(self.N, np.uint64)

@@ -22,6 +22,8 @@ class Builder:
         self.names: dict[int, str] = {}
         self.part = 0
         self.n_partitions = 1
+        self.mems: list[tuple[int, int, list[int]]] = []   # (width, depth, init values)
+        self.wports: list[tuple[int, int, int, int]] = []  # (mem, addr, data, en)
 
     # ---------------------------------------------------------- signals --
     def _sig(self, w: int, kind: int, name: str | None) -> int:
@@ -81,6 +83,22 @@ class Builder:
     def slice(self, a: int, lo: int, w: int) -> int:
         return self.op("SLICE", w, a, imm=lo)
 
+    # --------------------------------------------------------- memories --
+    def mem(self, width: int, depth: int, init=None) -> int:
+        """A memory of `depth` entries of `width` bits (ARRSEL target)."""
+        init = [0] * depth if init is None else [int(v) for v in init]
+        assert len(init) == depth
+        self.mems.append((int(width), int(depth), init))
+        return len(self.mems) - 1
+
+    def memrd(self, m: int, addr: int, out_name: str | None = None) -> int:
+        """Combinational read of entry `addr` of memory m (MEMRD)."""
+        return self.op("MEMRD", self.mems[m][0], addr, imm=m, out_name=out_name)
+
+    def wport(self, m: int, addr: int, data: int, en: int) -> None:
+        """Synchronous write port: at the clock edge, if en: mem[addr] := data."""
+        self.wports.append((m, addr, data, en))
+
     # ------------------------------------------------------------ build --
     def build(self) -> I.IR:
         for q, d, _ in self.regs:
@@ -104,4 +122,9 @@ class Builder:
             const_words=np.asarray(const_words, dtype=np.uint32),
             input_sig=self.inputs, output_sig=self.outputs,
             n_partitions=self.n_partitions, name=self.name,
-            meta={"names": dict(self.names)})
+            meta={"names": dict(self.names)},
+            mem_width=np.asarray([m[0] for m in self.mems], dtype=np.uint16),
+            mem_depth=np.asarray([m[1] for m in self.mems], dtype=np.uint32),
+            mem_init=np.asarray([w for m in self.mems for v in m[2] for w in I.int_to_words(v, m[0])],
+                                dtype=np.uint32),
+            mem_wport=np.asarray(self.wports, dtype=np.uint32).reshape(-1, 4))

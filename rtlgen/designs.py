@@ -151,7 +151,7 @@ def random_dag(seed: int, n_ops: int = 100, input_widths=(3, 5, 1, 4, 3),
         q = b.reg(w, init)
         regs.append(q)
         pool.append(q)
-    names = list(I.OPCODES)
+    names = list(I.VALUE_OPS)
     order = list(range(n_partitions))
     rng.shuffle(order)
     comb = []
@@ -230,3 +230,115 @@ def exhaustive_stimulus(ir: I.IR) -> np.ndarray:
             cols.append(np.zeros(n, dtype=np.uint32))
         sh += w
     return np.stack(cols, axis=1).reshape(n, 1, -1)
+
+
+# ------------------------------------------------------------- memories --
+# ARRSEL (§3.1.1, Fig 5): an array variable read at a run-time index,
+# written by synchronous ports (reading 12).
+MEMSEQ_INIT = [100 + i for i in range(8)]
+
+
+def mem_seq_dut() -> I.IR:
+    """Free-running 8-bit counter c; 8 x 8-bit memory; each cycle writes
+    c + 1 at entry c mod 8 and reads entry (c - 1) mod 8 (rd_prev) and entry
+    c mod 8 (rd_same, read-during-write). Closed forms (oracle pins):
+    rd_prev_c = c for c >= 1 (107 at c = 0); rd_same_c = c - 7 for c >= 8
+    (100 + c before): a read sees the memory as it was before the edge."""
+    b = Builder("memseq")
+    c = b.reg(8, 0, "c")
+    one = b.const(8, 1)
+    c1 = b.ADD(8, c, one)
+    b.set_d(c, c1)
+    m = b.mem(8, 8, MEMSEQ_INIT)
+    wa = b.slice(c, 0, 3)
+    cm1 = b.SUB(8, c, one)
+    ra = b.slice(cm1, 0, 3)
+    en = b.const(1, 1)
+    b.wport(m, wa, c1, en)
+    b.output(c)
+    b.output(b.memrd(m, ra, "rd_prev"))
+    b.output(b.memrd(m, wa, "rd_same"))
+    return b.build()
+
+
+MEMB_DEPTH = 5
+MEMB_INIT = [0x1111 * (i + 1) for i in range(MEMB_DEPTH)]
+
+
+def mem_bounds_dut() -> I.IR:
+    """Inputs we, waddr[2:0], wdata[15:0], raddr[2:0]; a 5 x 16-bit memory.
+    Entries 5..7 do not exist: writes there are ignored, reads return 0."""
+    b = Builder("membounds")
+    we = b.input(1, "we")
+    waddr = b.input(3, "waddr")
+    wdata = b.input(16, "wdata")
+    raddr = b.input(3, "raddr")
+    m = b.mem(16, MEMB_DEPTH, MEMB_INIT)
+    b.wport(m, waddr, wdata, we)
+    b.output(b.memrd(m, raddr, "rdata"))
+    return b.build()
+
+
+def mem_two_port_dut() -> I.IR:
+    """Two write ports hit the same entry every cycle (the counter's low 2
+    bits): port 0 writes c, port 1 writes ~c — the later port wins, so
+    rd_prev (entry (c - 1) mod 4) = ~(c - 1) for c >= 1."""
+    b = Builder("mem2p")
+    c = b.reg(8, 0, "c")
+    one = b.const(8, 1)
+    b.set_d(c, b.ADD(8, c, one))
+    m = b.mem(8, 4)
+    wa = b.slice(c, 0, 2)
+    en = b.const(1, 1)
+    b.wport(m, wa, c, en)
+    b.wport(m, wa, b.NOT(8, c), en)
+    ra = b.slice(b.SUB(8, c, one), 0, 2)
+    b.output(c)
+    b.output(b.memrd(m, ra, "rd_prev"))
+    return b.build()
+
+
+def regfile_dut(seed: int = 7, depth: int = 32, width: int = 32, n_read: int = 2, wide: int = 72,
+                parts: int = 1) -> I.IR:
+    """A register-file-heavy design: a depth x width memory with n_read read
+    ports and one write port driven from inputs, a depth/4 x `wide`-bit
+    memory (three-word entries) and a 16 x 1-bit memory, each read value
+    mixed through a little logic into registers and outputs; addresses are one
+    bit wider than needed (out-of-range reads and writes occur)."""
+    rng = np.random.default_rng(seed)
+    b = Builder("regfile")
+    aw = int(np.ceil(np.log2(depth))) + 1
+    we = b.input(1, "we")
+    waddr = b.input(aw, "waddr")
+    wdata = b.input(width, "wdata")
+    raddrs = [b.input(aw, f"raddr{i}") for i in range(n_read)]
+    m = b.mem(width, depth, [int(x) for x in rng.integers(0, 1 << min(width, 62), size=depth)])
+    b.wport(m, waddr, wdata, we)
+    acc = b.reg(width, 0, "acc")
+    vals = []
+    for i, ra in enumerate(raddrs):
+        if parts > 1:
+            b.partition(i % parts)
+        v = b.memrd(m, ra)
+        vals.append(v)
+        b.output(v)
+    s = b.ADD(width, vals[0], vals[-1])
+    b.set_d(acc, b.XOR(width, acc, s))
+    b.output(acc)
+    # a wide memory (entries of 3 words) written with {wdata, wdata, waddr}
+    dw = max(4, depth // 4)
+    mw = b.mem(wide, dw, [int(x) for x in rng.integers(0, 1 << 62, size=dw)])
+    aw2 = int(np.ceil(np.log2(dw))) + 1
+    wa2 = b.slice(waddr, 0, min(aw, aw2))
+    cat = b.CONCAT(wide, b.CONCAT(2 * width, wdata, wdata), waddr)
+    b.wport(mw, wa2, cat, we)
+    b.output(b.memrd(mw, b.slice(raddrs[0], 0, min(aw, aw2))))
+    # a 1-bit memory
+    m1 = b.mem(1, 16, [int(x) for x in rng.integers(0, 2, size=16)])
+    b.wport(m1, b.slice(waddr, 0, 4), b.slice(wdata, 0, 1), we)
+    r1 = b.memrd(m1, b.slice(raddrs[-1], 0, 4))
+    f = b.reg(1, 0, "f")
+    b.set_d(f, b.XOR(1, f, r1))
+    b.output(r1)
+    b.output(f)
+    return b.build()

@@ -49,12 +49,15 @@ OPCODES = {
     "REDAND": 28,
     "REDOR": 29,
     "REDXOR": 30,
+    "MEMRD": 31,  # dst := MEM[imm][a] (0 when a >= depth): ARRSEL read (reading 12)
 }
 OPNAMES = {v: k for k, v in OPCODES.items()}
+MEM_OPS = {"MEMRD"}                       # reads a memory: not a function of its operands alone
+VALUE_OPS = [k for k in OPCODES if k not in MEM_OPS]
 N_OPCODES = len(OPCODES)
 globals().update({"OP_" + k: v for k, v in OPCODES.items()})
 
-UNARY = {"COPY", "SEXT", "NOT", "NEG", "REDAND", "REDOR", "REDXOR", "SLICE"}
+UNARY = {"COPY", "SEXT", "NOT", "NEG", "REDAND", "REDOR", "REDXOR", "SLICE", "MEMRD"}
 TERNARY = {"MUX"}
 COMPARES = {"EQ", "NE", "LTU", "LEU", "GTU", "GEU", "LTS", "LES", "GTS", "GES"}
 REDUCTIONS = {"REDAND", "REDOR", "REDXOR"}
@@ -104,13 +107,24 @@ class IR:
     n_partitions: int = 1
     name: str = "design"
     meta: dict = dataclasses.field(default_factory=dict)
+    # memories (ARRSEL, §3.1.1 Fig 5; reading 12): memory m
+    # has mem_depth[m] entries of mem_width[m] bits; mem_init holds every
+    # entry's words (memory-major, entry-major); write port p is
+    # mem_wport[p] = (mem, addr signal, data signal, enable signal)
+    mem_width: np.ndarray = dataclasses.field(default_factory=lambda: np.zeros(0, np.uint16))
+    mem_depth: np.ndarray = dataclasses.field(default_factory=lambda: np.zeros(0, np.uint32))
+    mem_init: np.ndarray = dataclasses.field(default_factory=lambda: np.zeros(0, np.uint32))
+    mem_wport: np.ndarray = dataclasses.field(default_factory=lambda: np.zeros((0, 4), np.uint32))
 
     def __post_init__(self):
         self.width = np.ascontiguousarray(self.width, dtype=np.uint16)
         self.kind = np.ascontiguousarray(self.kind, dtype=np.uint8)
         self.ops = np.ascontiguousarray(self.ops, dtype=OP_DTYPE)
-        for f in ("reg_q", "reg_d", "reg_init", "const_sig", "const_words", "input_sig", "output_sig"):
+        for f in ("reg_q", "reg_d", "reg_init", "const_sig", "const_words", "input_sig", "output_sig",
+                  "mem_depth", "mem_init"):
             setattr(self, f, np.ascontiguousarray(getattr(self, f), dtype=np.uint32))
+        self.mem_width = np.ascontiguousarray(self.mem_width, dtype=np.uint16)
+        self.mem_wport = np.ascontiguousarray(self.mem_wport, dtype=np.uint32).reshape(-1, 4)
 
     # ------------------------------------------------------------ sizes --
     @property
@@ -142,6 +156,17 @@ class IR:
     def RW(self) -> int:
         return self._words(self.reg_q)
 
+    @property
+    def n_mems(self) -> int:
+        return int(self.mem_width.shape[0])
+
+    @property
+    def MW(self) -> int:
+        """words of all memories of one stimulus"""
+        if not self.n_mems:
+            return 0
+        return int((nwords(self.mem_width.astype(np.int64)) * self.mem_depth.astype(np.int64)).sum())
+
     def input_word_masks(self) -> np.ndarray:
         """u32 mask per stimulus word (bits >= width are ignored, reading 15)."""
         out = []
@@ -159,7 +184,9 @@ class IR:
             reg_q=self.reg_q, reg_d=self.reg_d, reg_init=self.reg_init,
             const_sig=self.const_sig, const_words=self.const_words,
             input_sig=self.input_sig, output_sig=self.output_sig,
-            n_partitions=np.asarray(self.n_partitions), name=np.asarray(self.name))
+            n_partitions=np.asarray(self.n_partitions), name=np.asarray(self.name),
+            mem_width=self.mem_width, mem_depth=self.mem_depth, mem_init=self.mem_init,
+            mem_wport=self.mem_wport)
 
     @classmethod
     def load(cls, path: str) -> "IR":
@@ -168,7 +195,8 @@ class IR:
                    reg_q=z["reg_q"], reg_d=z["reg_d"], reg_init=z["reg_init"],
                    const_sig=z["const_sig"], const_words=z["const_words"],
                    input_sig=z["input_sig"], output_sig=z["output_sig"],
-                   n_partitions=int(z["n_partitions"]), name=str(z["name"]))
+                   n_partitions=int(z["n_partitions"]), name=str(z["name"]),
+                   **{k: z[k] for k in ("mem_width", "mem_depth", "mem_init", "mem_wport") if k in z})
 
     def summary(self) -> dict:
         ops = self.ops

@@ -237,3 +237,27 @@ def test_jit_dead_store_elimination_compiles(R, tmp_path, monkeypatch):
         counts[dse] = (txt.count("st.shared"), txt.count("ld.shared"))
     assert counts["1"][0] < counts["0"][0]
     assert counts["1"][1] == counts["0"][1]
+
+
+def test_memory_validation_host_only(R):
+    """Memories (reading 12) through the C ABI on the host: accepted with the
+    JIT backend, E_UNSUPPORTED without it; a MEMRD of a missing memory and an
+    address wider than 32 bits are rejected."""
+    ir = designs.regfile_dut()
+    sim = R.Simulator(ir, flags=R.F_HOST_ONLY | R.F_JIT)
+    assert sim.stats()["n_live_ops"] > 0
+    with pytest.raises(R.RtlsimError) as ei:
+        R.Simulator(ir, flags=R.F_HOST_ONLY)
+    assert ei.value.code == -4
+    bad = designs.mem_seq_dut()
+    bad.ops["imm"][bad.ops["opcode"] == I.OPCODES["MEMRD"]] = 3
+    with pytest.raises(R.RtlsimError) as ei:
+        R.Simulator(bad, flags=R.F_HOST_ONLY | R.F_JIT)
+    assert ei.value.code == -2
+    b = Builder("wideaddr")
+    a = b.input(40)
+    m = b.mem(8, 4)
+    b.output(b.memrd(m, a))
+    with pytest.raises(R.RtlsimError) as ei:
+        R.Simulator(b.build(), flags=R.F_HOST_ONLY | R.F_JIT)
+    assert ei.value.code == -4

@@ -16,7 +16,7 @@ import pytest
 from rtlgen import ir as I
 from oracle import ops_ref
 
-ALL = list(I.OPCODES)
+ALL = list(I.VALUE_OPS)   # MEMRD reads a memory: tests/test_oracle_mem.py
 
 
 def ev(oracle_lib, name, wd, a=0, wa=0, b=0, wb=0, c=0, wc=0, imm=0):

@@ -37,7 +37,7 @@ def test_shaped_designs_valid_and_seeded(oracle_lib, cid, scale):
     s = a.summary()
     assert s["n_ops"] >= int(shaped.SHAPES[cid].n_ops * scale) * 0.95
     # every opcode of the mix appears
-    assert len(s["opcode_hist"]) == len(I.OPCODES)
+    assert len(s["opcode_hist"]) == len(I.VALUE_OPS)
 
 
 def test_opcode_numbering_mirrored():
