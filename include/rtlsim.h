@@ -145,10 +145,11 @@ typedef struct {
 #define RTLSIM_F_STREAM 0x80u     /* ablation (Table 4): the per-(cycle,
                                      partition) launches of graph mode issued
                                      one by one into the stream, no graph     */
-#define RTLSIM_F_V4 0x40u         /* run-based micro-op evaluator (lower.cpp +
-                                     rtl_eval_v4) instead of the per-descriptor
-                                     interpreter; measured slower on configs
-                                     3-4 (run-dispatch overhead), kept for A/B */
+#define RTLSIM_F_V4 0x40u         /* reserved: the round-1 run-based micro-op
+                                     evaluator, removed in round 2 (slower than
+                                     the JIT and the descriptor interpreter on
+                                     every config); rtlsim_load returns
+                                     RTLSIM_E_UNSUPPORTED                     */
 #define RTLSIM_F_COVERAGE 0x200u  /* toggle coverage (N5): after every cycle,
                                      bit j of register word k is set when it
                                      differs between R_c and R_{c+1} in any

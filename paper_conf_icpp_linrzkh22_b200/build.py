@@ -14,7 +14,7 @@ HERE = os.path.dirname(os.path.abspath(__file__))
 ROOT = os.path.dirname(HERE)
 CSRC = os.path.join(HERE, "csrc")
 LIB = os.path.join(HERE, "librtlsim.so")
-SOURCES = ["compile.cpp", "lower.cpp", "kernels.cu", "runtime.cu", "jit.cpp"]
+SOURCES = ["compile.cpp", "kernels.cu", "runtime.cu", "jit.cpp"]
 HEADERS = ["program.h", "kernels.h", "device_ops.cuh", "jit_rt.cu", "jit.h"]
 JIT_RT_PTX = os.path.join(HERE, "jit_rt.ptx")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]

@@ -394,6 +394,13 @@ int compile_program(const rtlsim_ir *ir, uint32_t op_lanes, uint32_t smem_limit_
         if (--indeg[s] == 0) q.push(s);
     }
     if (porder.size() != NP) return fail(err, RTLSIM_E_IR, "partition DAG has a cycle");
+    // the DAG in execution-order indices (a concurrent per-cycle graph waits
+    // only for these)
+    std::vector<uint32_t> eidx(NP);
+    for (uint32_t i = 0; i < NP; i++) eidx[porder[i]] = i;
+    G.part_dep.assign(NP, {});
+    for (uint32_t p = 0; p < NP; p++)
+      for (uint32_t s2 : succ[p]) G.part_dep[eidx[s2]].push_back(eidx[p]);
   }
   const uint32_t P_last = porder.back();
 
@@ -493,6 +500,7 @@ int compile_program(const rtlsim_ir *ir, uint32_t op_lanes, uint32_t smem_limit_
       smem_limit_words > stage_words ? smem_limit_words - stage_words : (smem_limit_words ? 1u : 0xFFFFFFFFu);
 
   std::vector<int32_t> vid_of(n, -1);   // per partition: signal -> value id (reset per partition)
+  int32_t last_spiller = -1;
   for (uint32_t p : porder) {
     const std::vector<uint32_t> &ops_p = part_ops[p];
     std::vector<Value> vals;
@@ -1091,6 +1099,15 @@ int compile_program(const rtlsim_ir *ir, uint32_t op_lanes, uint32_t smem_limit_
       break;
     }
     for (int c = 0; c < 4; c++) max_spill_rows[c] = std::max(max_spill_rows[c], spill_rows[c]);
+    {
+      // partitions share the spill rows: the ones that spill run one after
+      // the other even in a concurrent graph
+      const uint32_t ei = (uint32_t)G.part_steps.size() - 1;
+      if (spill_rows[0] | spill_rows[1] | spill_rows[2] | spill_rows[3]) {
+        if (last_spiller >= 0) G.part_dep[ei].push_back((uint32_t)last_spiller);
+        last_spiller = (int32_t)ei;
+      }
+    }
     for (auto &st : steps) all_steps.push_back(std::move(st));
     G.part_steps.push_back((uint32_t)all_steps.size());
     for (uint32_t s : touched) vid_of[s] = -1;

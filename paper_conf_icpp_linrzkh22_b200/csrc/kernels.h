@@ -48,17 +48,11 @@ struct EvalParams {
   uint32_t *out;              // [n_cycles][OW][N_pad]
   const uint32_t *consts;
   unsigned long long *digest; // [n_cycles][N_pad] (XOR-accumulated) or NULL
-  // run-based evaluator (rtl_eval_v4, program.h U_* classes)
-  const uint4 *ustream;       // runs: header {class, count} + payload
-  const uint32_t *uptr;       // [n_steps * L + 1]
-  uint32_t zero_off;          // word offset of the zero row in shared memory
 };
 
 // N1: op-stream evaluator. grid = N_pad/32 tiles, block = 32*L threads.
 cudaError_t launch_eval(const EvalParams &p, uint32_t smem_bytes, cudaStream_t st);
 cudaError_t eval_set_smem(uint32_t smem_bytes);
-// N1 v4: run-based evaluator over the lowered micro-op stream (same grid).
-cudaError_t launch_eval_v4(const EvalParams &p, uint32_t smem_bytes, cudaStream_t st);
 
 // N2: stimulus chunk [N][nc][IW] (row pitch src_pitch words) -> per-cycle
 // class-formatted input rows (map[k]: class and row of input word k), masked

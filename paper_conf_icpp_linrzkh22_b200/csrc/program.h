@@ -109,65 +109,6 @@ struct WideRec {
 };
 static_assert(sizeof(WideRec) == 48, "wide record layout");
 
-// ------------------------------------------------------------------ uops --
-// The run-based evaluator (kernels.cu rtl_eval_v4) executes, per step and
-// op-lane warp, a list of RUNS: a header uint4 {class, count, 0, 0} followed
-// by `count` 16-byte micro-ops of that class. lower.cpp builds them from the
-// descriptor schedule: narrow ops whose operand layouts match become
-// class-specialized micro-ops (no per-op decode), wide ops are lowered into
-// 32-bit word micro-ops (bitwise / MUX / funnel-shift words, carry and
-// compare loops), register / xnet / input loads and stores are batched
-// several rows per warp instruction (lane = row part). Anything else stays a
-// generic descriptor (class U_GEN, the Desc format above). Slot fields are
-// BYTE offsets of the stimulus-lane-0 element (slot word * 4); a missing
-// operand word reads the zero row at Program::zero_off.
-enum : uint32_t {
-  // compute, lane = stimulus; E = element bytes of the U8 / U16 / U32 layout
-  U_GEN = 0,        // payload: Desc (generic decode path)
-  U_BIN = 1,        // + 3*op_idx(AND,OR,XOR,ADD,SUB,MUL) * 3 + e_idx  : {d, a, b, mask}
-  U_BINI = 19,      // + same: b is the immediate in .z                 : {d, a, imm, mask}
-  U_UN = 37,        // + 3*k(COPY,NOT,NEG,SHR,SEXT) + e_idx             : {d, a, param, mask}
-  U_MUX = 52,       // + e_idx: sel BIT                                 : {d | ms << 24, sel, t, e}
-  U_CMP = 55,       // + 3*k(EQ,NE,LTU,LEU,GTU,GEU) + e_idx -> BIT       : {d, a, b, 0}
-  U_CATBB = 73,     // + e_idx: {a(1), b(1)} -> E                       : {d, a, b, 0}
-  U_FUN = 76,       // word: (fshr(lo, hi, sh) | z) & (~0 >> ms)         : {d | ms << 24, lo, hi, z | sh << 24}
-  U_CONST = 77,     // word: d <- value (every lane)                    : {d, value, 0, 0}
-  U_WADD = 78,      // wide add / sub loop                              : {d, a, b, nd | na<<6 | nb<<12 | sub<<18 | ms<<24}
-  U_WCMP = 79,      // wide unsigned compare loop -> BIT                 : {d, a, b, n | na<<6 | nb<<12 | cc<<18}
-  // row loads (global -> smem, cp.async) / stores (smem -> global), lane = row part
-  U_LD = 80,        // + 4*arena(REG, X, IN) + cls                      : {slot, row, 0, 0}
-  U_ST = 92,        // + 4*arena(NXT, X) + cls                          : {slot, row, aux, 0}
-  U_CONSTB = 100,   // broadcast word: smem[d] <- value                  : {d, value, 0, 0}
-  U_MIX = 101,      // + opcode: narrow op, operand layouts decoded per micro-op (Desc)
-  // narrow ops with any operand / result layouts (generic-layout fetch, no
-  // per-op decode of the opcode): {d | la<<18 | lb<<21 | lc<<24 | ms<<27, a, b, c|param | ld<<24}
-  U_GXLA = 132,     // + AND OR XOR ADD SUB
-  U_GXUN = 137,     // + COPY NOT SLICE (param = shift)
-  U_GXCAT = 140,    // CONCAT (param = wb)
-  U_GXMUX = 141,
-  U_GXCMP = 142,    // + EQ NE LTU LEU GTU GEU -> 0 / 1
-  U_NCLASS = 148
-};
-// Run header {group, count, p0, p1}: the evaluator has one handler per group
-// (small code: the whole hot loop must stay in the instruction cache); the
-// run-uniform parameters p0 / p1 select the op inside the group.
-enum : uint32_t {
-  G_GEN = 0, G_MIX = 1,      // p0 = opcode
-  G_LOG = 2,                 // + e_idx: (a & b & p0) | ((a ^ b) & p1)   (AND / OR / XOR)
-  G_ARI = 5,                 // + e_idx: a + (b ^ p0) + p1               (ADD / SUB)
-  G_UN = 8,                  // + e_idx: ((a >> z) ^ p0) & mask          (COPY / NOT / SLICE)
-  G_MUX = 11,                // + e_idx
-  G_CMP = 14,                // + e_idx: p0 = EQ NE LTU LEU GTU GEU
-  G_FUN = 17, G_CONST = 18, G_CONSTB = 19, G_WADD = 20, G_WCMP = 21,
-  G_LD = 22,                 // p0 = class, p1 = arena (REG, X, IN)
-  G_ST = 23,                 // p0 = class, p1 = arena (NXT, X)
-  G_GXLA = 24,               // p0 = AND OR XOR ADD SUB
-  G_GXUN = 25,               // p0 = inversion mask (NOT)
-  G_GXCAT = 26, G_GXMUX = 27,
-  G_GXCMP = 28,              // p0 = cc
-  G_NGROUP = 29
-};
-
 struct RegInfo {
   uint32_t sig, width, cls, row, word;   // row in its class arena; word = first RW index
 };
@@ -198,12 +139,8 @@ struct Program {
   std::vector<uint32_t> step_wait;      // [n_steps] cp.async groups allowed pending at the step end
   std::vector<WideRec> wide;            // records referenced by CODE_WIDE
   std::vector<uint32_t> part_steps;     // exec-order partition boundaries in steps (size P+1)
+  std::vector<std::vector<uint32_t>> part_dep;   // exec-order partitions each one waits for in a cycle
   uint32_t smem_words = 0;              // shared words per tile (slots)
-  // ---- run-based micro-op stream (lower.cpp)
-  std::vector<Desc> ustream;            // runs: header + payload, per (step, lane)
-  std::vector<uint32_t> uptr;           // [n_steps * L + 1] offsets into ustream
-  uint32_t zero_off = 0;                // word offset of the 32-word zero row
-  uint64_t u_class_count[U_NCLASS] = {};
   // ---- memories (ARRSEL, reading 12; JIT backend only)
   std::vector<uint16_t> mem_width;
   std::vector<uint32_t> mem_depth, mem_row0;  // first u32 row of each memory in the memory arena
@@ -221,13 +158,6 @@ struct Program {
   double b_floor = 0, b_state = 0, b_part = 0, b_spill = 0;
   uint64_t n_live_ops = 0, live_word_ops = 0;
 };
-
-// Lower the descriptor schedule of a compiled Program into the run-based
-// micro-op stream (ustream / uptr / zero_off); grows smem_words by the zero row.
-void lower_program(Program &G);
-// micro-op classes executed in groups of kUnroll (runs padded by lower_program)
-constexpr uint32_t kUnroll = 4;
-bool unrolled(uint32_t cls);
 
 // Returns RTLSIM_OK or a negative status with *err set.
 int compile_program(const rtlsim_ir *ir, uint32_t op_lanes, uint32_t smem_limit_words, Program *out,

@@ -69,8 +69,7 @@ struct rtlsim_ctx {
   std::vector<void *> bind_allocs;    // freed at re-bind
   std::vector<void *> host_allocs;    // pinned, freed at re-bind
   // static device data
-  uint4 *d_desc = nullptr, *d_bitdesc = nullptr, *d_ustream = nullptr;
-  uint32_t *d_uptr = nullptr;
+  uint4 *d_desc = nullptr, *d_bitdesc = nullptr;
   uint32_t *d_bitptr = nullptr, *d_stepwait = nullptr;
   WideRec *d_wide = nullptr;
   uint32_t *d_step = nullptr, *d_consts = nullptr, *d_mask = nullptr, *d_reginit = nullptr;
@@ -113,6 +112,10 @@ struct rtlsim_ctx {
   JitKernels jit_dig;    // RTLSIM_F_JIT check-mode variant, built on the first digest run
   std::string jit_rt_path;
   uint32_t jit_smem = 0, jit_smem_cap = 0;
+  // concurrent per-cycle graph: fork / join streams and per-partition events
+  std::vector<cudaStream_t> dag_streams;
+  std::vector<cudaEvent_t> dag_events;
+  cudaEvent_t dag_fork = nullptr;
 };
 
 #define CK(call)                                                                       \
@@ -169,7 +172,7 @@ static void free_binding(rtlsim_ctx *ctx) {
 }
 
 
-constexpr uint32_t kJitMaxLanes = 4;
+constexpr uint32_t kJitMaxLanes = 8;   // JIT op-lanes by default (16 when few tiles fit a CTA, see load)
 constexpr uint64_t kMaxStimuli = 65535ull * 32ull;   // per context: transposes' grid.y bound
 
 // descriptor staging buffers start after the slots, 16-byte aligned
@@ -232,7 +235,15 @@ extern "C" int rtlsim_load(const rtlsim_ir *ir, const rtlsim_options *opt, rtlsi
     delete ctx;
     return RTLSIM_E_UNSUPPORTED;
   }
-  const bool legacy = (ctx->opt.flags & RTLSIM_F_V4) == 0;
+  if (ctx->opt.flags & RTLSIM_F_V4) {
+    // the round-1 run-based micro-op evaluator was removed (slower than the
+    // JIT kernels and the descriptor interpreter on every config)
+    g_load_error = "RTLSIM_F_V4: the run-based evaluator was removed";
+    delete ctx;
+    return RTLSIM_E_UNSUPPORTED;
+  }
+  const bool legacy = true;   // the descriptor interpreter: staging buffers per op-lane
+  uint32_t budget_words = smem_limit / 4u;
   if ((ctx->opt.flags & RTLSIM_F_JIT) && !ctx->opt.smem_limit &&
       (ctx->prog.smem_words + 64u) * 4u > smem_limit / 2u) {
     // JIT kernels are instruction-fetch bound: two tiles per CTA (the warps
@@ -242,13 +253,32 @@ extern "C" int rtlsim_load(const rtlsim_ir *ir, const rtlsim_options *opt, rtlsi
     // spill to HBM rows)
     rtlsim::Program half;
     std::string e2;
-    if (compile_program(ir, ctx->prog.L, (smem_limit / 2u - 1024u) / 4u, &half, &e2, dce, fold) == RTLSIM_OK)
+    if (compile_program(ir, ctx->prog.L, (smem_limit / 2u - 1024u) / 4u, &half, &e2, dce, fold) == RTLSIM_OK) {
       ctx->prog = std::move(half);
+      budget_words = (smem_limit / 2u - 1024u) / 4u;
+    }
   }
-  // bytes after lowering: slots, the 32-word zero row (lower_program) and,
-  // for the interpreter, one 512-byte descriptor staging buffer per op-lane
+  if ((ctx->opt.flags & RTLSIM_F_JIT) && !ctx->opt.op_lanes && ctx->prog.L == kJitMaxLanes) {
+    // Occupancy: as many warps per SM as a 1024-thread CTA holds. K tiles fit
+    // the shared memory; more op-lanes per tile fill the CTA when K is small
+    // (measured round 2, profiles/r02_sweep_*.log: config 4 (K = 2) 4 / 8 /
+    // 16 op-lanes 145 / 79 / 75 ms per cycle; config 3 (K = 4) 8 op-lanes
+    // 1.22 ms vs 16 x 2 tiles 2.19 ms)
+    const uint32_t K = std::max<uint32_t>(
+        1u, std::min<uint32_t>(jit_default_tiles(), smem_limit / std::max<uint32_t>(jit_tile_bytes(ctx->prog), 1u)));
+    const uint32_t want = std::min<uint32_t>(16u, 32u / K);
+    if (want > ctx->prog.L) {
+      rtlsim::Program wide;
+      std::string e2;
+      if (compile_program(ir, want, budget_words, &wide, &e2, dce, fold) == RTLSIM_OK &&
+          wide.smem_words <= ctx->prog.smem_words)
+        ctx->prog = std::move(wide);
+    }
+  }
+  // bytes: slots and, for the interpreter, one 512-byte descriptor staging
+  // buffer per op-lane
   auto final_bytes = [&](const Program &P) {
-    uint32_t w = ((P.smem_words + 3u) & ~3u) + 32u;
+    uint32_t w = (P.smem_words + 3u) & ~3u;
     return (legacy ? ((w + 3u) & ~3u) * 4u + P.L * 512u : w * 4u);
   };
   if (final_bytes(ctx->prog) > smem_limit) {
@@ -268,9 +298,7 @@ extern "C" int rtlsim_load(const rtlsim_ir *ir, const rtlsim_options *opt, rtlsi
     }
   }
   Program &G = ctx->prog;
-  lower_program(G);   // run-based micro-op stream (+ the zero row)
-  // legacy interpreter: slots + one 512-byte descriptor staging buffer per
-  // op-lane warp; v4: slots (micro-ops are read from L1 / L2)
+  // interpreter: slots + one 512-byte descriptor staging buffer per op-lane warp
   ctx->smem_bytes = legacy ? desc_smem_off(G) * 4u + G.L * 512u : G.smem_words * 4u;
   if (ctx->smem_bytes > smem_limit) {
     g_load_error = "per-tile working set of " + std::to_string(ctx->smem_bytes) +
@@ -329,12 +357,6 @@ extern "C" int rtlsim_load(const rtlsim_ir *ir, const rtlsim_options *opt, rtlsi
   padded.resize(G.desc.size() + 32, Desc{});   // chunk prefetch reads up to 32 past any start
   if (e == cudaSuccess) e = up((void **)&ctx->d_desc, padded.data(), padded.size() * sizeof(Desc));
   if (e == cudaSuccess) e = up((void **)&ctx->d_bitdesc, G.bitdesc.data(), G.bitdesc.size() * sizeof(BitDesc));
-  {
-    std::vector<Desc> us(G.ustream);
-    us.resize(G.ustream.size() + 64, Desc{});   // L1 prefetch lines past the end
-    if (e == cudaSuccess) e = up((void **)&ctx->d_ustream, us.data(), us.size() * sizeof(Desc));
-  }
-  if (e == cudaSuccess) e = up((void **)&ctx->d_uptr, G.uptr.data(), G.uptr.size() * 4);
   if (e == cudaSuccess) e = up((void **)&ctx->d_bitptr, G.bit_ptr.data(), G.bit_ptr.size() * 4);
   if (e == cudaSuccess) e = up((void **)&ctx->d_stepwait, G.step_wait.data(), G.step_wait.size() * 4);
   if (e == cudaSuccess) e = up((void **)&ctx->d_wide, G.wide.data(), G.wide.size() * sizeof(WideRec));
@@ -538,9 +560,6 @@ static EvalParams eval_params(rtlsim_ctx *ctx, int b, uint64_t cycle0, uint32_t 
   p.out = ctx->d_out[b];
   p.consts = ctx->d_consts;
   p.digest = digest ? ctx->d_dig[b] : nullptr;
-  p.ustream = ctx->d_ustream;
-  p.uptr = ctx->d_uptr;
-  p.zero_off = G.zero_off;
   return p;
 }
 
@@ -584,7 +603,6 @@ static uint32_t jit_tiles_per_cta(rtlsim_ctx *ctx, const JitKernels &JK, uint32_
 }
 
 static cudaError_t evaluator(rtlsim_ctx *ctx, const EvalParams &p, cudaStream_t st) {
-  if (ctx->opt.flags & RTLSIM_F_V4) return launch_eval_v4(p, ctx->smem_bytes, st);
   return launch_eval(p, ctx->smem_bytes, st);
 }
 
@@ -643,13 +661,49 @@ static int launch_chunk(rtlsim_ctx *ctx, int b, uint64_t cycle0, uint32_t nc, bo
     if (jr != RTLSIM_OK) return jr;
   }
   const JitKernels &JK = digest ? ctx->jit_dig : ctx->jit;
-  // Tc x P per-(cycle, partition) kernel nodes (graph / JIT / stream modes)
+  // Tc x P per-(cycle, partition) kernel nodes (graph / JIT / stream modes).
+  // Captured graphs (RTLSIM_DAG, default on) get the partition DAG's edges
+  // instead of a chain: within a cycle a partition waits only for the
+  // partitions whose nets it reads (and spilling partitions for each other),
+  // so independent partitions overlap (partitioning "maximizes
+  // the kernel concurrency of the induced CUDA graph"); every cycle still
+  // starts after the whole previous cycle (registers and nets are reused).
+  const bool dag_env = !getenv("RTLSIM_DAG") || atoi(getenv("RTLSIM_DAG")) != 0;
   auto issue = [&](cudaStream_t cap) -> cudaError_t {
     const uint32_t NP = (uint32_t)G.part_steps.size() - 1;
+    const bool dag = dag_env && cap != ctx->st && NP > 1;
+    if (dag && ctx->dag_streams.empty()) {
+      for (int i = 0; i < 8; i++) {
+        cudaStream_t x;
+        cudaError_t e = cudaStreamCreateWithFlags(&x, cudaStreamNonBlocking);
+        if (e != cudaSuccess) return e;
+        ctx->dag_streams.push_back(x);
+      }
+      cudaError_t e = cudaEventCreateWithFlags(&ctx->dag_fork, cudaEventDisableTiming);
+      if (e != cudaSuccess) return e;
+    }
+    while (dag && ctx->dag_events.size() < NP) {
+      cudaEvent_t x;
+      cudaError_t e = cudaEventCreateWithFlags(&x, cudaEventDisableTiming);
+      if (e != cudaSuccess) return e;
+      ctx->dag_events.push_back(x);
+    }
     for (uint32_t c = 0; c < nc; c++) {
+      if (dag) {
+        cudaError_t e = cudaEventRecord(ctx->dag_fork, cap);
+        if (e != cudaSuccess) return e;
+      }
+      std::vector<char> issued(NP, 0);
       for (uint32_t q = 0; q < NP; q++) {
         if (G.part_steps[q] == G.part_steps[q + 1]) continue;
         cudaError_t e;
+        cudaStream_t sq = cap;
+        if (dag) {
+          sq = ctx->dag_streams[q % ctx->dag_streams.size()];
+          if ((e = cudaStreamWaitEvent(sq, ctx->dag_fork, 0)) != cudaSuccess) return e;
+          for (uint32_t p : G.part_dep[q])
+            if (issued[p] && (e = cudaStreamWaitEvent(sq, ctx->dag_events[p], 0)) != cudaSuccess) return e;
+        }
         if (jit) {
           if (!JK.kern[q]) continue;
           const uint32_t par = (uint32_t)(((cycle0 & 1ull) + c) & 1ull);
@@ -674,7 +728,7 @@ static int launch_chunk(rtlsim_ctx *ctx, int b, uint64_t cycle0, uint32_t nc, bo
           jp.tpc = jit_tiles_per_cta(ctx, JK, q);
           void *args[] = {&jp};
           e = cudaLaunchKernel((const void *)JK.kern[q], dim3(ctx->N_pad / 32u / jp.tpc),
-                               dim3(32u * G.L * jp.tpc), args, jit_tile_smem(ctx, JK, q) * jp.tpc, cap);
+                               dim3(32u * G.L * jp.tpc), args, jit_tile_smem(ctx, JK, q) * jp.tpc, sq);
         } else {
           EvalParams p = eval_params(ctx, b, (cycle0 & 1ull) + c, 1, digest);
           p.step_begin = G.part_steps[q];
@@ -685,10 +739,20 @@ static int launch_chunk(rtlsim_ctx *ctx, int b, uint64_t cycle0, uint32_t nc, bo
           p.in.u32 = ctx->d_in[b].u32 + (size_t)c * ctx->in_stride.s[CLS_U32];
           p.out = ctx->d_out[b] + (size_t)c * G.OW * ctx->N_pad;
           if (digest) p.digest = ctx->d_dig[b] + (size_t)c * ctx->N_pad;
-          e = evaluator(ctx, p, cap);
+          e = evaluator(ctx, p, sq);
         }
         if (e != cudaSuccess) return e;
+        if (dag) {
+          if ((e = cudaEventRecord(ctx->dag_events[q], sq)) != cudaSuccess) return e;
+          issued[q] = 1;
+        }
       }
+      if (dag)   // join: the cycle's sinks (memory ports, coverage) and the next cycle follow every partition
+        for (uint32_t q = 0; q < NP; q++)
+          if (issued[q]) {
+            cudaError_t e = cudaStreamWaitEvent(cap, ctx->dag_events[q], 0);
+            if (e != cudaSuccess) return e;
+          }
       if (!G.wports.empty()) {   // memory write ports at the clock edge, after every partition
         cudaError_t e = launch_mem_commit(ctx->d_mem, ctx->d_port, ctx->d_ports, (uint32_t)G.wports.size(),
                                           (uint32_t)ctx->N, ctx->N_pad, cap);
@@ -1113,6 +1177,9 @@ extern "C" void rtlsim_free(rtlsim_ctx *ctx) {
     free_binding(ctx);
     jit_free(&ctx->jit);
     jit_free(&ctx->jit_dig);
+    for (cudaStream_t x : ctx->dag_streams) cudaStreamDestroy(x);
+    for (cudaEvent_t x : ctx->dag_events) cudaEventDestroy(x);
+    if (ctx->dag_fork) cudaEventDestroy(ctx->dag_fork);
     for (auto &t : ctx->timed_pending) {
       cudaEventDestroy(t.a);
       cudaEventDestroy(t.b);

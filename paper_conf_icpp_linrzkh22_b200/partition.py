@@ -85,12 +85,22 @@ def partition_order(ir) -> list[int]:
 
 @dataclasses.dataclass
 class Optimizer:
-    """Algorithm 1's optimizer: weights over T, proposal = merged task graph."""
+    """Algorithm 1's optimizer: weights over T, proposal = a task graph.
+
+    split=False: tasks merge consecutive IR partitions (topological order).
+    split=True: tasks are contiguous chunks of the global op sequence (IR
+    partitions in topological order, each partition's ops in topological
+    order), cut where the running weight_sum crosses multiples of
+    total / n_tasks — a cut may fall inside an IR partition, so n_tasks above
+    the IR's partition count splits partitions: smaller per-task working sets
+    (more tiles per CTA on the B200) for more cross-task nets (HBM bytes).
+    Contiguous chunks of a topological order keep the task graph acyclic."""
     ir: object
     n_tasks: int
     k: int = 30
     step: float = 1.0
     seed: int = 0
+    split: bool = False
 
     def __post_init__(self):
         self.T = top_types(self.ir, self.k)
@@ -123,10 +133,32 @@ class Optimizer:
     def weight_sum(self, w: np.ndarray) -> np.ndarray:
         return self.count @ w + self.other
 
-    # line 8: merge consecutive partitions (topological order) into tasks
+    # Eq 1 per op (weights of the op's node type; 1 outside T)
+    def op_weights(self, w: np.ndarray) -> np.ndarray:
+        idx = {int(t): j for j, t in enumerate(self.T)}
+        col = np.array([idx.get(int(t), -1) for t in self.types])
+        return np.where(col >= 0, w[np.maximum(col, 0)], 1.0)
+
+    def op_sequence(self) -> np.ndarray:
+        """Op indices: IR partitions in topological order, ops in IR order
+        (the IR lists ops topologically) within each."""
+        parts = self.ir.ops["part"].astype(np.int64)
+        return np.concatenate([np.nonzero(parts == p)[0] for p in self.order]).astype(np.int64)
+
+    # line 8: the partitioner the weights parameterise
     def propose(self, w: np.ndarray | None = None) -> np.ndarray:
-        """Returns the new partition id of every IR partition."""
+        """split=False: the new partition id of every IR partition;
+        split=True: the task id of every op."""
         w = self.candidate if w is None else w
+        if self.split:
+            seq = self.op_sequence()
+            ow = self.op_weights(w)[seq]
+            cum = np.cumsum(ow) - ow          # weight before each op
+            cap = ow.sum() / max(1, self.n_tasks)
+            t = np.minimum((cum / cap).astype(np.int64), self.n_tasks - 1)
+            task = np.zeros(self.ir.n_ops, np.int64)
+            task[seq] = t
+            return task
         ws = self.weight_sum(w)
         cap = ws.sum() / max(1, self.n_tasks)
         task = np.zeros(len(ws), np.int64)
@@ -145,10 +177,17 @@ class Optimizer:
 
 
 def apply(ir, task: np.ndarray):
-    """The IR with every op moved to its merged task (same semantics)."""
+    """The IR with every op moved to its task (same semantics): `task` maps
+    IR partitions (merge proposals) or ops (split proposals) to tasks."""
     ops = ir.ops.copy()
-    ops["part"] = task[ops["part"].astype(np.int64)].astype(ops["part"].dtype)
-    return dataclasses.replace(ir, ops=ops, n_partitions=int(task.max()) + 1)
+    if len(task) == ir.n_ops and len(task) != int(ir.n_partitions):
+        t = np.asarray(task, np.int64)
+    else:
+        t = task[ops["part"].astype(np.int64)]
+    # renumber the used tasks densely, in order
+    used, t = np.unique(t, return_inverse=True)
+    ops["part"] = t.astype(ops["part"].dtype)
+    return dataclasses.replace(ir, ops=ops, n_partitions=int(len(used)))
 
 
 def accept_rate(cost: float, cur_cost: float, beta: float) -> float:
@@ -159,11 +198,11 @@ def accept_rate(cost: float, cur_cost: float, beta: float) -> float:
 
 
 def mcmc_partition(ir, estimate_cost: Callable[[object], float], n_tasks: int, max_iter: int = 150,
-                   max_unimproved: int = 30, beta: float = 1.0, seed: int = 0, log=None):
+                   max_unimproved: int = 30, beta: float = 1.0, seed: int = 0, log=None, split: bool = False):
     """Algorithm 1. estimate_cost(ir_candidate) -> cost (e.g. ms).
     Returns (best_ir, best_cost, history); history rows are
     (iter, cost, accepted, cur_cost), row 0 being the all-ones weights."""
-    opt = Optimizer(ir, n_tasks=n_tasks, seed=seed)   # lines 3-5
+    opt = Optimizer(ir, n_tasks=n_tasks, seed=seed, split=split)   # lines 3-5
     rng = random.Random(seed ^ 0x5A5A)
     # reference point (not part of Algorithm 1): the initial, all-ones weights
     cand = apply(ir, opt.propose(opt.weights))

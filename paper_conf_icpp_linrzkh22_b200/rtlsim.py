@@ -22,6 +22,7 @@ RTLSIM_OK = 0
 STATUS = {0: "OK", -1: "E_ARG", -2: "E_IR", -3: "E_COMB_LOOP", -4: "E_UNSUPPORTED", -5: "E_NOMEM",
           -6: "E_CUDA", -7: "E_STATE", -8: "E_RANGE"}
 F_DIGEST, F_NO_PIPELINE, F_GRAPH, F_HOST_ONLY, F_TIMING, F_JIT, F_V4, F_STREAM = 0x1, 0x2, 0x4, 0x8, 0x10, 0x20, 0x40, 0x80
+# F_V4 is reserved (the removed run-based evaluator): loading with it fails with E_UNSUPPORTED
 F_NO_DCE = 0x100
 F_COVERAGE = 0x200
 

@@ -150,7 +150,8 @@ def test_modes_agree(R, oracle_lib):
     st = stim.stimulus(ir, 21, np.arange(70), 0, 33)
     want = oracle_lib.simulate(ir, st, digest=True, threads=8)
     for opt in (dict(flags=R.F_GRAPH, chunk_cycles=8), dict(flags=R.F_NO_PIPELINE), dict(op_lanes=1),
-                dict(flags=R.F_STREAM, chunk_cycles=6), dict(flags=R.F_V4, chunk_cycles=9), dict(flags=R.F_V4 | R.F_GRAPH, chunk_cycles=4),
+                dict(flags=R.F_STREAM, chunk_cycles=6), dict(flags=R.F_JIT | R.F_STREAM, chunk_cycles=9),
+                dict(flags=R.F_JIT | R.F_COVERAGE, chunk_cycles=4), dict(flags=R.F_GRAPH | R.F_COVERAGE, chunk_cycles=7),
                 dict(op_lanes=7, chunk_cycles=5), dict(flags=R.F_GRAPH | R.F_NO_PIPELINE, chunk_cycles=33),
                 dict(flags=R.F_NO_DCE), dict(flags=R.F_NO_DCE | R.F_JIT, chunk_cycles=11)):
         assert_same(gpu_run(R, ir, st, **opt), want, str(opt))
@@ -243,13 +244,36 @@ def test_jit_tiles_per_cta(R, oracle_lib, tpc, monkeypatch):
                 oracle_lib.simulate(ir, st, digest=True, threads=8), f"jit tpc{tpc}")
 
 
-@pytest.mark.parametrize("cid,scale,N,T", [(2, 1.0, 256, 30), (3, 0.25, 160, 16), (4, 0.02, 96, 8)])
-def test_v4_shaped_reduced(R, oracle_lib, cid, scale, N, T):
-    """The run-based micro-op evaluator (RTLSIM_F_V4) on the shaped designs."""
-    ir = shaped.generate(cid, scale=scale)
-    st = stim.stimulus(ir, stim.STIM_SEED_BASE + cid, np.arange(N), 0, T)
-    assert_same(gpu_run(R, ir, st, chunk_cycles=16, flags=R.F_V4),
-                oracle_lib.simulate(ir, st, digest=True, threads=16), f"v4 config{cid}@{scale}")
+def test_v4_removed(R):
+    """RTLSIM_F_V4 (the round-1 run-based evaluator) is gone: E_UNSUPPORTED."""
+    with pytest.raises(R.RtlsimError) as ei:
+        R.Simulator(designs.tiny_dut(), flags=R.F_V4)
+    assert ei.value.code == -4
+
+
+@pytest.mark.parametrize("dag", ["0", "1"])
+def test_jit_dag_graph(R, oracle_lib, dag, monkeypatch):
+    """The per-cycle graph with the partition DAG's edges (RTLSIM_DAG=1,
+    concurrent partitions) and as a chain (0) give the oracle's results; the
+    design spills (a small shared-memory budget), so spilling partitions must
+    also be ordered."""
+    monkeypatch.setenv("RTLSIM_DAG", dag)
+    ir = shaped.generate(3, scale=0.25)
+    st = stim.stimulus(ir, 0xDA6, np.arange(200), 0, 12)
+    want = oracle_lib.simulate(ir, st, digest=True, threads=8)
+    assert_same(gpu_run(R, ir, st, chunk_cycles=6, flags=R.F_JIT), want, f"dag={dag}")
+    assert_same(gpu_run(R, ir, st, chunk_cycles=5, flags=R.F_JIT, smem_limit=12 * 1024), want, f"dag={dag} spill")
+
+
+def test_mcmc_split_partitions(R, oracle_lib):
+    """A split proposal (tasks cut inside IR partitions) is bit-identical."""
+    from paper_conf_icpp_linrzkh22_b200 import partition as MP
+    ir = shaped.generate(3, scale=0.1)
+    opt = MP.Optimizer(ir, n_tasks=3 * ir.n_partitions, split=True)
+    new = MP.apply(ir, opt.propose(opt.weights))
+    st = stim.stimulus(ir, 77, np.arange(96), 0, 10)
+    assert_same(gpu_run(R, new, st, chunk_cycles=5, flags=R.F_JIT),
+                oracle_lib.simulate(ir, st, digest=True, threads=8), "split tasks")
 
 
 def test_mcmc_merged_partitions(R, oracle_lib):

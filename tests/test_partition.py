@@ -88,3 +88,30 @@ def test_algorithm1_loop_with_stand_in_estimator():
     assert it_costs[0][2]
     # unimproved counter: the loop ends either at max_iter or after 8 non-improving iterations
     assert len(it_costs) == 40 or sum(1 for h in it_costs[-8:] if h[1] >= h[3] or not h[2]) >= 1
+
+
+def test_split_proposal_chunks_the_op_sequence():
+    """split=True: tasks are contiguous chunks of the partitions' topological
+    op sequence, so n_tasks above the IR's partition count splits partitions
+    and the task DAG stays acyclic; the compiler accepts it, the oracle's
+    results do not change (partitions only change the schedule)."""
+    import oracle
+    from rtlgen import stim
+    ir = shaped.generate(3, scale=0.1)
+    opt = MP.Optimizer(ir, n_tasks=3 * ir.n_partitions, split=True)
+    task = opt.propose(opt.weights)
+    seq = opt.op_sequence()
+    assert sorted(seq.tolist()) == list(range(ir.n_ops))
+    assert np.all(np.diff(task[seq]) >= 0)                       # contiguous, in order
+    new = MP.apply(ir, task)
+    assert new.n_partitions > ir.n_partitions                    # partitions were split
+    MP.partition_order(new)                                        # acyclic
+    # raising a weight moves the cuts
+    w = opt.weights.copy()
+    w[0] += 5
+    assert not np.array_equal(opt.propose(w), task)
+    from paper_conf_icpp_linrzkh22_b200 import rtlsim as R
+    assert R.Simulator(new, flags=R.F_HOST_ONLY | R.F_JIT).stats()["n_partitions"] == new.n_partitions
+    st = stim.stimulus(ir, 5, np.arange(8), 0, 6)
+    a, b = oracle.simulate(ir, st, digest=True), oracle.simulate(new, st, digest=True)
+    assert np.array_equal(a["digest"], b["digest"])

@@ -69,7 +69,6 @@ def host_run(flags, reps=2):
 
 variants = [
     ("fused interpreter (default)", "device", 0),
-    ("fused run-based v4 evaluator", "device", R.F_V4),
     ("graph: per-(cycle,partition) interpreter nodes", "device", R.F_GRAPH),
     ("stream: per-(cycle,partition) interpreter launches", "device", R.F_STREAM),
     ("jit (graph-launched)", "device", R.F_JIT),

@@ -19,7 +19,7 @@ for cid in cfgs:
     T = Tc * 4
     t0 = time.time()
     import os
-    jit = (R.F_JIT if os.environ.get('JIT') else 0) | (R.F_V4 if os.environ.get('V4') else 0)
+    jit = (R.F_JIT if os.environ.get('JIT') else 0)
     sim = R.Simulator(ir, chunk_cycles=Tc, flags=R.F_TIMING | jit, op_lanes=int(os.environ.get('LANES', '0')), smem_limit=int(os.environ.get('SMEM_KB','0'))*1024, stream=torch.cuda.current_stream().cuda_stream)
     tl = time.time() - t0
     st = sim.stats()

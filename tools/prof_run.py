@@ -11,7 +11,7 @@ ir = designs.tiny_dut() if cid == 1 else shaped.generate(cid)
 import os
 N = int(os.environ.get('PROF_N', NS[cid]))
 s = torch.cuda.Stream(); torch.cuda.set_stream(s)
-flags = (R.F_JIT if os.environ.get('JIT') else 0) | (R.F_V4 if os.environ.get('V4') else 0)
+flags = (R.F_JIT if os.environ.get('JIT') else 0)
 sim = R.Simulator(ir, chunk_cycles=Tc, stream=s.cuda_stream, flags=flags, op_lanes=int(os.environ.get('LANES', '0')), smem_limit=int(os.environ.get('SMEM_KB','0'))*1024)
 d_stim = stim.stimulus_torch(ir, stim.STIM_SEED_BASE + cid, 0, N, 0, Tc * nl)
 out = torch.empty((N, Tc, ir.OW), dtype=torch.int32, device='cuda')
