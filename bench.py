@@ -371,6 +371,12 @@ def run_ours(a):
                 "stimuli_total": n_total, "stimuli_per_gpu": N, "cycles_per_step": Tc,
                 "n_ops": st["n_ops"], "n_live_ops": st["n_live_ops"], "word_ops": st["word_ops"],
                 "live_word_ops": st["live_word_ops"],
+                "op_lanes": st["op_lanes"], "tiles_per_cta": st["jit_tiles_per_cta"],
+                "warps_per_cta": st["op_lanes"] * max(1, st["jit_tiles_per_cta"]),
+                "sass_instructions": st["jit_sass_instructions"],
+                "warp_instructions_per_live_op": (st["jit_sass_instructions"] / max(1, st["n_live_ops"])
+                                                  if st["jit_sass_instructions"] else None),
+                "warps_sharing_each_fetched_instruction": st["jit_tiles_per_cta"] or None,
                 "design_seed": hex(stim.DESIGN_SEED_BASE + cid), "stim_seed": hex(seed),
                 "parallelism": f"contiguous stimulus shards x{world} (parallel.run_sharded)",
                 "schedule": "jit per-(cycle, partition) kernels, graph-launched" if a.backend == "jit"

@@ -48,11 +48,29 @@ std::string fmt(const char *f, ...) {
 }
 
 // context values passed from the kernel to every step function
-const char *kCtx32[] = {"smb", "lane", "wl", "N", "tbar"};
+const char *kCtx32[] = {"smb", "lane", "wl", "N", "tbar", "mbar"};
 const char *kCtx64[] = {"tb_c0", "tb_c1", "tb_c2", "tb_c3", "tb_n0", "tb_n1", "tb_n2", "tb_n3",
                         "tb_x0", "tb_x1", "tb_x2", "tb_x3", "tb_i0", "tb_i1", "tb_i2", "tb_i3",
                         "outb", "dig", "wide", "smg", "bitl", "memb", "portb"};
-constexpr int kN32 = 5, kN64 = 23;
+constexpr int kN32 = 6, kN64 = 23;
+
+// Split-phase step barrier (RTLSIM_JIT_SPLIT=1; default off, see below):
+// instead of bar.sync at every step end, a warp arrives on an mbarrier (two,
+// alternating by step parity) and, before waiting for the other warps, runs
+// the next step's ops that cannot depend on them — operands written by this
+// warp, or by other warps two or more steps earlier (not by a cp.async of
+// another warp), destinations whose slot no other warp touched in the
+// previous step. Measured cause (profiles/r02_ncu_c4_l16k2.txt): 54 % of the
+// warp stall samples of a config-4 kernel at 16 op-lanes were the barrier.
+// Off by default: ptxas treats code after a (non-.aligned) mbarrier.arrive as
+// possibly divergent and duplicates blocks with divergence fallbacks around
+// every vote.sync — config 3 SASS 195K -> 408K with the arrive alone — and
+// only 18 % of the ops qualify as early (loads are late, 23 % read a value of
+// the previous step, 17 % a value another warp loaded).
+int jit_split() {
+  const char *e = getenv("RTLSIM_JIT_SPLIT");
+  return e ? atoi(e) : 0;
+}
 
 // Step barrier (RTLSIM_JIT_TBAR, read per build): 0 = one CTA-wide barrier
 // per step (all K tiles x L op-lanes); 1 = a named barrier per tile (id
@@ -72,6 +90,7 @@ inline uint64_t skey(uint64_t sp, uint32_t off) { return (sp << 32) | off; }
 // Writes of one step function, by (step, warp), per slot key (dry pass).
 struct WriteLog {
   std::unordered_map<uint64_t, std::vector<std::pair<int32_t, uint32_t>>> w;
+  std::unordered_map<uint64_t, std::vector<std::pair<int32_t, uint32_t>>> wo;   // of which opaque (cp.async / generic)
   // steps of the shared-memory reads of `key` (any warp), recorded by the
   // probe pass for dead slot-store elimination
   std::unordered_map<uint64_t, std::vector<int32_t>> rd;
@@ -273,7 +292,10 @@ void sts(Em &e, uint64_t sp, uint32_t off, const std::string &r) {
 // a write this warp cannot forward (cp.async, generic path)
 void opaque_write(Em &e, uint64_t sp, uint32_t off) {
   const uint64_t k = skey(sp, off);
-  if (e.dry) e.log->w[k].push_back({e.step, e.warp});
+  if (e.dry) {
+    e.log->w[k].push_back({e.step, e.warp});
+    e.log->wo[k].push_back({e.step, e.warp});
+  }
   else e.fwd.erase(k);
   const int64_t id = inst_of(e, sp, off);
   if (id >= 0 && e.probe) (*e.inst)[(size_t)id].need = true;
@@ -1246,6 +1268,58 @@ std::string func_proto(const std::string &name) {
 // (bar.sync 0, counted per CTA, not per PC) inside every warp's stream — so
 // a warp's instruction fetch is sequential across steps instead of jumping
 // over the other warps' code at every step.
+// ---------------------------------------------- split-phase step barrier --
+// slot row keys of a value (layout lay at slot offset off, width w)
+void value_keys(uint32_t lay, uint32_t off, uint32_t w, std::vector<uint64_t> &out) {
+  if (lay == LC_IMM || w == 0) return;
+  if (lay == LC_U32) {
+    for (uint32_t i = 0; i < nwords(w); i++) out.push_back(skey(SP_W, off + 32 * i));
+  } else if (lay == LC_BCAST) {
+    for (uint32_t i = 0; i < nwords(w); i++) out.push_back(skey(SP_S, off + i));
+  } else {
+    out.push_back(skey(layout_space(lay), off));
+  }
+}
+// operand and destination slot keys of a descriptor (every operand, whether
+// or not the emitter forwards it); *ld: a cp.async load
+void desc_keys(const Program &G, const Desc &q, std::vector<uint64_t> &src, std::vector<uint64_t> &dst, bool *ld) {
+  const uint32_t code = q.x & 0xFFu;
+  *ld = false;
+  if (code < 32u) {
+    const uint32_t la = (q.x >> 8) & 7u, lb = (q.x >> 11) & 7u, lc = (q.x >> 14) & 7u, ldl = (q.x >> 17) & 7u;
+    value_keys(la, q.y >> 16, 32, src);
+    if ((q.w >> 11) & 1u) value_keys(lb, q.z & 0xFFFFu, 32, src);
+    if ((q.w >> 12) & 1u) value_keys(lc, q.z >> 16, 32, src);
+    value_keys(ldl, q.y & 0xFFFFu, 32, dst);
+  } else if (code == CODE_WIDE) {
+    const WideRec &r = G.wide[q.y];
+    value_keys(r.lays & 0xFFu, r.a, r.wa, src);
+    value_keys((r.lays >> 8) & 0xFFu, r.b, r.wb, src);
+    value_keys((r.lays >> 16) & 0xFFu, r.c, r.wc, src);
+    value_keys(r.wd <= 32 ? value_layout(r.wd, false) : LC_U32, r.d, r.wd, dst);
+  } else if (code == CODE_LD_REG || code == CODE_LD_X || code == CODE_LD_IN) {
+    *ld = true;
+    const uint32_t cls = (q.x >> 8) & 3u, nw = (q.x >> 12) & 63u;
+    value_keys(cls == CLS_U32 ? LC_U32 : cls == CLS_U16 ? LC_U16 : cls == CLS_U8 ? LC_U8 : LC_BIT, q.y,
+               cls == CLS_U32 ? 32 * nw : 1, dst);
+  } else if (code == CODE_LD_CONST) {
+    const uint32_t nw = (q.x >> 12) & 63u;
+    value_keys(((q.x >> 18) & 1u) ? LC_BCAST : LC_U32, q.y, 32 * nw, dst);
+  } else if (code == CODE_ST_REG || code == CODE_ST_X || code == CODE_ST_OUT || code == CODE_ST_PORT) {
+    const uint32_t nw = (q.x >> 12) & 63u, lay = (q.x >> 18) & 7u;
+    value_keys(lay, q.y, lay == LC_U32 ? 32 * nw : 32, src);
+  } else if (code == CODE_ST_REGC) {
+    value_keys((q.x >> 18) & 7u, q.y, q.x >> 21, src);
+  }
+}
+void bit_keys(const BitDesc &q, std::vector<uint64_t> &src, std::vector<uint64_t> &dst) {
+  const uint32_t lut = q.x & 0xFFu, immf = q.x >> 8;
+  const uint32_t f[3] = {q.y >> 16, q.z & 0xFFFFu, q.z >> 16};
+  for (uint32_t k = 0; k < 3; k++)
+    if (!(immf & (1u << k)) && lut_uses(lut, k)) src.push_back(skey(SP_S, f[k]));
+  dst.push_back(skey(SP_S, q.y & 0xFFFFu));
+}
+
 bool jit_compact_env(const Program &G) {
   const char *e = getenv("RTLSIM_JIT_COMPACT");
   return G.L == 1 && (e ? atoi(e) != 0 : true);
@@ -1279,6 +1353,100 @@ std::string step_function(const Program &G, const std::string &name, uint32_t s0
         for (uint32_t k = G.step_ptr[s * G.L + w]; k < G.step_ptr[s * G.L + w + 1]; k++) emit_desc(d, G, G.desc[k]);
       }
   }
+  // split-phase barrier: which ops of each (warp, step) may run before the
+  // wait for the previous step's barrier (see jit_split)
+  const bool split = jit_split() != 0 && G.L > 1;
+  std::vector<std::vector<char>> early_bit, early_desc;   // [w * nsteps + (s - s0)][k]
+  if (split) {
+    const uint32_t ns = s1 - s0;
+    early_bit.assign((size_t)G.L * ns, {});
+    early_desc.assign((size_t)G.L * ns, {});
+    std::unordered_map<uint64_t, std::vector<std::pair<int32_t, uint32_t>>> uses;
+    std::vector<uint64_t> src, dst;
+    bool ld;
+    for (uint32_t w = 0; w < G.L; w++)
+      for (uint32_t st = s0; st < s1; st++) {
+        for (uint32_t k = G.bit_ptr[st] + w; k < G.bit_ptr[st + 1]; k += G.L) {
+          src.clear(); dst.clear();
+          bit_keys(G.bitdesc[k], src, dst);
+          for (uint64_t x : src) uses[x].push_back({(int32_t)st, w});
+        }
+        for (uint32_t k = G.step_ptr[st * G.L + w]; k < G.step_ptr[st * G.L + w + 1]; k++) {
+          src.clear(); dst.clear();
+          desc_keys(G, G.desc[k], src, dst, &ld);
+          for (uint64_t x : src) uses[x].push_back({(int32_t)st, w});
+        }
+      }
+    auto is_opaque = [&](uint64_t k, int32_t t, uint32_t w) {
+      auto it = log.wo.find(k);
+      if (it == log.wo.end()) return false;
+      for (auto &x : it->second)
+        if (x.first == t && x.second == w) return true;
+      return false;
+    };
+    auto ok = [&](int32_t t, uint32_t w) {
+      if (t == (int32_t)s0 || jit_split() == 2) return false;   // 2: A/B, no early ops
+      for (uint64_t k : src) {   // the value read: the latest write before step t
+        int32_t tw = -1;
+        uint32_t ww = 0;
+        auto it = log.w.find(k);
+        if (it == log.w.end()) return false;
+        for (auto &x : it->second)
+          if (x.first < t && x.first > tw) tw = x.first, ww = x.second;
+        if (tw < 0) return false;
+        if (ww == w) continue;                       // this warp's own write
+        if (tw > t - 2 || is_opaque(k, tw, ww)) return false;
+      }
+      for (uint64_t k : dst) {   // no other warp touches the slot in step t - 1
+        auto u = uses.find(k);
+        if (u != uses.end())
+          for (auto &x : u->second)
+            if (x.first == t - 1 && x.second != w) return false;
+        auto it = log.w.find(k);
+        if (it != log.w.end())
+          for (auto &x : it->second)
+            if (x.first == t - 1 && x.second != w) return false;
+      }
+      return true;
+    };
+    static const bool dbg = getenv("RTLSIM_JIT_SPLIT_DEBUG") != nullptr;
+    uint64_t n_src_recent = 0, n_src_opq = 0, n_dst = 0, n_ld = 0, n_ok = 0, n_all = 0;
+    auto why = [&](int32_t t, uint32_t w) {
+      for (uint64_t k : src) {
+        int32_t tw = -1; uint32_t ww = 0;
+        auto it = log.w.find(k);
+        if (it == log.w.end()) continue;
+        for (auto &x : it->second) if (x.first < t && x.first > tw) tw = x.first, ww = x.second;
+        if (tw >= 0 && ww != w) { if (tw > t - 2) { n_src_recent++; return; } if (is_opaque(k, tw, ww)) { n_src_opq++; return; } }
+      }
+      n_dst++;
+    };
+    for (uint32_t w = 0; w < G.L; w++)
+      for (uint32_t st = s0; st < s1; st++) {
+        auto &eb = early_bit[(size_t)w * ns + (st - s0)];
+        auto &ed = early_desc[(size_t)w * ns + (st - s0)];
+        for (uint32_t k = G.bit_ptr[st] + w; k < G.bit_ptr[st + 1]; k += G.L) {
+          src.clear(); dst.clear();
+          bit_keys(G.bitdesc[k], src, dst);
+          eb.push_back(ok((int32_t)st, w));
+        }
+        for (uint32_t k = G.step_ptr[st * G.L + w]; k < G.step_ptr[st * G.L + w + 1]; k++) {
+          src.clear(); dst.clear();
+          desc_keys(G, G.desc[k], src, dst, &ld);
+          ed.push_back(!ld && ok((int32_t)st, w));
+          if (dbg && st > s0) {
+            n_all++;
+            if (ld) n_ld++;
+            else if (ed.back()) n_ok++;
+            else why((int32_t)st, w);
+          }
+        }
+      }
+    if (dbg)
+      fprintf(stderr, "split %s: %llu descs, early %llu, loads %llu, late by recent src %llu, opaque src %llu, dst %llu\n",
+              name.c_str(), (unsigned long long)n_all, (unsigned long long)n_ok, (unsigned long long)n_ld,
+              (unsigned long long)n_src_recent, (unsigned long long)n_src_opq, (unsigned long long)n_dst);
+  }
   auto emit_real = [&](Em &e, bool probe, bool dse) {
   e.dig = dig;
   e.dry = false;
@@ -1310,6 +1478,42 @@ std::string step_function(const Program &G, const std::string &name, uint32_t s0
     e.warp = w;
     for (uint32_t s = s0; s < s1; s++) {
       e.step = (int32_t)s;
+      if (split) {
+        // early ops, the wait for the previous step's barrier, late ops
+        const auto &eb = early_bit[(size_t)w * (s1 - s0) + (s - s0)];
+        const auto &ed = early_desc[(size_t)w * (s1 - s0) + (s - s0)];
+        for (int pass = 0; pass < 2; pass++) {
+          if (pass == 1 && s > s0 && jit_split() != 3) {   // 3: code-size probe only (no wait: racy)
+            // the wait loop lives in a called function: a loop inside the
+            // straight-line code makes ptxas duplicate blocks and add
+            // divergence fallbacks around every vote (SASS x1.5 - x2)
+            const std::string ra = e.R();
+            e.l(fmt("add.u32 %s, %%mbar, %u", ra.c_str(), 8u * ((s - 1) & 1u)));
+            e.s += "\t{\n\t.param .b32 mw0;\n\t.param .b64 mw1;\n";
+            e.l(fmt("st.param.b32 [mw0], %s", ra.c_str()));
+            e.l(fmt("st.param.b64 [mw1], %%mtok%u", (s - 1) & 1u));
+            e.l("call.uni rtl_mbar_wait, (mw0, mw1)");
+            e.s += "\t}\n";
+          }
+          uint32_t j = 0;
+          for (uint32_t k = G.bit_ptr[s] + w; k < G.bit_ptr[s + 1]; k += G.L, j++) {
+            if ((eb[j] != 0) != (pass == 0)) continue;
+            const size_t from = e.s.size();
+            e.opn++;
+            emit_bit(e, G.bitdesc[k]);
+            note_kind(e, pass == 0 ? "bit:early" : "bit", from);
+          }
+          j = 0;
+          for (uint32_t k = G.step_ptr[s * G.L + w]; k < G.step_ptr[s * G.L + w + 1]; k++, j++) {
+            if ((ed[j] != 0) != (pass == 0)) continue;
+            emit_desc(e, G, G.desc[k]);
+          }
+        }
+        e.l("cp.async.commit_group");
+        e.l(fmt("cp.async.wait_group %u", G.step_wait[s]));
+        if (s + 1 < s1) e.l(fmt("mbarrier.arrive.shared::cta.b64 %%mtok%u, [%%mbar+%u]", s & 1u, 8u * (s & 1u)));
+        continue;
+      }
       {
         // this warp's bit ops of the step: groups sharing a truth table
         // (immediates folded in) of >= RTLSIM_JIT_BITBATCH ops run
@@ -1361,7 +1565,7 @@ std::string step_function(const Program &G, const std::string &name, uint32_t s0
       else if (jit_tbar() == 2)
         e.l("barrier.sync 0");
       else if (G.L > 1)
-        e.l(fmt("barrier.sync %%tbar, %u", 32u * G.L));
+        e.l(fmt("bar.sync %%tbar, %u", 32u * G.L));   // aligned: one per step in every warp of the tile
       else
         e.l("bar.warp.sync -1");
     }
@@ -1427,7 +1631,8 @@ std::string step_function(const Program &G, const std::string &name, uint32_t s0
   }
   std::string out = func_proto(name) + "\n{\n";
   out += fmt("\t.reg .b32 %%r<%u>;\n\t.reg .b64 %%rd<%u>;\n\t.reg .pred %%p<%u>;\n", e.nr + 1, e.nrd + 1, e.np + 1);
-  out += "\t.reg .b32 %smb, %lane, %wl, %N, %tbar, %rw, %rh, %rb, %N4, %N2, %Nb, %lsh;\n\t.reg .b64 %tbb1, %tbb2, %tlw, ";
+  out += "\t.reg .b64 %mtok0, %mtok1;\n";
+  out += "\t.reg .b32 %smb, %lane, %wl, %N, %tbar, %mbar, %rw, %rh, %rb, %N4, %N2, %Nb, %lsh;\n\t.reg .b64 %tbb1, %tbb2, %tlw, ";
   for (int i = 0; i < kN64; i++) out += fmt("%s%%%s", i ? ", " : "", kCtx64[i]);
   out += ";\n\t.reg .pred %pl0, %pl8, %pl16, %pdig;\n";
   for (int i = 0; i < kN32; i++) out += fmt("\tld.param.u32 %%%s, [a_%s];\n", kCtx32[i], kCtx32[i]);
@@ -1456,6 +1661,10 @@ std::string jit_partition_ptx(const Program &G, uint32_t q, const std::string &r
   mod += ".version 8.8\n.target sm_100a\n.address_size 64\n\n";
   mod += rt_ptx;
   mod += "\n.extern .shared .align 16 .b8 dyn_smem[];\n\n";
+  // wait for a phase of a split-phase step barrier (jit_split)
+  mod += ".func rtl_mbar_wait(.param .b32 mb_a, .param .b64 mb_t)\n{\n\t.reg .b32 %ra;\n\t.reg .b64 %rt;\n"
+         "\t.reg .pred %pw;\n\tld.param.b32 %ra, [mb_a];\n\tld.param.b64 %rt, [mb_t];\n$MBW:\n"
+         "\tmbarrier.try_wait.shared::cta.b64 %pw, [%ra], %rt;\n\t@!%pw bra.uni $MBW;\n\tret;\n}\n\n";
   // step groups of bounded size (ptxas time is superlinear in function size).
   // Default: one function per partition. With several called functions
   // ptxas keeps the global-memory descriptor in a uniform register only in
@@ -1492,7 +1701,7 @@ std::string jit_partition_ptx(const Program &G, uint32_t q, const std::string &r
   // lock-step and share its instruction fetch.
   mod += fmt(".visible .entry rtl_jit_part(.param .align 8 .b8 prm[%zu])\n.maxntid %u, 1, 1\n{\n",
              sizeof(JitParams), 32u * G.L * std::max<uint32_t>(tmax, 1u));
-  mod += "\t.reg .b32 %tidx, %tile, %s, %smb, %lane, %wl, %N, %wg, %tsub, %tpc, %tbar;\n\t.reg .b64 %t64, %b64, %digb;\n\t.reg .pred %pz;\n\t.reg .b64 ";
+  mod += "\t.reg .b32 %tidx, %tile, %s, %smb, %lane, %wl, %N, %wg, %tsub, %tpc, %tbar, %mbar, %nthr;\n\t.reg .b64 %t64, %b64, %digb;\n\t.reg .pred %pz;\n\t.reg .b64 ";
   for (int i = 0; i < kN64; i++) mod += fmt("%s%%%s", i ? ", " : "", kCtx64[i]);
   mod += ";\n";
   mod += fmt("\tmov.u32 %%tidx, %%tid.x;\n\tand.b32 %%lane, %%tidx, 31;\n\tshr.u32 %%wg, %%tidx, 5;\n"
@@ -1527,6 +1736,12 @@ std::string jit_partition_ptx(const Program &G, uint32_t q, const std::string &r
   mod += fmt("\tld.param.u64 %%b64, [prm+%zu];\n\tmul.wide.u32 %%t64, %%s, 4;\n\tadd.u64 %%memb, %%b64, %%t64;\n",
              offsetof(JitParams, mem));
   mod += fmt("\tld.param.u64 %%b64, [prm+%zu];\n\tadd.u64 %%portb, %%b64, %%t64;\n", offsetof(JitParams, port));
+  // the split-phase step barrier pair after the CTA's tiles (16 bytes)
+  mod += fmt("\tmov.u32 %%mbar, dyn_smem;\n\tmad.lo.u32 %%mbar, %%tpc, %u, %%mbar;\n", tbytes);
+  if (jit_split() != 0 && G.L > 1)
+    mod += "\tmov.u32 %nthr, %ntid.x;\n\t{\n\t.reg .pred %p0;\n\tsetp.eq.u32 %p0, %tidx, 0;\n"
+           "\t@%p0 mbarrier.init.shared::cta.b64 [%mbar], %nthr;\n\t@%p0 mbarrier.init.shared::cta.b64 [%mbar+8], %nthr;\n"
+           "\tbar.sync 0;\n\t}\n";
   mod += fmt("\tmov.u32 %%smb, dyn_smem;\n\tmad.lo.u32 %%smb, %%tsub, %u, %%smb;\n\tcvta.shared.u64 %%smg, dyn_smem;\n"
              "\tmul.wide.u32 %%t64, %%tsub, %u;\n\tadd.u64 %%smg, %%smg, %%t64;\n",
              tbytes, tbytes);

@@ -595,9 +595,14 @@ static uint32_t jit_tiles_per_cta(rtlsim_ctx *ctx, const JitKernels &JK, uint32_
   // the kernel set being launched (the check-mode variant may have been built
   // with another RTLSIM_JIT_TMAX than the plain one): its .maxntid bound; the
   // partition's own shared memory per tile (compacted kernels differ)
-  uint32_t m = std::min<uint32_t>(JK.tmax, (uint32_t)optin / std::max<uint32_t>(jit_tile_smem(ctx, JK, q), 1u));
+  uint32_t m = std::min<uint32_t>(JK.tmax, ((uint32_t)optin - 16u) / std::max<uint32_t>(jit_tile_smem(ctx, JK, q), 1u));
   if (const char *e = getenv("RTLSIM_JIT_TPC")) m = std::min<uint32_t>(m, (uint32_t)atoi(e));
   m = std::max<uint32_t>(m, 1u);
+  // small batches (config 2: 128 tiles): fewer tiles per CTA so that every
+  // SM gets a CTA, rather than K tiles on a quarter of the SMs
+  int sms = 148;
+  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, ctx->device);
+  while (m > 1 && tiles / m < (uint32_t)sms) m--;
   while (m > 1 && tiles % m) m--;
   return m;
 }
@@ -668,7 +673,20 @@ static int launch_chunk(rtlsim_ctx *ctx, int b, uint64_t cycle0, uint32_t nc, bo
   // so independent partitions overlap (partitioning "maximizes
   // the kernel concurrency of the induced CUDA graph"); every cycle still
   // starts after the whole previous cycle (registers and nets are reused).
-  const bool dag_env = !getenv("RTLSIM_DAG") || atoi(getenv("RTLSIM_DAG")) != 0;
+  // Default: on when a partition launch is at most 4 waves of CTAs (its tail
+  // is a large share; config 3: 1.22 -> 1.12 ms/cycle), off for long
+  // launches (config 4, 6.9 waves: 75.6 -> 84.1 ms/cycle with it, two
+  // partitions' code streams compete for instruction fetch);
+  // profiles/r02_f_probe.log
+  bool dag_env = !getenv("RTLSIM_DAG") || atoi(getenv("RTLSIM_DAG")) != 0;
+  if (!getenv("RTLSIM_DAG") && jit) {
+    uint32_t ctas = 0;
+    for (uint32_t q = 0; q + 1 < G.part_steps.size(); q++)
+      if (q < JK.kern.size() && JK.kern[q]) ctas = std::max(ctas, ctx->N_pad / 32u / jit_tiles_per_cta(ctx, JK, q));
+    int sms = 148;
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, ctx->device);
+    dag_env = ctas <= 4u * (uint32_t)sms;
+  }
   auto issue = [&](cudaStream_t cap) -> cudaError_t {
     const uint32_t NP = (uint32_t)G.part_steps.size() - 1;
     const bool dag = dag_env && cap != ctx->st && NP > 1;
@@ -728,7 +746,7 @@ static int launch_chunk(rtlsim_ctx *ctx, int b, uint64_t cycle0, uint32_t nc, bo
           jp.tpc = jit_tiles_per_cta(ctx, JK, q);
           void *args[] = {&jp};
           e = cudaLaunchKernel((const void *)JK.kern[q], dim3(ctx->N_pad / 32u / jp.tpc),
-                               dim3(32u * G.L * jp.tpc), args, jit_tile_smem(ctx, JK, q) * jp.tpc, sq);
+                               dim3(32u * G.L * jp.tpc), args, jit_tile_smem(ctx, JK, q) * jp.tpc + 16u, sq);
         } else {
           EvalParams p = eval_params(ctx, b, (cycle0 & 1ull) + c, 1, digest);
           p.step_begin = G.part_steps[q];
