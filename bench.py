@@ -393,7 +393,11 @@ def run_ours(a):
                                    else "rtl_eval_kernel",
                          "peak_source": peak_src,
                          "algorithmic_bytes_per_stim_cycle": st["b_floor"],
-                         "eval_ms_per_launch": avg_ms, "eval_share_of_step": ev_ms / max(ms, 1e-9)},
+                         # the timed unit is one graph launch: cycles_per_step x partitions kernel nodes
+                         "eval_ms_per_graph_launch": avg_ms,
+                         "kernel_nodes_per_graph_launch": Tc * st["n_partitions"] if a.backend == "jit" else None,
+                         "eval_share_of_step": ev_ms / max(ms, 1e-9),
+                         "traffic_source": "profiles/ncu_config%d.json (ncu DRAM bytes of one full cycle)" % cid},
             "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": info["launches"], "clocks": info["clocks"],
         }
         print(json.dumps(line), flush=True)

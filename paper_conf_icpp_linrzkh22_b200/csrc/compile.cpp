@@ -1210,6 +1210,17 @@ int compile_program(const rtlsim_ir *ir, uint32_t op_lanes, uint32_t smem_limit_
       lanes[best].push_back(sd.first);
       load[best] += sd.second;
     }
+    if (getenv("RTLSIM_BALANCE_DEBUG")) {
+      static double sum_max = 0, sum_avg = 0;
+      static uint64_t nst = 0;
+      uint64_t mx = 0, tot = 0;
+      for (uint32_t l = 0; l < L; l++) mx = std::max(mx, load[l]), tot += load[l];
+      sum_max += (double)mx;
+      sum_avg += (double)tot / L;
+      if (++nst % 500 == 0 || si + 1 == all_steps.size())
+        fprintf(stderr, "balance: %llu steps, sum(max lane cost) / sum(avg) = %.3f\n", (unsigned long long)nst,
+                sum_max / std::max(1.0, sum_avg));
+    }
     for (uint32_t l = 0; l < L; l++) {
       G.step_ptr.push_back((uint32_t)G.desc.size());
       // loads first (their latency overlaps the step's compute; they are
