@@ -223,9 +223,16 @@ def run_ours(a):
 
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
-    local = int(os.environ.get("LOCAL_RANK", "0"))
+    # RTLSIM_BENCH_BACKEND=gloo (tests only): several ranks on one GPU, CPU
+    # collectives — exercises the multi-rank path where only one GPU exists
+    backend = os.environ.get("RTLSIM_BENCH_BACKEND", "nccl")
+    local = int(os.environ.get("LOCAL_RANK", "0")) % max(1, torch.cuda.device_count())
     if world > 1:
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        if backend == "nccl":
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        else:
+            dist.init_process_group(backend)
+    coll_dev = "cuda" if backend == "nccl" else "cpu"
     torch.cuda.set_device(local)
 
     def staged(fn):
@@ -319,14 +326,14 @@ def run_ours(a):
             t = time.perf_counter()
             for _ in range(a.steps):
                 R.rtlsim_run(sim.ctx, Tc, h_out.numpy(), None, None)
-            el = torch.tensor([time.perf_counter() - t], dtype=torch.float64, device="cuda")
+            el = torch.tensor([time.perf_counter() - t], dtype=torch.float64, device=coll_dev)
             if world > 1:
                 dist.all_reduce(el, op=dist.ReduceOp.MAX)
             info["e2e_s"] = float(el.item())
         del sim
         return {"elapsed": ms / 1e3, "reg_digest": reg_dig, "coverage": None}
 
-    res = parallel.run_sharded(simulate, n_total, device="cuda")
+    res = parallel.run_sharded(simulate, n_total, device=coll_dev)
     st, s_before, ms, N = info["stats"], info["s_before"], info["ms"], info["N"]
     ms_max = res.elapsed_max * 1e3
     total = n_total * Tc * a.steps

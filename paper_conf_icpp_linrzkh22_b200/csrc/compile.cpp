@@ -1187,7 +1187,8 @@ int compile_program(const rtlsim_ir *ir, uint32_t op_lanes, uint32_t smem_limit_
     std::vector<uint64_t> load(L, 0);
     uint64_t step_cost = 0;
     for (auto &sd : st.lane) step_cost += sd.second;
-    const uint64_t slack = std::max<uint64_t>(8, step_cost / L / 6);
+    static const uint64_t slack_div = getenv("RTLSIM_AFFINITY_SLACK") ? std::max(1, atoi(getenv("RTLSIM_AFFINITY_SLACK"))) : 6;
+    const uint64_t slack = std::max<uint64_t>(8, step_cost / L / slack_div);
     std::vector<uint32_t> score(L);
     for (auto &sd : st.lane) {
       uint32_t best = (uint32_t)(std::min_element(load.begin(), load.end()) - load.begin());
