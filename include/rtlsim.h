@@ -237,9 +237,16 @@ int rtlsim_load(const rtlsim_ir *ir, const rtlsim_options *opt, rtlsim_ctx **out
  * whole. N is 1..2097120 (65535 tiles of 32) per context: shard larger
  * batches over contexts / GPUs (§8(e)); a larger N returns RTLSIM_E_ARG. */
 int rtlsim_bind(rtlsim_ctx *ctx, uint64_t N, uint64_t T, const uint32_t *stim);
-/* Same with a DEVICE pointer to stim[N][T][IW] (resident in HBM). */
+/* Same with a DEVICE pointer to stim[N][T][IW] (resident in HBM; the
+ * stimulus is already on the GPU, so the set_inputs stage of the P:L919-963
+ * pipeline is a device-side transpose only). Borrowed until the last run that
+ * reads it returns; E_ARG for N out of range. */
 int rtlsim_bind_device(rtlsim_ctx *ctx, uint64_t N, uint64_t T, const uint32_t *stim_dev);
-/* Same with a producer callback instead of a buffer. */
+/* Same with a producer callback instead of a buffer: the CPU set_inputs task
+ * of PAPER.md §3.2.3 (Fig 11) called per stimulus group (chunk of
+ * cycles) into pinned staging, overlapped with the GPU's evaluation of the
+ * previous chunk. prod must stay valid until the last run; a non-zero return
+ * aborts that run (see rtlsim_producer). */
 int rtlsim_bind_stream(rtlsim_ctx *ctx, uint64_t N, uint64_t T, rtlsim_producer prod, void *user);
 
 /* Simulate `cycles` cycles c0..c0+cycles-1 from the ctx's cycle cursor c0
@@ -247,15 +254,23 @@ int rtlsim_bind_stream(rtlsim_ctx *ctx, uint64_t N, uint64_t T, rtlsim_producer 
  * be NULL): out[N][cycles][OW] (outputs sampled before the clock edge,
  * reading 3), regs[N][RW] after the last cycle, digest[N][cycles]. Blocking. */
 int rtlsim_run(rtlsim_ctx *ctx, uint64_t cycles, uint32_t *out, uint32_t *regs, uint64_t *digest);
-/* Same with DEVICE output buffers (either may be NULL). Asynchronous on the
- * ctx's stream: call rtlsim_sync before reading them. */
+/* Same with DEVICE output buffers (either may be NULL): out_dev[N][cycles][OW],
+ * digest_dev[N][cycles]. Asynchronous on the ctx's stream: call rtlsim_sync
+ * before reading them. The per-cycle evaluation is the CUDA-graph schedule of
+ * P:L852-917 (one node per partition per cycle). */
 int rtlsim_run_device(rtlsim_ctx *ctx, uint64_t cycles, uint32_t *out_dev, uint64_t *digest_dev);
-/* Same with a consumer callback receiving each chunk. */
+/* Same with a consumer callback receiving each chunk (host, transposed to
+ * [N][nc][OW]; digest [N][nc] when loaded with RTLSIM_F_DIGEST): the output
+ * drain end of the P:L919-963 pipeline. Blocking; a non-zero return aborts
+ * the run (see rtlsim_consumer). */
 int rtlsim_run_stream(rtlsim_ctx *ctx, uint64_t cycles, rtlsim_consumer cons, void *user);
+/* Wait for everything queued on the ctx's streams (rtlsim_run_device). */
 int rtlsim_sync(rtlsim_ctx *ctx);
 
 /* Register state checkpoint: regs[N][RW] host (get/set), or reset to reg_init
- * and cycle 0. */
+ * (and memories to their initial contents) and cycle 0. The register state R
+ * is what Listing 1's loop carries from cycle to cycle; E_STATE
+ * before bind; set_regs does not move the cycle cursor. */
 int rtlsim_get_regs(rtlsim_ctx *ctx, uint32_t *regs);
 int rtlsim_set_regs(rtlsim_ctx *ctx, const uint32_t *regs);
 int rtlsim_reset(rtlsim_ctx *ctx);
@@ -270,7 +285,8 @@ int rtlsim_reset(rtlsim_ctx *ctx);
 int rtlsim_coverage(rtlsim_ctx *ctx, uint32_t *bitmap, int clear);
 /* Memory contents mems[N][MW] (host; MW = sum over memories of depth x
  * ceil(width/32) words, memories and entries in IR order) after the last
- * simulated cycle. E_STATE before bind. */
+ * simulated cycle: the ARRSEL array variables of PAPER.md §3.1.1 (Fig 5,
+ * P:L496-531), per stimulus. E_STATE before bind. */
 int rtlsim_get_mems(rtlsim_ctx *ctx, uint32_t *mems);
 /* Per-stimulus digest of the current register state, digest[s] (host, N
  * words) = XOR_k mix(((k + 1 + 2^31) << 32) | R[s][k]) — the register half of
@@ -279,13 +295,19 @@ int rtlsim_get_mems(rtlsim_ctx *ctx, uint32_t *mems);
  * registers themselves). P:L1128-1129: results compared per stimulus. */
 int rtlsim_reg_digest(rtlsim_ctx *ctx, uint64_t *digest);
 
+/* Compiled-design and run accounting (rtlsim_stats_t): op counts, the
+ * algorithmic bytes per stimulus-cycle of SURVEY §8(d) (b_floor), the JIT's
+ * SASS size and tiles per CTA, timing of evaluator launches (RTLSIM_F_TIMING).
+ * Works on host-only contexts. E_ARG for NULL. */
 int rtlsim_stats(const rtlsim_ctx *ctx, rtlsim_stats_t *st);
 /* Kernel launches issued by this ctx since load (for the bench's gpu_launches). */
 uint64_t rtlsim_launch_count(const rtlsim_ctx *ctx);
 /* Message for the last failing call on ctx (NULL: the thread's last
  * rtlsim_load failure). Owned by the library; valid until the next call. */
 const char *rtlsim_last_error(const rtlsim_ctx *ctx);
-void rtlsim_free(rtlsim_ctx *ctx); /* NULL-safe */
+/* Release the ctx and everything it owns (device memory, streams, graphs,
+ * JIT modules). NULL-safe; valid after a sticky failure. */
+void rtlsim_free(rtlsim_ctx *ctx);
 
 #ifdef __cplusplus
 }
