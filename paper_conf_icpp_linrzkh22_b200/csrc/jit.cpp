@@ -1745,6 +1745,12 @@ std::string jit_partition_ptx(const Program &G, uint32_t q, const std::string &r
   mod += fmt("\tmov.u32 %%smb, dyn_smem;\n\tmad.lo.u32 %%smb, %%tsub, %u, %%smb;\n\tcvta.shared.u64 %%smg, dyn_smem;\n"
              "\tmul.wide.u32 %%t64, %%tsub, %u;\n\tadd.u64 %%smg, %%smg, %%t64;\n",
              tbytes, tbytes);
+  // M1 cycle loop (nc > 1, single-partition designs only): after each cycle
+  // the state buffers swap, the input / output / digest rows advance, and a
+  // CTA barrier orders this cycle's register stores before the next cycle's
+  // loads (the tile's stimuli are its own: no other CTA is involved)
+  mod += "\t{\n\t.reg .b32 %cyc, %ncy;\n\t.reg .b64 %tsw, %stp;\n\t.reg .pred %pcy;\n";
+  mod += fmt("\tld.param.u32 %%ncy, [prm+%zu];\n\tmov.u32 %%cyc, 0;\n$CYC:\n", offsetof(JitParams, nc));
   for (size_t g = 0; g < groups.size(); g++) {
     mod += "\t{\n";
     std::string args;
@@ -1759,6 +1765,16 @@ std::string jit_partition_ptx(const Program &G, uint32_t q, const std::string &r
     }
     mod += fmt("\tcall.uni rtl_steps_%zu, (%s);\n\t}\n", g, args.c_str());
   }
+  mod += "\tadd.u32 %cyc, %cyc, 1;\n\tsetp.lt.u32 %pcy, %cyc, %ncy;\n\t@!%pcy bra.uni $CYCE;\n";
+  for (int k = 0; k < 4; k++) {
+    mod += fmt("\tmov.u64 %%tsw, %%tb_c%d;\n\tmov.u64 %%tb_c%d, %%tb_n%d;\n\tmov.u64 %%tb_n%d, %%tsw;\n", k, k, k, k);
+    mod += fmt("\tld.param.u64 %%stp, [prm+%zu];\n\tadd.u64 %%tb_i%d, %%tb_i%d, %%stp;\n",
+               offsetof(JitParams, in_step) + 8 * k, k, k);
+  }
+  mod += fmt("\tld.param.u64 %%stp, [prm+%zu];\n\tadd.u64 %%outb, %%outb, %%stp;\n", offsetof(JitParams, out_step));
+  mod += fmt("\tld.param.u64 %%stp, [prm+%zu];\n\tsetp.ne.u64 %%pcy, %%dig, 0;\n\t@%%pcy add.u64 %%dig, %%dig, %%stp;\n",
+             offsetof(JitParams, dig_step));
+  mod += "\tbar.sync 0;\n\tbra.uni $CYC;\n$CYCE:\n\t}\n";
   mod += "\tret;\n}\n";
   return mod;
 }

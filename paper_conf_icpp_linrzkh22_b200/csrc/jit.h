@@ -30,8 +30,14 @@ struct JitParams {
   uint64_t bittab;                           // this partition's bit-op batch table (uint4 per op) or 0
   uint64_t mem;                              // memory arena [MR][N_pad] u32 (MEMRD) or 0
   uint64_t port;                             // write-port arena [PW][N_pad] u32 (CODE_ST_PORT) or 0
+  // cycles simulated by this launch (M1 persistent mode: single-partition
+  // designs loop over a chunk's cycles inside the kernel; 1 otherwise) and
+  // the per-cycle advance of the input / output / digest rows
+  uint32_t nc, pad;
+  uint64_t in_step[4];                       // bytes per cycle in the input arena, per class
+  uint64_t out_step, dig_step;               // bytes per cycle of the output / digest rows
 };
-static_assert(sizeof(JitParams) == 184, "JitParams layout is read through offsetof in the PTX generator");
+static_assert(sizeof(JitParams) == 240, "JitParams layout is read through offsetof in the PTX generator");
 
 // Maximum tiles per CTA the kernels are compiled for (.maxntid 32 * L * kJitMaxTiles).
 constexpr uint32_t kJitMaxTiles = 16;

@@ -666,6 +666,11 @@ static int launch_chunk(rtlsim_ctx *ctx, int b, uint64_t cycle0, uint32_t nc, bo
     if (jr != RTLSIM_OK) return jr;
   }
   const JitKernels &JK = digest ? ctx->jit_dig : ctx->jit;
+  // M1 persistent mode: a single-partition design with no
+  // per-cycle sink kernels (memory ports, coverage) runs a whole chunk of
+  // cycles in one launch per CTA; RTLSIM_M1=0 keeps one launch per cycle
+  const bool m1 = jit && G.part_steps.size() == 2 && G.wports.empty() && !ctx->d_cov &&
+                  !(ctx->opt.flags & RTLSIM_F_STREAM) && !(getenv("RTLSIM_M1") && atoi(getenv("RTLSIM_M1")) == 0);
   // Tc x P per-(cycle, partition) kernel nodes (graph / JIT / stream modes).
   // Captured graphs (RTLSIM_DAG, default on) get the partition DAG's edges
   // instead of a chain: within a cycle a partition waits only for the
@@ -706,7 +711,7 @@ static int launch_chunk(rtlsim_ctx *ctx, int b, uint64_t cycle0, uint32_t nc, bo
       if (e != cudaSuccess) return e;
       ctx->dag_events.push_back(x);
     }
-    for (uint32_t c = 0; c < nc; c++) {
+    for (uint32_t c = 0; c < nc; c += (m1 ? nc : 1)) {
       if (dag) {
         cudaError_t e = cudaEventRecord(ctx->dag_fork, cap);
         if (e != cudaSuccess) return e;
@@ -743,6 +748,13 @@ static int launch_chunk(rtlsim_ctx *ctx, int b, uint64_t cycle0, uint32_t nc, bo
           jp.bittab = JK.d_bittab ? (uint64_t)(JK.d_bittab + 4ull * JK.bit_base[q]) : 0;
           jp.mem = (uint64_t)ctx->d_mem;
           jp.port = (uint64_t)ctx->d_port;
+          jp.nc = m1 ? nc : 1;
+          jp.in_step[0] = (uint64_t)ctx->in_stride.s[CLS_BIT] * 4;
+          jp.in_step[1] = (uint64_t)ctx->in_stride.s[CLS_U8];
+          jp.in_step[2] = (uint64_t)ctx->in_stride.s[CLS_U16] * 2;
+          jp.in_step[3] = (uint64_t)ctx->in_stride.s[CLS_U32] * 4;
+          jp.out_step = (uint64_t)G.OW * ctx->N_pad * 4;
+          jp.dig_step = (uint64_t)ctx->N_pad * 8;
           jp.tpc = jit_tiles_per_cta(ctx, JK, q);
           void *args[] = {&jp};
           e = cudaLaunchKernel((const void *)JK.kern[q], dim3(ctx->N_pad / 32u / jp.tpc),
@@ -789,7 +801,7 @@ static int launch_chunk(rtlsim_ctx *ctx, int b, uint64_t cycle0, uint32_t nc, bo
     // the paper's stream-based baseline (Table 4): the same per-(cycle,
     // partition) launches issued one by one every chunk, no graph
     CK(issue(ctx->st));
-    ctx->launches += (uint64_t)nc * (G.part_steps.size() - 1 + (ctx->d_cov ? 1 : 0) + (G.wports.empty() ? 0 : 1));
+    ctx->launches += m1 ? 1 : (uint64_t)nc * (G.part_steps.size() - 1 + (ctx->d_cov ? 1 : 0) + (G.wports.empty() ? 0 : 1));
     if (timing) {
       CK(cudaEventRecord(tm.b, ctx->st));
       ctx->timed_pending.push_back(tm);
@@ -816,7 +828,7 @@ static int launch_chunk(rtlsim_ctx *ctx, int b, uint64_t cycle0, uint32_t nc, bo
     it = ctx->graphs.emplace(key, ge).first;
   }
   CK(cudaGraphLaunch(it->second, ctx->st));
-  ctx->launches += (uint64_t)nc * (G.part_steps.size() - 1 + (ctx->d_cov ? 1 : 0) + (G.wports.empty() ? 0 : 1));
+  ctx->launches += m1 ? 1 : (uint64_t)nc * (G.part_steps.size() - 1 + (ctx->d_cov ? 1 : 0) + (G.wports.empty() ? 0 : 1));
   if (timing) {
     CK(cudaEventRecord(tm.b, ctx->st));
     ctx->timed_pending.push_back(tm);

@@ -317,3 +317,20 @@ def test_jit_rebind_new_n(R, oracle_lib, generic, monkeypatch):
         sim.bind(st)
         got = sim.run(12, out=True, regs=True, digest=N != 33)   # both kernel variants
         assert_same(got, oracle_lib.simulate(ir, st, digest=True, threads=8), f"jit rebind N={N}")
+
+
+@pytest.mark.parametrize("m1", ["1", "0"])
+def test_jit_m1_cycle_loop(R, oracle_lib, m1, monkeypatch):
+    """M1 persistent mode: a single-partition design runs each chunk of
+    cycles inside one launch per CTA (state buffers swap and input / output /
+    digest rows advance in the kernel); identical to one launch per cycle and
+    to the oracle, with ragged chunks and a ragged N."""
+    monkeypatch.setenv("RTLSIM_M1", m1)
+    ir = shaped.generate(2, scale=0.3)
+    st = stim.stimulus(ir, 0x3141, np.arange(100), 0, 29)
+    want = oracle_lib.simulate(ir, st, digest=True, threads=8)
+    got = gpu_run(R, ir, st, chunk_cycles=8, flags=R.F_JIT)
+    assert_same(got, want, f"m1={m1}")
+    chunks = -(-29 // 8)
+    if m1 == "1":
+        assert got["launches"] < chunks * 8     # one evaluator launch per chunk, not per cycle
