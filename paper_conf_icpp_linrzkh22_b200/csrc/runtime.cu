@@ -266,7 +266,9 @@ extern "C" int rtlsim_load(const rtlsim_ir *ir, const rtlsim_options *opt, rtlsi
     // 1.22 ms vs 16 x 2 tiles 2.19 ms)
     const uint32_t K = std::max<uint32_t>(
         1u, std::min<uint32_t>(jit_default_tiles(), smem_limit / std::max<uint32_t>(jit_tile_bytes(ctx->prog), 1u)));
-    const uint32_t want = std::min<uint32_t>(16u, 32u / K);
+    // (r2 sweep, profiles/r02_i_probe.log / r02_j_probe.log, config 4 at two
+    // tiles: 10 / 12 / 13 / 14 / 16 op-lanes 73.6 / 72.6 / 73.0 / 72.4 / 75.5 ms)
+    const uint32_t want = K == 1 ? 16u : K == 2 ? 14u : std::min<uint32_t>(16u, 32u / K);
     if (want > ctx->prog.L) {
       rtlsim::Program wide;
       std::string e2;

@@ -63,7 +63,10 @@ def read(cid):
     for line in open(p):
         if line.startswith("#") or not line.strip():
             continue
-        s, dh, rh = line.split()
+        parts = line.split()
+        if len(parts) != 3 or len(parts[1]) != 32:   # a line cut short by a killed run
+            continue
+        s, dh, rh = parts
         res[int(s)] = (dh, None if rh == "-" else rh)
     return res
 
@@ -97,12 +100,14 @@ def main():
         blk = np.array(todo[k:k + a.block], dtype=np.int64)
         st = stim.stimulus(ir, seed, blk, 0, T)
         r = D.simulate(st, out=False, regs=True, digest=True, threads=a.threads)
-        with open(p, "a") as f:
-            for j, s in enumerate(blk):
-                dh = hashlib.sha256(np.ascontiguousarray(r["digest"][j], "<u8").tobytes()).hexdigest()[:32]
-                rh = hashlib.sha256(np.ascontiguousarray(r["regs"][j], "<u4").tobytes()).hexdigest()[:32] \
-                    if want_regs else "-"
-                f.write(f"{int(s)} {dh} {rh}\n")
+        lines = []
+        for j, s in enumerate(blk):
+            dh = hashlib.sha256(np.ascontiguousarray(r["digest"][j], "<u8").tobytes()).hexdigest()[:32]
+            rh = hashlib.sha256(np.ascontiguousarray(r["regs"][j], "<u4").tobytes()).hexdigest()[:32] \
+                if want_regs else "-"
+            lines.append(f"{int(s)} {dh} {rh}\n")
+        with open(p, "a") as f:   # one write per block, flushed at once
+            f.write("".join(lines))
         el = time.time() - t0
         print(f"config {cid}: {k + len(blk)}/{len(todo)} stimuli, {el:.0f} s", flush=True)
 
