@@ -160,6 +160,7 @@ struct Em {
   std::unordered_map<uint64_t, uint32_t> cur;   // row key -> current instance
   std::vector<WideRec> *wrec = nullptr;     // generic-path records with compacted offsets
   std::vector<uint32_t> *bittab = nullptr;  // bit-op batch table (uint4 per op)
+  std::unordered_map<uint64_t, std::vector<std::string>> vpend;   // wide groups awaiting their vector store
   std::unordered_map<uint64_t, Fwd> fwd;
   uint32_t nr = 0, nrd = 0, np = 0, nlab = 0;
   // N_pad the code is specialised for (0: generic, row stride from %N at run
@@ -289,6 +290,100 @@ void sts(Em &e, uint64_t sp, uint32_t off, const std::string &r) {
   if (e.dry) e.log->w[k].push_back({e.step, e.warp});
   else e.fwd[k] = Em::Fwd{r, e.step, e.opn};
 }
+// ----------------------------------------------- vector layout of wide values --
+// (r2, RTLSIM_JIT_VWIDE, default on) A value of >= 2 words in a U32 slot is
+// laid out in groups of up to 4 words: group g (words 4g..4g+gs-1, gs =
+// min(4, nw - 4g)) occupies 32 lanes x gs words at byte 16 * 32 * g of the
+// slot, lane l's words contiguous — one LDS.128 / STS.128 (LDS.64 for a pair)
+// moves a lane's whole group, where the row layout needs one instruction per
+// word. Same slot size; keys stay (SP_W, off + 32 i) per word. Only the JIT
+// uses it (the interpreter keeps rows); variable wide shifts are emitted
+// inline (no generic call reading the row layout).
+bool jit_vwide() {
+  static const bool on = !getenv("RTLSIM_JIT_VWIDE") || atoi(getenv("RTLSIM_JIT_VWIDE")) != 0;
+  return on;
+}
+bool is_vwide(uint32_t lay, uint32_t w) { return jit_vwide() && lay == LC_U32 && nwords(w) >= 2; }
+const char *kLaneBase[5] = {"", "%rw", "%rq2", "%rq3", "%rq4"};
+uint32_t vgs(uint32_t nw, uint32_t g) { return std::min<uint32_t>(4u, nw - 4u * g); }
+// byte offset of word i of the wide value at slot off (from the lane base of its group size)
+uint32_t vbyte(Em &e, uint32_t off, uint32_t nw, uint32_t i) {
+  return xoff(e, SP_W, off) * 4u + 512u * (i / 4u) + 4u * (i % 4u);
+}
+// a still-valid forwarded register for key, or ""
+std::string fwd_get(Em &e, uint64_t k) {
+  if (e.dry || e.fwd_max <= 0) return "";
+  auto it = e.fwd.find(k);
+  if (it == e.fwd.end()) return "";
+  if (e.step - it->second.step <= e.fwd_max && e.opn - it->second.op <= e.fwd_ops &&
+      !e.log->other(k, e.warp, it->second.step, e.step))
+    return it->second.reg;
+  e.fwd.erase(it);
+  return "";
+}
+// word i of the wide value at slot off (nw words): forwarded, or its group loaded at once
+std::string vword(Em &e, uint32_t off, uint32_t nw, uint32_t i) {
+  const uint64_t k = skey(SP_W, off + 32u * i);
+  std::string r = fwd_get(e, k);
+  if (!r.empty()) return r;
+  const uint32_t g = i / 4u, gs = vgs(nw, g);
+  if (gs == 1 || gs == 3) {   // no vector width: only the word asked for
+    r = e.R();
+    e.l(fmt("ld.shared.u32 %s, [%s+%u]", r.c_str(), kLaneBase[gs], vbyte(e, off, nw, i)));
+    if (e.probe) e.log->rd[k].push_back(e.step);
+    inst_read(e, SP_W, off + 32u * i);
+    if (!e.dry) e.fwd[k] = Em::Fwd{r, e.step - 1, e.opn};
+    return r;
+  }
+  std::string regs[4];
+  for (uint32_t j = 0; j < gs; j++) regs[j] = e.R();
+  const uint32_t b = vbyte(e, off, nw, 4u * g);
+  if (gs == 4) {
+    e.l(fmt("ld.shared.v4.u32 {%s, %s, %s, %s}, [%%rq4+%u]", regs[0].c_str(), regs[1].c_str(), regs[2].c_str(),
+            regs[3].c_str(), b));
+  } else {
+    e.l(fmt("ld.shared.v2.u32 {%s, %s}, [%%rq2+%u]", regs[0].c_str(), regs[1].c_str(), b));
+  }
+  for (uint32_t j = 0; j < gs; j++) {
+    const uint64_t kj = skey(SP_W, off + 32u * (4u * g + j));
+    if (e.probe) e.log->rd[kj].push_back(e.step);
+    inst_read(e, SP_W, off + 32u * (4u * g + j));
+    if (!e.dry) e.fwd[kj] = Em::Fwd{regs[j], e.step - 1, e.opn};
+  }
+  return regs[i % 4u];
+}
+// word i of a wide result: buffered until its group is complete, then one
+// vector store (kept when any word of the group is read back from shared memory)
+void vstore(Em &e, uint32_t off, uint32_t nw, uint32_t i, const std::string &v) {
+  const uint32_t g = i / 4u, gs = vgs(nw, g);
+  auto &pend = e.vpend[((uint64_t)off << 8) | g];
+  if (pend.size() < gs) pend.resize(gs);
+  pend[i % 4u] = v;
+  const uint64_t k = skey(SP_W, off + 32u * i);
+  if (e.dry) e.log->w[k].push_back({e.step, e.warp});
+  else e.fwd[k] = Em::Fwd{v, e.step, e.opn};
+  for (uint32_t j = 0; j < gs; j++)
+    if (pend[j].empty()) return;
+  bool live = false;
+  for (uint32_t j = 0; j < gs; j++) {
+    const uint64_t kj = skey(SP_W, off + 32u * (4u * g + j));
+    const int64_t id = inst_of(e, SP_W, off + 32u * (4u * g + j));
+    const bool unread = id >= 0 && !e.probe && !(*e.inst)[(size_t)id].need;
+    if (!unread && !(e.dse && e.log->dead_store(kj, e.step, e.to_end))) live = true;
+  }
+  if (live) {
+    const uint32_t b = vbyte(e, off, nw, 4u * g);
+    if (gs == 4)
+      e.l(fmt("st.shared.v4.u32 [%%rq4+%u], {%s, %s, %s, %s}", b, pend[0].c_str(), pend[1].c_str(), pend[2].c_str(),
+              pend[3].c_str()));
+    else if (gs == 2)
+      e.l(fmt("st.shared.v2.u32 [%%rq2+%u], {%s, %s}", b, pend[0].c_str(), pend[1].c_str()));
+    else
+      for (uint32_t j = 0; j < gs; j++) e.l(fmt("st.shared.u32 [%s+%u], %s", kLaneBase[gs], b + 4u * j, pend[j].c_str()));
+  }
+  e.vpend.erase(((uint64_t)off << 8) | g);
+}
+
 // a write this warp cannot forward (cp.async, generic path)
 void opaque_write(Em &e, uint64_t sp, uint32_t off) {
   const uint64_t k = skey(sp, off);
@@ -384,6 +479,8 @@ std::string wword(Em &e, WOp &o, uint32_t i, bool sx) {
     if (o.w <= 32) {
       if (o.narrow.empty()) o.narrow = fetch_narrow(e, o.lay, o.off, o.w);
       r = o.narrow;
+    } else if (is_vwide(o.lay, o.w)) {
+      r = vword(e, o.off, n, j);
     } else {
       r = o.lay == LC_BCAST ? lds(e, SP_S, o.off + j) : lds(e, SP_W, o.off + 32 * j);
     }
@@ -426,7 +523,8 @@ void wstore(Em &e, uint32_t off, uint32_t wd, uint32_t i, const std::string &v) 
     e.l(fmt("and.b32 %s, %s, %u", m.c_str(), x.c_str(), mask_of(rem)));
     x = m;
   }
-  sts(e, SP_W, off + 32 * i, x);
+  if (jit_vwide()) vstore(e, off, n, i, x);
+  else sts(e, SP_W, off + 32 * i, x);
 }
 
 std::string reg_of(Em &e, const std::string &v) {
@@ -670,6 +768,166 @@ void generic_wide(Em &e, const WideRec &w, uint32_t idx) {
   }
 }
 
+// SHL / SHRL / SHRA of a wide value by a variable amount, inline (vector
+// layout): word i of the result is a funnel shift of the
+// operand's words i -/+ q and i -/+ q + 1 (q = s / 32), read at run-time
+// word indices (per lane) straight from shared memory.
+void emit_vshift(Em &e, const WideRec &w, WOp &A, WOp &B) {
+  const uint32_t op = w.op, wd = w.wd, nd = nwords(wd), wa = A.w, nwa = nwords(wa);
+  const uint32_t Ws = std::max(wd, wa);
+  const uint32_t limit = op == RTLSIM_OP_SHL ? wd : Ws;
+  const bool sra = op == RTLSIM_OP_SHRA;
+  // the shift amount, saturated to 2^32 - 1 when it does not fit 32 bits
+  std::string sam = reg_of(e, wword(e, B, 0, false));
+  if (nwords(B.w) > 1) {
+    std::string hi = e.R();
+    e.l(fmt("mov.u32 %s, 0", hi.c_str()));
+    for (uint32_t i = 1; i < nwords(B.w); i++) {
+      std::string t = e.R();
+      e.l(fmt("or.b32 %s, %s, %s", t.c_str(), hi.c_str(), reg_of(e, wword(e, B, i, false)).c_str()));
+      hi = t;
+    }
+    std::string p = e.P(), t = e.R();
+    e.l(fmt("setp.ne.u32 %s, %s, 0", p.c_str(), hi.c_str()));
+    e.l(fmt("selp.u32 %s, -1, %s, %s", t.c_str(), sam.c_str(), p.c_str()));
+    sam = t;
+  }
+  // operand kind: 0 = a narrow value (a0), 1 = broadcast constant words, 2 = vector layout
+  uint32_t kind = 0, abase = 0;
+  std::string a0 = "0", fill = "0";
+  if (wa <= 32) {
+    a0 = reg_of(e, wword(e, A, 0, sra));
+  } else if (A.lay == LC_BCAST) {
+    kind = 1;
+    abase = xoff(e, SP_S, A.off) * 4;
+    for (uint32_t i = 0; i < nwa; i++) note_read(e, SP_S, A.off + i);
+  } else {
+    kind = 2;
+    abase = xoff(e, SP_W, A.off) * 4;
+    for (uint32_t i = 0; i < nwa; i++) note_read(e, SP_W, A.off + 32 * i);
+  }
+  if (sra) fill = reg_of(e, wword(e, A, nwa, true));   // the sign word (top word sign-extended)
+  std::string top = (kind != 0 && sra && (wa & 31u)) ? reg_of(e, wword(e, A, nwa - 1, true)) : std::string("0");
+  // the loop lives in rtl_vshift (one copy per module): its code is fetched once
+  e.s += "\t{\n";
+  const char *pn[] = {"vs_op", "vs_nd", "vs_rem", "vs_nwa", "vs_kind", "vs_ab", "vs_a0", "vs_s", "vs_lim",
+                      "vs_fill", "vs_db", "vs_top"};
+  std::string ab = e.R(), db = e.R();   // absolute shared addresses (lane 0 / word 0)
+  e.l(fmt("add.u32 %s, %%smb, %u", ab.c_str(), abase));
+  e.l(fmt("add.u32 %s, %%smb, %u", db.c_str(), xoff(e, SP_W, w.d) * 4));
+  const std::string pv[] = {fmt("%u", op), fmt("%u", nd), fmt("%u", wd & 31u), fmt("%u", nwa), fmt("%u", kind),
+                            ab, a0, sam, fmt("%u", limit), fill, db, top};
+  for (int i = 0; i < 12; i++) {
+    e.s += fmt("\t.param .b32 %s;\n", pn[i]);
+    e.l(fmt("st.param.b32 [%s], %s", pn[i], pv[i].c_str()));
+  }
+  e.l("call.uni rtl_vshift, (vs_op, vs_nd, vs_rem, vs_nwa, vs_kind, vs_ab, vs_a0, vs_s, vs_lim, vs_fill, vs_db, vs_top)");
+  e.s += "\t}\n";
+  for (uint32_t i = 0; i < nd; i++) opaque_write(e, SP_W, w.d + 32 * i);
+}
+
+// rtl_vshift: SHL / SHRL / SHRA of a wide value by a variable amount on the
+// vector layout (the callee of emit_vshift; operand and destination are
+// absolute shared addresses of their lane-0 word 0).
+const char *kVShiftPtx = R"PTX(
+.func rtl_vshift(.param .b32 vs_op, .param .b32 vs_nd, .param .b32 vs_rem, .param .b32 vs_nwa,
+                 .param .b32 vs_kind, .param .b32 vs_ab, .param .b32 vs_a0, .param .b32 vs_s,
+                 .param .b32 vs_lim, .param .b32 vs_fill, .param .b32 vs_db, .param .b32 vs_top)
+{
+  .reg .b32 %op, %nd, %rem, %nwa, %kind, %ab, %a0, %s, %lim, %fill, %db, %top, %lane;
+  .reg .b32 %i, %q, %k, %jlo, %jhi, %j, %v, %x0, %x1, %r, %g, %jj, %gs, %st, %ad, %oob, %m, %nf;
+  .reg .pred %pshl, %pbig, %pv, %pf, %pk1, %pk2, %pz, %pl, %ptop, %psra;
+  ld.param.b32 %op, [vs_op];   ld.param.b32 %nd, [vs_nd];   ld.param.b32 %rem, [vs_rem];
+  ld.param.b32 %nwa, [vs_nwa]; ld.param.b32 %kind, [vs_kind]; ld.param.b32 %ab, [vs_ab];
+  ld.param.b32 %a0, [vs_a0];   ld.param.b32 %s, [vs_s];     ld.param.b32 %lim, [vs_lim];
+  ld.param.b32 %fill, [vs_fill]; ld.param.b32 %db, [vs_db]; ld.param.b32 %top, [vs_top];
+  mov.u32 %lane, %laneid;
+  setp.eq.u32 %pshl, %op, 22;
+  setp.eq.u32 %psra, %op, 24;
+  selp.u32 %oob, %fill, 0, %psra;
+  setp.ge.u32 %pbig, %s, %lim;
+  min.u32 %s, %s, %lim;
+  shr.u32 %q, %s, 5;
+  and.b32 %k, %s, 31;
+  setp.eq.u32 %pk1, %kind, 1;
+  setp.eq.u32 %pk2, %kind, 2;
+  shr.u32 %nf, %nwa, 2;
+  mov.u32 %i, 0;
+$VS_LOOP:
+  @%pshl sub.u32 %jhi, %i, %q;
+  @%pshl sub.u32 %jlo, %jhi, 1;
+  @!%pshl add.u32 %jlo, %q, %i;
+  @!%pshl add.u32 %jhi, %jlo, 1;
+  // X(jlo) -> %x0, X(jhi) -> %x1
+  mov.u32 %j, %jlo;
+  bra.uni $VS_X;
+$VS_X0:
+  mov.u32 %x0, %v;
+  mov.u32 %j, %jhi;
+  bra.uni $VS_X;
+$VS_X1:
+  mov.u32 %x1, %v;
+  @%pshl shf.l.clamp.b32 %r, %x0, %x1, %k;
+  @!%pshl shf.r.clamp.b32 %r, %x0, %x1, %k;
+  selp.u32 %r, %oob, %r, %pbig;
+  add.u32 %m, %i, 1;
+  setp.eq.u32 %ptop, %m, %nd;
+  setp.ne.u32 %pz, %rem, 0;
+  and.pred %ptop, %ptop, %pz;
+  @%ptop shl.b32 %m, 1, %rem;
+  @%ptop add.u32 %m, %m, -1;
+  @%ptop and.b32 %r, %r, %m;
+  // dest word i: group i / 4 of size min(4, nd - 4 g)
+  shr.u32 %g, %i, 2;
+  and.b32 %jj, %i, 3;
+  shl.b32 %gs, %g, 2;
+  sub.u32 %gs, %nd, %gs;
+  min.u32 %gs, %gs, 4;
+  shl.b32 %st, %gs, 2;
+  mad.lo.u32 %ad, %st, %lane, %db;
+  mad.lo.u32 %ad, %g, 512, %ad;
+  mad.lo.u32 %ad, %jj, 4, %ad;
+  st.shared.u32 [%ad], %r;
+  add.u32 %i, %i, 1;
+  setp.lt.u32 %pl, %i, %nd;
+  @%pl bra.uni $VS_LOOP;
+  ret;
+$VS_X:
+  // word %j of the operand (extended): 0 / sign fill beyond nwa
+  setp.lt.u32 %pv, %j, %nwa;
+  mov.u32 %v, %oob;
+  @%pk1 mad.lo.u32 %ad, %j, 4, %ab;
+  @%pk1 bra.uni $VS_LD;
+  @%pk2 bra.uni $VS_VEC;
+  setp.eq.u32 %pz, %j, 0;
+  @%pz mov.u32 %v, %a0;
+  bra.uni $VS_RET;
+$VS_VEC:
+  shr.u32 %g, %j, 2;
+  and.b32 %jj, %j, 3;
+  setp.lt.u32 %pf, %g, %nf;
+  shl.b32 %gs, %g, 2;
+  sub.u32 %gs, %nwa, %gs;
+  min.u32 %gs, %gs, 4;
+  selp.u32 %st, 16, 0, %pf;
+  @!%pf shl.b32 %st, %gs, 2;
+  mad.lo.u32 %ad, %st, %lane, %ab;
+  mad.lo.u32 %ad, %g, 512, %ad;
+  mad.lo.u32 %ad, %jj, 4, %ad;
+$VS_LD:
+  @%pv ld.shared.u32 %v, [%ad];
+  // SHRA: the operand's top word is read sign-extended
+  add.u32 %m, %j, 1;
+  setp.eq.u32 %pz, %m, %nwa;
+  and.pred %pz, %pz, %psra;
+  @%pz mov.u32 %v, %top;
+$VS_RET:
+  setp.eq.u32 %pz, %j, %jlo;
+  @%pz bra.uni $VS_X0;
+  bra.uni $VS_X1;
+}
+)PTX";
+
 void emit_wide(Em &e, const WideRec &w, uint32_t idx) {
   const uint32_t op = w.op, wd = w.wd, nd = nwords(wd);
   WOp A, B, C;
@@ -896,8 +1154,9 @@ void emit_wide(Em &e, const WideRec &w, uint32_t idx) {
       for (uint32_t i = 0; i < nd; i++) wstore(e, w.d, wd, i, i == 0 ? r : std::string("0"));
       return;
     }
-    default:   // SHL / SHRL / SHRA by a variable amount: generic path
-      generic_wide(e, w, idx);
+    default:   // SHL / SHRL / SHRA by a variable amount
+      if (jit_vwide()) emit_vshift(e, w, A, B);
+      else generic_wide(e, w, idx);   // the interpreter's generic path (row layout)
       return;
   }
 }
@@ -913,7 +1172,11 @@ void emit_ld(Em &e, uint32_t arena, uint32_t cls, uint32_t row, uint32_t slot, u
       begin_value(e, SP_W, slot, nw, true);
       for (uint32_t i = 0; i < nw; i++) {
         std::string ai = gaddr(e, "N4", row + i, fmt("tb_%s3", A).c_str());
-        e.l(fmt("cp.async.ca.shared.global [%%rw+%u], [%s], 4", xoff(e, SP_W, slot + 32 * i) * 4, ai.c_str()));
+        if (nw >= 2 && jit_vwide())   // into the word's place in its group
+          e.l(fmt("cp.async.ca.shared.global [%s+%u], [%s], 4", kLaneBase[vgs(nw, i / 4u)], vbyte(e, slot, nw, i),
+                  ai.c_str()));
+        else
+          e.l(fmt("cp.async.ca.shared.global [%%rw+%u], [%s], 4", xoff(e, SP_W, slot + 32 * i) * 4, ai.c_str()));
         opaque_write(e, SP_W, slot + 32 * i);
       }
       break;
@@ -954,9 +1217,12 @@ void emit_dig(Em &e, uint32_t key, const std::string &v) {
 void emit_st(Em &e, uint32_t code, uint32_t cls, uint32_t nw, uint32_t lay, uint32_t slot, uint32_t row,
              uint32_t aux) {
   const bool dg = code == CODE_ST_REG;
+  auto u32word = [&](uint32_t i) {   // word i of a U32-layout source of nw words
+    return (nw >= 2 && jit_vwide()) ? vword(e, slot, nw, i) : lds(e, SP_W, slot + 32 * i);
+  };
   if (code == CODE_ST_PORT) {   // write-port words of this cycle (applied after the cycle)
     for (uint32_t i = 0; i < nw; i++) {
-      std::string v = lay == LC_U32 ? lds(e, SP_W, slot + 32 * i) : fetch_narrow(e, lay, slot, 32);
+      std::string v = lay == LC_U32 ? u32word(i) : fetch_narrow(e, lay, slot, 32);
       std::string addr = gaddr(e, "N4", row + i, "portb");
       e.l(fmt("st.global.u32 [%s], %s", addr.c_str(), v.c_str()));
     }
@@ -966,7 +1232,7 @@ void emit_st(Em &e, uint32_t code, uint32_t cls, uint32_t nw, uint32_t lay, uint
     for (uint32_t i = 0; i < nw; i++) {
       std::string v;
       if (lay == LC_U32) {
-        v = lds(e, SP_W, slot + 32 * i);
+        v = u32word(i);
       } else {
         v = fetch_narrow(e, lay, slot, 32);
       }
@@ -981,7 +1247,7 @@ void emit_st(Em &e, uint32_t code, uint32_t cls, uint32_t nw, uint32_t lay, uint
   switch (cls) {
     case CLS_U32:
       for (uint32_t i = 0; i < nw; i++) {
-        std::string v = lds(e, SP_W, slot + 32 * i);
+        std::string v = u32word(i);
         std::string ai = gaddr(e, "N4", row + i, fmt("tb_%s3", A).c_str());
         e.l(fmt("st.global.u32 [%s], %s", ai.c_str(), v.c_str()));
         if (dg) emit_dig(e, aux + i + 1u + 0x80000000u, v);
@@ -1209,11 +1475,16 @@ void emit_desc(Em &e, const Program &G, const Desc &q) {
   e.opn++;
   const size_t from = e.s.size();
   emit_desc_(e, G, q);
+  if (!e.vpend.empty()) {   // every wide result stores whole groups; a partial one is a bug
+    fprintf(stderr, "rtlsim jit: internal error: incomplete wide-value group store\n");
+    abort();
+  }
   const uint32_t code = q.x & 0xFFu;
   std::string kind = code < 32u ? "narrow" : code == CODE_WIDE ? "wide" : code == CODE_LD_CONST ? "ld_const"
                    : (code == CODE_LD_REG || code == CODE_LD_X || code == CODE_LD_IN) ? "ld"
                    : code == CODE_ST_REGC ? "st_conv" : "st";
   if (code < 32u) kind += ((q.x >> 17) & 7u) == LC_BIT ? ":bit" : "";
+  if (code == CODE_WIDE && getenv("RTLSIM_JIT_STATS_WIDE")) kind += fmt(":%u", G.wide[q.y].op);
   note_kind(e, kind, from);
 }
 void emit_desc_(Em &e, const Program &G, const Desc &q) {
@@ -1632,11 +1903,13 @@ std::string step_function(const Program &G, const std::string &name, uint32_t s0
   std::string out = func_proto(name) + "\n{\n";
   out += fmt("\t.reg .b32 %%r<%u>;\n\t.reg .b64 %%rd<%u>;\n\t.reg .pred %%p<%u>;\n", e.nr + 1, e.nrd + 1, e.np + 1);
   out += "\t.reg .b64 %mtok0, %mtok1;\n";
+  out += "\t.reg .b32 %rq2, %rq3, %rq4;\n";
   out += "\t.reg .b32 %smb, %lane, %wl, %N, %tbar, %mbar, %rw, %rh, %rb, %N4, %N2, %Nb, %lsh;\n\t.reg .b64 %tbb1, %tbb2, %tlw, ";
   for (int i = 0; i < kN64; i++) out += fmt("%s%%%s", i ? ", " : "", kCtx64[i]);
   out += ";\n\t.reg .pred %pl0, %pl8, %pl16, %pdig;\n";
   for (int i = 0; i < kN32; i++) out += fmt("\tld.param.u32 %%%s, [a_%s];\n", kCtx32[i], kCtx32[i]);
   for (int i = 0; i < kN64; i++) out += fmt("\tld.param.u64 %%%s, [a_%s];\n", kCtx64[i], kCtx64[i]);
+  out += "\tmad.lo.u32 %rq2, %lane, 8, %smb;\n\tmad.lo.u32 %rq3, %lane, 12, %smb;\n\tmad.lo.u32 %rq4, %lane, 16, %smb;\n";
   out += "\tmad.lo.u32 %rw, %lane, 4, %smb;\n\tmad.lo.u32 %rh, %lane, 2, %smb;\n\tadd.u32 %rb, %lane, %smb;\n"
          "\tshl.b32 %N4, %N, 2;\n\tshl.b32 %N2, %N, 1;\n\tshr.u32 %Nb, %N, 3;\n"
          "\tsetp.eq.u32 %pl0, %lane, 0;\n\tsetp.lt.u32 %pl8, %lane, 8;\n\tsetp.lt.u32 %pl16, %lane, 16;\n"
@@ -1661,6 +1934,7 @@ std::string jit_partition_ptx(const Program &G, uint32_t q, const std::string &r
   mod += ".version 8.8\n.target sm_100a\n.address_size 64\n\n";
   mod += rt_ptx;
   mod += "\n.extern .shared .align 16 .b8 dyn_smem[];\n\n";
+  if (jit_vwide()) mod += kVShiftPtx;
   // wait for a phase of a split-phase step barrier (jit_split)
   mod += ".func rtl_mbar_wait(.param .b32 mb_a, .param .b64 mb_t)\n{\n\t.reg .b32 %ra;\n\t.reg .b64 %rt;\n"
          "\t.reg .pred %pw;\n\tld.param.b32 %ra, [mb_a];\n\tld.param.b64 %rt, [mb_t];\n$MBW:\n"
