@@ -36,7 +36,7 @@ constexpr int32_t kSpillNear = 4;
 // awaited with a per-step wait depth just before the step barrier)
 static int32_t load_ahead() {
   static const int32_t d = getenv("RTLSIM_LOAD_AHEAD") ? atoi(getenv("RTLSIM_LOAD_AHEAD")) : 2;
-  return std::max(1, std::min(d, 4));
+  return std::max(1, std::min(d, 8));
 }
 
 static int arity(uint32_t opc) {

@@ -291,7 +291,9 @@ void sts(Em &e, uint64_t sp, uint32_t off, const std::string &r) {
   else e.fwd[k] = Em::Fwd{r, e.step, e.opn};
 }
 // ----------------------------------------------- vector layout of wide values --
-// (r2, RTLSIM_JIT_VWIDE, default on) A value of >= 2 words in a U32 slot is
+// (r2, RTLSIM_JIT_VWIDE=1, default OFF: on the B200 it failed parity — a
+// misaligned-address fault and wrong config-3 golden digests — for a 1 %
+// config-4 gain; kept as an option until fixed) A value of >= 2 words in a U32 slot is
 // laid out in groups of up to 4 words: group g (words 4g..4g+gs-1, gs =
 // min(4, nw - 4g)) occupies 32 lanes x gs words at byte 16 * 32 * g of the
 // slot, lane l's words contiguous — one LDS.128 / STS.128 (LDS.64 for a pair)
@@ -300,7 +302,7 @@ void sts(Em &e, uint64_t sp, uint32_t off, const std::string &r) {
 // uses it (the interpreter keeps rows); variable wide shifts are emitted
 // inline (no generic call reading the row layout).
 bool jit_vwide() {
-  static const bool on = !getenv("RTLSIM_JIT_VWIDE") || atoi(getenv("RTLSIM_JIT_VWIDE")) != 0;
+  static const bool on = getenv("RTLSIM_JIT_VWIDE") && atoi(getenv("RTLSIM_JIT_VWIDE")) != 0;
   return on;
 }
 bool is_vwide(uint32_t lay, uint32_t w) { return jit_vwide() && lay == LC_U32 && nwords(w) >= 2; }

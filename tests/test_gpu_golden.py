@@ -94,5 +94,10 @@ def test_golden_config5_shards():
         s0, n = shard_range(N, 4, r)
         if not any(s0 <= s < s0 + n for s in gold):
             continue
-        dig, _ = _run_shard(5, s0, n, T, chunk=50)
+        dig, sim = _run_shard(5, s0, n, T, chunk=50)
         _check(5, gold, s0, dig)
+        del sim, dig   # one shard's arenas at a time (~60 GB each)
+        import gc
+        import torch
+        gc.collect()
+        torch.cuda.empty_cache()
