@@ -204,7 +204,7 @@ typedef struct {
   uint32_t jit_tiles_per_cta;  /* RTLSIM_F_JIT: tiles per CTA of the largest launch
                                 (warps of one op-lane that share each fetched
                                 instruction)                                  */
-  uint32_t pad0;
+  uint32_t tmem_cols;         /* (r2) TMEM columns per tile holding computed U32 values (RTLSIM_JIT_TMEM), else 0 */
 } rtlsim_stats_t;
 
 typedef struct rtlsim_ctx rtlsim_ctx;

@@ -153,8 +153,9 @@ static uint32_t fast_handler(uint32_t opc, int ar, const uint32_t *lay, uint32_t
 }
 
 int compile_program(const rtlsim_ir *ir, uint32_t op_lanes, uint32_t smem_limit_words, Program *P,
-                    std::string *err, bool dce, bool fold_conv) {
+                    std::string *err, bool dce, bool fold_conv, uint32_t tmem_cols) {
   if (!ir || !P) return fail(err, RTLSIM_E_ARG, "NULL ir");
+  tmem_cols = std::min<uint32_t>(tmem_cols, 512u);
   const uint32_t n = ir->n_signals;
   if (n == 0 || !ir->width || !ir->kind) return fail(err, RTLSIM_E_IR, "no signals");
   if ((ir->n_ops && !ir->ops) || (ir->n_regs && (!ir->reg_q || !ir->reg_d || !ir->reg_init)) ||
@@ -829,15 +830,48 @@ int compile_program(const rtlsim_ir *ir, uint32_t op_lanes, uint32_t smem_limit_
         born[vals[v].def_step].push_back((int32_t)v);
         dies[vals[v].last_use].push_back((int32_t)v);
       }
-      SlotAlloc sa((dump_words + 3u) & ~3u);
+      // (r2) TMEM: U32-layout values computed by this partition's ops (not
+      // cp.async load targets, not operands / results of the generic wide
+      // path, which addresses shared memory) take TMEM columns while they fit
+      std::vector<char> tm_ok(vals.size(), 0);
+      if (tmem_cols) {
+        for (size_t v = 0; v < vals.size(); v++) tm_ok[v] = vals[v].layout == LC_U32 && vals[v].def_step >= 0;
+        for (const Load &ld : loads) tm_ok[ld.val] = 0;
+        for (size_t j = 0; j < ops_p.size(); j++) {
+          const rtlsim_op &o = G.ops[ops_p[j]];
+          if (o.opcode != RTLSIM_OP_SHL && o.opcode != RTLSIM_OP_SHRL && o.opcode != RTLSIM_OP_SHRA) continue;
+          const int32_t vd = vid(o.dst), va = op_vals[j][0], vb = op_vals[j][1];
+          if (vd < 0 || va < 0 || vb < 0) continue;
+          const bool wide = vals[vd].width > 32 || vals[va].width > 32 || vals[vb].width > 32 ||
+                            vals[va].layout == LC_BCAST || vals[vb].layout == LC_BCAST;
+          if (wide) tm_ok[vd] = tm_ok[va] = tm_ok[vb] = 0;
+        }
+      }
+      SlotAlloc sa((dump_words + 3u) & ~3u), ta(0);
       for (int32_t s = 0; s < nsteps; s++) {
         // largest first keeps wide values contiguous and packs better
         std::sort(born[s].begin(), born[s].end(),
                   [&](int32_t x, int32_t y) { return vals[x].words() > vals[y].words(); });
-        for (int32_t v : born[s]) vals[v].slot = sa.alloc(vals[v].words());
-        for (int32_t v : dies[s]) sa.release(vals[v].slot, vals[v].words());
+        for (int32_t v : born[s]) {
+          if (tm_ok[v]) {
+            const uint32_t nw = nwords(vals[v].width), col = ta.alloc(nw);
+            if (col + nw <= tmem_cols) {
+              vals[v].slot = kTmemBase + 32u * col;
+              continue;
+            }
+            ta.release(col, nw);
+          }
+          vals[v].slot = sa.alloc(vals[v].words());
+        }
+        for (int32_t v : dies[s]) {
+          if (in_tmem(vals[v].slot) && vals[v].layout == LC_U32)
+            ta.release((vals[v].slot - kTmemBase) / 32u, nwords(vals[v].width));
+          else
+            sa.release(vals[v].slot, vals[v].words());
+        }
       }
       part_peak = sa.peak;
+      G.tmem_cols = std::max(G.tmem_cols, std::min(ta.peak, tmem_cols));
     }
       if (part_peak > slot_budget) {
         // spill more: local values live (beyond their near uses) across the
@@ -845,7 +879,7 @@ int compile_program(const rtlsim_ir *ir, uint32_t op_lanes, uint32_t smem_limit_
         // steps first, until the projected working set fits
         std::vector<double> live(nsteps + 1, 0.0);
         for (auto &v : vals) {
-          if (v.layout == LC_IMM || v.last_use < 0) continue;
+          if (v.layout == LC_IMM || v.last_use < 0 || (v.layout == LC_U32 && in_tmem(v.slot))) continue;
           for (int32_t t = v.def_step; t <= v.last_use; t++) live[t] += v.words();
         }
         // live words that fit the budget, given the allocator's fragmentation
@@ -854,6 +888,7 @@ int compile_program(const rtlsim_ir *ir, uint32_t op_lanes, uint32_t smem_limit_
         std::vector<std::pair<double, uint32_t>> cand;
         for (auto &v : vals) {
           if (v.layout == LC_IMM || v.last_use < 0 || !is_local(v.sig) || spilled.count(v.sig)) continue;
+          if (v.layout == LC_U32 && in_tmem(v.slot)) continue;   // spilling it frees no shared memory
           if (vid(v.sig) < 0 || &vals[vid(v.sig)] != &v) continue;   // the defining value only
           int32_t over = 0;
           for (int32_t t = v.def_step + kSpillNear; t <= v.last_use; t++) over += live[t] > target;

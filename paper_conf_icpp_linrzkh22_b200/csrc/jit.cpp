@@ -48,11 +48,11 @@ std::string fmt(const char *f, ...) {
 }
 
 // context values passed from the kernel to every step function
-const char *kCtx32[] = {"smb", "lane", "wl", "N", "tbar", "mbar"};
+const char *kCtx32[] = {"smb", "lane", "wl", "N", "tbar", "mbar", "tmt"};
 const char *kCtx64[] = {"tb_c0", "tb_c1", "tb_c2", "tb_c3", "tb_n0", "tb_n1", "tb_n2", "tb_n3",
                         "tb_x0", "tb_x1", "tb_x2", "tb_x3", "tb_i0", "tb_i1", "tb_i2", "tb_i3",
                         "outb", "dig", "wide", "smg", "bitl", "memb", "portb"};
-constexpr int kN32 = 6, kN64 = 23;
+constexpr int kN32 = 7, kN64 = 23;
 
 // Split-phase step barrier (RTLSIM_JIT_SPLIT=1; default off, see below):
 // instead of bar.sync at every step end, a warp arrives on an mbarrier (two,
@@ -271,7 +271,13 @@ std::string lds(Em &e, uint64_t sp, uint32_t off) {
     }
   }
   std::string r = e.R();
-  e.l(fmt("ld.shared.%s %s, [%s+%u]", kSpTy[sp], r.c_str(), kSpBase[sp], xoff(e, sp, off) * 4));
+  if (sp == SP_W && in_tmem(off)) {
+    // (r2) TMEM word: column (off - base) / 32 of this tile's lane quarter
+    e.l(fmt("tcgen05.ld.sync.aligned.32x32b.x1.b32 {%s}, [%%tmt+%u]", r.c_str(), (off - kTmemBase) / 32u));
+    e.l("tcgen05.wait::ld.sync.aligned");
+  } else {
+    e.l(fmt("ld.shared.%s %s, [%s+%u]", kSpTy[sp], r.c_str(), kSpBase[sp], xoff(e, sp, off) * 4));
+  }
   if (e.probe) e.log->rd[k].push_back(e.step);
   inst_read(e, sp, off);
   // a read-created entry is only as good as the read itself: a write by
@@ -285,8 +291,12 @@ void sts(Em &e, uint64_t sp, uint32_t off, const std::string &r) {
   const uint64_t k = skey(sp, off);
   const int64_t id = inst_of(e, sp, off);
   const bool unread = id >= 0 && !e.probe && !(*e.inst)[(size_t)id].need;   // compacted away
-  if (!unread && !(e.dse && e.log->dead_store(k, e.step, e.to_end)))
-    e.l(fmt("st.shared.%s [%s+%u], %s", kSpTy[sp], kSpBase[sp], xoff(e, sp, off) * 4, r.c_str()));
+  if (!unread && !(e.dse && e.log->dead_store(k, e.step, e.to_end))) {
+    if (sp == SP_W && in_tmem(off))
+      e.l(fmt("tcgen05.st.sync.aligned.32x32b.x1.b32 [%%tmt+%u], {%s}", (off - kTmemBase) / 32u, r.c_str()));
+    else
+      e.l(fmt("st.shared.%s [%s+%u], %s", kSpTy[sp], kSpBase[sp], xoff(e, sp, off) * 4, r.c_str()));
+  }
   if (e.dry) e.log->w[k].push_back({e.step, e.warp});
   else e.fwd[k] = Em::Fwd{r, e.step, e.opn};
 }
@@ -503,6 +513,45 @@ std::string wword(Em &e, WOp &o, uint32_t i, bool sx) {
   return o.fill;
 }
 
+// (r2) word i of a wide result held in TMEM: buffered until all n words are
+// there, then runs of live (not dead-store-eliminated) consecutive columns
+// go out as vector tcgen05.st (.x2 .. .x32)
+void tm_vstore(Em &e, uint32_t off, uint32_t n, uint32_t i, const std::string &v) {
+  auto &pend = e.vpend[((uint64_t)off << 8) | 0xFFu];
+  if (pend.size() < n) pend.resize(n);
+  pend[i] = v;
+  const uint64_t k = skey(SP_W, off + 32u * i);
+  if (e.dry) e.log->w[k].push_back({e.step, e.warp});
+  else e.fwd[k] = Em::Fwd{v, e.step, e.opn};
+  for (uint32_t j = 0; j < n; j++)
+    if (pend[j].empty()) return;
+  std::vector<char> live(n, 1);
+  for (uint32_t j = 0; j < n; j++)
+    live[j] = !(e.dse && e.log->dead_store(skey(SP_W, off + 32u * j), e.step, e.to_end));
+  const uint32_t c0 = (off - kTmemBase) / 32u;
+  for (uint32_t j = 0; j < n;) {
+    if (!live[j]) {
+      j++;
+      continue;
+    }
+    uint32_t m = j + 1;
+    while (m < n && live[m]) m++;
+    uint32_t c = c0 + j, rem = m - j, w = j;
+    while (rem) {
+      uint32_t cnt = 1;
+      while (cnt * 2 <= rem && cnt * 2 <= 32u && (c % (cnt * 2)) == 0) cnt *= 2;
+      std::string regs;
+      for (uint32_t t = 0; t < cnt; t++) regs += (t ? ", " : "") + pend[w + t];
+      e.l(fmt("tcgen05.st.sync.aligned.32x32b.x%u.b32 [%%tmt+%u], {%s}", cnt, c, regs.c_str()));
+      c += cnt;
+      w += cnt;
+      rem -= cnt;
+    }
+    j = m;
+  }
+  e.vpend.erase(((uint64_t)off << 8) | 0xFFu);
+}
+
 // store word i of a wide result (masking the top word)
 void wstore(Em &e, uint32_t off, uint32_t wd, uint32_t i, const std::string &v) {
   const uint32_t n = nwords(wd), rem = wd & 31u;
@@ -525,7 +574,8 @@ void wstore(Em &e, uint32_t off, uint32_t wd, uint32_t i, const std::string &v) 
     e.l(fmt("and.b32 %s, %s, %u", m.c_str(), x.c_str(), mask_of(rem)));
     x = m;
   }
-  if (jit_vwide()) vstore(e, off, n, i, x);
+  if (in_tmem(off) && n >= 2) tm_vstore(e, off, n, i, x);
+  else if (jit_vwide()) vstore(e, off, n, i, x);
   else sts(e, SP_W, off + 32 * i, x);
 }
 
@@ -744,6 +794,9 @@ void emit_generic_call(Em &e, uint32_t idx) {
   e.s += "\t}\n";
 }
 void generic_wide(Em &e, const WideRec &w, uint32_t idx) {
+  if (getenv("RTLSIM_TMEM_DEBUG") && (in_tmem(w.a) || in_tmem(w.b) || in_tmem(w.c) || in_tmem(w.d)))
+    fprintf(stderr, "generic wide op %u with a TMEM operand: d %x a %x b %x c %x wd %u wa %u wb %u lays %x\n", w.op,
+            w.d, w.a, w.b, w.c, w.wd, w.wa, w.wb, w.lays);
   note_operand_reads(e, w.a, w.wa, w.lays & 0xFFu);
   note_operand_reads(e, w.b, w.wb, (w.lays >> 8) & 0xFFu);
   note_operand_reads(e, w.c, w.wc, (w.lays >> 16) & 0xFFu);
@@ -1473,9 +1526,68 @@ void note_kind(Em &e, const std::string &kind, size_t from) {
 }
 
 void emit_desc_(Em &e, const Program &G, const Desc &q);
+void desc_keys(const Program &G, const Desc &q, std::vector<uint64_t> &src, std::vector<uint64_t> &dst, bool *ld);
+// (r2) TMEM operands of a descriptor: every word not already in a register
+// is loaded up front — runs of consecutive columns as vector tcgen05.ld
+// (.x2 .. .x32), one tcgen05.wait::ld for all — and handed to the emitter as
+// forwarded registers (lds() then finds them)
+void tm_prefetch(Em &e, const Program &G, const Desc &q) {
+  std::vector<uint64_t> src, dst;
+  bool ld = false;
+  desc_keys(G, q, src, dst, &ld);
+  const uint32_t code = q.x & 0xFFu;
+  uint32_t lo = 0, hi = UINT32_MAX;   // SLICE of a wide operand: only the words it reads
+  if (code == CODE_WIDE && G.wide[q.y].op == RTLSIM_OP_SLICE) {
+    const WideRec &r = G.wide[q.y];
+    lo = r.imm / 32u;
+    hi = (r.imm + r.wd - 1u) / 32u;
+  }
+  std::vector<uint32_t> cols;
+  for (uint64_t k : src) {
+    const uint32_t off = (uint32_t)k;
+    if ((k >> 32) != SP_W || !in_tmem(off) || !fwd_get(e, k).empty()) continue;
+    if (code == CODE_WIDE && G.wide[q.y].op == RTLSIM_OP_SLICE) {
+      const uint32_t i = (off - G.wide[q.y].a) / 32u;
+      if (i < lo || i > hi) continue;
+    }
+    cols.push_back((off - kTmemBase) / 32u);
+  }
+  if (cols.empty()) return;
+  std::sort(cols.begin(), cols.end());
+  cols.erase(std::unique(cols.begin(), cols.end()), cols.end());
+  std::vector<std::pair<uint32_t, std::string>> got;
+  for (size_t i = 0; i < cols.size();) {
+    size_t j = i + 1;
+    while (j < cols.size() && cols[j] == cols[j - 1] + 1) j++;
+    uint32_t c = cols[i], rem = (uint32_t)(j - i);
+    while (rem) {
+      uint32_t n = 1;
+      while (n * 2 <= rem && n * 2 <= 32u && (c % (n * 2)) == 0) n *= 2;   // naturally aligned chunks
+      std::string regs;
+      for (uint32_t t = 0; t < n; t++) {
+        std::string r = e.R();
+        regs += (t ? ", " : "") + r;
+        got.push_back({c + t, r});
+      }
+      e.l(fmt("tcgen05.ld.sync.aligned.32x32b.x%u.b32 {%s}, [%%tmt+%u]", n, regs.c_str(), c));
+      c += n;
+      rem -= n;
+    }
+    i = j;
+  }
+  e.l("tcgen05.wait::ld.sync.aligned");
+  for (auto &g : got) {
+    const uint32_t off = kTmemBase + 32u * g.first;
+    const uint64_t k = skey(SP_W, off);
+    if (e.probe) e.log->rd[k].push_back(e.step);
+    inst_read(e, SP_W, off);
+    e.fwd[k] = Em::Fwd{g.second, e.step - 1, e.opn};
+  }
+}
 void emit_desc(Em &e, const Program &G, const Desc &q) {
   e.opn++;
   const size_t from = e.s.size();
+  if (G.tmem_cols && !e.dry && e.fwd_max > 0) tm_prefetch(e, G, q);
   emit_desc_(e, G, q);
   if (!e.vpend.empty()) {   // every wide result stores whole groups; a partial one is a bug
     fprintf(stderr, "rtlsim jit: internal error: incomplete wide-value group store\n");
@@ -1833,6 +1945,12 @@ std::string step_function(const Program &G, const std::string &name, uint32_t s0
       // CUTLASS kernels rely on when producer and consumer warps meet at a
       // named barrier from different code. The aligned form is kept;
       // RTLSIM_JIT_TBAR=2 emits the non-aligned one for A/B.
+      // (r2) TMEM values: this warp's tcgen05.st complete and ordered before
+      // the barrier, other warps' after it (fence / sync / fence)
+      if (G.tmem_cols) {
+        e.l("tcgen05.wait::st.sync.aligned");
+        e.l("tcgen05.fence::before_thread_sync");
+      }
       if (jit_tbar() == 0)
         e.l("bar.sync 0");
       else if (jit_tbar() == 2)
@@ -1841,6 +1959,7 @@ std::string step_function(const Program &G, const std::string &name, uint32_t s0
         e.l(fmt("bar.sync %%tbar, %u", 32u * G.L));   // aligned: one per step in every warp of the tile
       else
         e.l("bar.warp.sync -1");
+      if (G.tmem_cols) e.l("tcgen05.fence::after_thread_sync");
     }
     if (G.L > 1) e.l(fmt("bra.uni %s", end.c_str()));
   }
@@ -1906,7 +2025,7 @@ std::string step_function(const Program &G, const std::string &name, uint32_t s0
   out += fmt("\t.reg .b32 %%r<%u>;\n\t.reg .b64 %%rd<%u>;\n\t.reg .pred %%p<%u>;\n", e.nr + 1, e.nrd + 1, e.np + 1);
   out += "\t.reg .b64 %mtok0, %mtok1;\n";
   out += "\t.reg .b32 %rq2, %rq3, %rq4;\n";
-  out += "\t.reg .b32 %smb, %lane, %wl, %N, %tbar, %mbar, %rw, %rh, %rb, %N4, %N2, %Nb, %lsh;\n\t.reg .b64 %tbb1, %tbb2, %tlw, ";
+  out += "\t.reg .b32 %smb, %lane, %wl, %N, %tbar, %mbar, %tmt, %rw, %rh, %rb, %N4, %N2, %Nb, %lsh;\n\t.reg .b64 %tbb1, %tbb2, %tlw, ";
   for (int i = 0; i < kN64; i++) out += fmt("%s%%%s", i ? ", " : "", kCtx64[i]);
   out += ";\n\t.reg .pred %pl0, %pl8, %pl16, %pdig;\n";
   for (int i = 0; i < kN32; i++) out += fmt("\tld.param.u32 %%%s, [a_%s];\n", kCtx32[i], kCtx32[i]);
@@ -1976,12 +2095,19 @@ std::string jit_partition_ptx(const Program &G, uint32_t q, const std::string &r
   // the warps of one op-lane (one per tile) run identical code in step
   // lock-step and share its instruction fetch.
   mod += fmt(".visible .entry rtl_jit_part(.param .align 8 .b8 prm[%zu])\n.maxntid %u, 1, 1\n{\n",
-             sizeof(JitParams), 32u * G.L * std::max<uint32_t>(tmax, 1u));
-  mod += "\t.reg .b32 %tidx, %tile, %s, %smb, %lane, %wl, %N, %wg, %tsub, %tpc, %tbar, %mbar, %nthr;\n\t.reg .b64 %t64, %b64, %digb;\n\t.reg .pred %pz;\n\t.reg .b64 ";
+             sizeof(JitParams), 32u * G.L * (G.tmem_cols ? 4u : std::max<uint32_t>(tmax, 1u)));
+  mod += "\t.reg .b32 %tidx, %tile, %s, %smb, %lane, %wl, %N, %wg, %tsub, %tpc, %tbar, %mbar, %nthr, %tmt, %tmb;\n\t.reg .b64 %t64, %b64, %digb;\n\t.reg .pred %pz, %pw0;\n\t.reg .b64 ";
   for (int i = 0; i < kN64; i++) mod += fmt("%s%%%s", i ? ", " : "", kCtx64[i]);
   mod += ";\n";
-  mod += fmt("\tmov.u32 %%tidx, %%tid.x;\n\tand.b32 %%lane, %%tidx, 31;\n\tshr.u32 %%wg, %%tidx, 5;\n"
-             "\trem.u32 %%wl, %%wg, %u;\n\tdiv.u32 %%tsub, %%wg, %u;\n", G.L, G.L);
+  if (G.tmem_cols)
+    // (r2) TMEM mode: 4 tiles per CTA, tile t on lane quarter / SMSP t (warp
+    // w: tile w & 3, op-lane w >> 2) — a warp reaches only its quarter's lanes
+    mod += "\tmov.u32 %tidx, %tid.x;\n\tand.b32 %lane, %tidx, 31;\n\tshr.u32 %wg, %tidx, 5;\n"
+           "\tshr.u32 %wl, %wg, 2;\n\tand.b32 %tsub, %wg, 3;\n";
+  else
+    mod += fmt("\tmov.u32 %%tidx, %%tid.x;\n\tand.b32 %%lane, %%tidx, 31;\n\tshr.u32 %%wg, %%tidx, 5;\n"
+               "\trem.u32 %%wl, %%wg, %u;\n\tdiv.u32 %%tsub, %%wg, %u;\n", G.L, G.L);
+  mod += "\tsetp.lt.u32 %pw0, %tidx, 32;\n\tmov.u32 %tmt, 0;\n\tmov.u32 %tmb, 0;\n";
   mod += fmt("\tld.param.u32 %%tpc, [prm+%zu];\n", offsetof(JitParams, tpc));
   mod += "\tadd.u32 %tbar, %tsub, 1;\n";
   mod += "\tmov.u32 %tile, %ctaid.x;\n\tmad.lo.u32 %tile, %tile, %tpc, %tsub;\n\tmad.lo.u32 %s, %tile, 32, %lane;\n";
@@ -2021,6 +2147,18 @@ std::string jit_partition_ptx(const Program &G, uint32_t q, const std::string &r
   mod += fmt("\tmov.u32 %%smb, dyn_smem;\n\tmad.lo.u32 %%smb, %%tsub, %u, %%smb;\n\tcvta.shared.u64 %%smg, dyn_smem;\n"
              "\tmul.wide.u32 %%t64, %%tsub, %u;\n\tadd.u64 %%smg, %%smg, %%t64;\n",
              tbytes, tbytes);
+  uint32_t tcols = 32;   // TMEM allocation: a power of two >= 32 columns
+  while (tcols < G.tmem_cols) tcols *= 2;
+  if (G.tmem_cols) {
+    // (r2) warp 0 allocates the TMEM columns (one CTA per SM: the tiles
+    // fill the shared memory) and publishes the base after the split-barrier
+    // pair; lane quarter t of the allocation belongs to tile t
+    mod += "\t{\n\t.reg .b32 %ta;\n\tadd.u32 %ta, %mbar, 16;\n";
+    mod += fmt("\t@%%pw0 tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%%ta], %u;\n", tcols);
+    mod += "\t@%pw0 tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;\n"
+           "\ttcgen05.fence::before_thread_sync;\n\tbar.sync 0;\n\ttcgen05.fence::after_thread_sync;\n"
+           "\tld.shared.u32 %tmb, [%ta];\n\tshl.b32 %ta, %tsub, 21;\n\tadd.u32 %tmt, %tmb, %ta;\n\t}\n";
+  }
   // M1 cycle loop (nc > 1, single-partition designs only): after each cycle
   // the state buffers swap, the input / output / digest rows advance, and a
   // CTA barrier orders this cycle's register stores before the next cycle's
@@ -2051,6 +2189,9 @@ std::string jit_partition_ptx(const Program &G, uint32_t q, const std::string &r
   mod += fmt("\tld.param.u64 %%stp, [prm+%zu];\n\tsetp.ne.u64 %%pcy, %%dig, 0;\n\t@%%pcy add.u64 %%dig, %%dig, %%stp;\n",
              offsetof(JitParams, dig_step));
   mod += "\tbar.sync 0;\n\tbra.uni $CYC;\n$CYCE:\n\t}\n";
+  if (G.tmem_cols)
+    mod += "\ttcgen05.fence::before_thread_sync;\n\tbar.sync 0;\n\ttcgen05.fence::after_thread_sync;\n" +
+           fmt("\t@%%pw0 tcgen05.dealloc.cta_group::1.sync.aligned.b32 %%tmb, %u;\n", tcols);
   mod += "\tret;\n}\n";
   return mod;
 }
@@ -2129,7 +2270,7 @@ int jit_build(const Program &G, const std::string &rt_ptx_path, uint32_t smem_by
       : std::max<uint32_t>(
             1u, std::min<uint32_t>(std::min<uint32_t>(jit_default_tiles(), 32u / std::max<uint32_t>(G.L, 1u)),
                                    smem_bytes / jit_tile_bytes(G)));
-  out->tmax = tmax;
+  out->tmax = G.tmem_cols ? 4u : tmax;   // TMEM: four tiles, one per lane quarter
   out->compact = compact;
   std::vector<JitPartInfo> infos(NP);
   out->nspec = nspec;
@@ -2168,6 +2309,8 @@ int jit_build(const Program &G, const std::string &rt_ptx_path, uint32_t smem_by
     th.emplace_back([&]() {
       for (uint32_t q; (q = next++) < NP;) {
         if (G.part_steps[q] == G.part_steps[q + 1]) continue;
+        // debugging aid (host-only inspection): RTLSIM_JIT_ONLY=q emits one partition
+        if (getenv("RTLSIM_JIT_ONLY") && (uint32_t)atoi(getenv("RTLSIM_JIT_ONLY")) != q) continue;
         std::string ptx = jit_partition_ptx(G, q, rt, tmax, dig, nspec, &infos[q]);
         ptx_bytes += ptx.size();
         if (const char *dir = getenv("RTLSIM_JIT_SAVE")) {   // debugging aid: keep the module

@@ -45,6 +45,11 @@ constexpr uint32_t kJitMaxTiles = 16;
 // overrides, up to kJitMaxTiles and 1024 threads per CTA).
 uint32_t jit_default_tiles(bool compact = false);
 // Bytes of shared memory per tile in a JIT CTA (16-byte aligned).
+// (r2) RTLSIM_JIT_TMEM=1: computed U32 values in tensor memory (four tiles per CTA)
+inline bool jit_tmem_env() {
+  const char *e = getenv("RTLSIM_JIT_TMEM");
+  return e && atoi(e) != 0;
+}
 inline uint32_t jit_tile_bytes(const Program &G) { return ((G.smem_words * 4u) + 15u) & ~15u; }
 
 // What the generator decided for one partition kernel beyond its PTX.

@@ -54,6 +54,13 @@ enum : uint32_t {
 };
 
 inline uint32_t nwords(uint32_t w) { return (w + 31u) / 32u; }
+
+// (r2) TMEM-resident values (JIT, RTLSIM_JIT_TMEM): a U32-layout value computed
+// by an op may live in tensor memory instead of a shared-memory slot. Its
+// "slot" is kTmemBase + 32 * column (word i at column + i, one TMEM lane per
+// stimulus), so the per-word key arithmetic off + 32 i stays the same.
+constexpr uint32_t kTmemBase = 0x8000u;
+inline bool in_tmem(uint32_t slot) { return slot >= kTmemBase && slot < kTmemBase + 32u * 512u; }
 inline uint32_t width_class(uint32_t w) {
   return w == 1 ? CLS_BIT : w <= 8 ? CLS_U8 : w <= 16 ? CLS_U16 : CLS_U32;
 }
@@ -141,6 +148,7 @@ struct Program {
   std::vector<uint32_t> part_steps;     // exec-order partition boundaries in steps (size P+1)
   std::vector<std::vector<uint32_t>> part_dep;   // exec-order partitions each one waits for in a cycle
   uint32_t smem_words = 0;              // shared words per tile (slots)
+  uint32_t tmem_cols = 0;               // (r2) TMEM columns per tile (0: no TMEM values)
   // ---- memories (ARRSEL, reading 12; JIT backend only)
   std::vector<uint16_t> mem_width;
   std::vector<uint32_t> mem_depth, mem_row0;  // first u32 row of each memory in the memory arena
@@ -161,7 +169,7 @@ struct Program {
 
 // Returns RTLSIM_OK or a negative status with *err set.
 int compile_program(const rtlsim_ir *ir, uint32_t op_lanes, uint32_t smem_limit_words, Program *out,
-                    std::string *err, bool dce = true, bool fold_conv = false);
+                    std::string *err, bool dce = true, bool fold_conv = false, uint32_t tmem_cols = 0);
 
 // 3-input truth table (bit k = f(a = k&1, b = k>>1&1, c = k>>2&1)) of an IR
 // opcode on 1-bit operands and a 1-bit result.

@@ -216,8 +216,15 @@ extern "C" int rtlsim_load(const rtlsim_ir *ir, const rtlsim_options *opt, rtlsi
   const bool dce = (ctx->opt.flags & RTLSIM_F_NO_DCE) == 0;
   const bool fold = (ctx->opt.flags & RTLSIM_F_JIT) != 0 && !getenv("RTLSIM_NO_FOLD");   // JIT-only store-with-conversion descriptors
   if (!lanes && (ctx->opt.flags & RTLSIM_F_JIT)) lanes = kJitMaxLanes;
-  int rc = compile_program(ir, lanes, smem_limit / 4u, &ctx->prog, &err, dce, fold);
-  if (rc == RTLSIM_OK && !ctx->opt.op_lanes && (ctx->opt.flags & RTLSIM_F_JIT) && ctx->prog.L > 1) {
+  // (r2) RTLSIM_JIT_TMEM=1: U32 values computed by ops live in tensor memory;
+  // four tiles per CTA (one per TMEM lane quarter / SMSP), up to 8 op-lanes
+  const bool tmem = (ctx->opt.flags & RTLSIM_F_JIT) && jit_tmem_env();
+  if (tmem) lanes = std::min<uint32_t>(ctx->opt.op_lanes ? ctx->opt.op_lanes : 8u, 8u);
+  int rc = tmem ? compile_program(ir, lanes, (smem_limit - 256u) / 4u / 4u, &ctx->prog, &err, dce, fold, 512u)
+                : compile_program(ir, lanes, smem_limit / 4u, &ctx->prog, &err, dce, fold);
+  if (rc == RTLSIM_OK && tmem) {
+    // no recompiles below: the TMEM schedule's budget is fixed
+  } else if (rc == RTLSIM_OK && !ctx->opt.op_lanes && (ctx->opt.flags & RTLSIM_F_JIT) && ctx->prog.L > 1) {
     // keep the auto choice when it is smaller than the cap
     rtlsim::Program probe;
     std::string e2;
@@ -244,7 +251,7 @@ extern "C" int rtlsim_load(const rtlsim_ir *ir, const rtlsim_options *opt, rtlsi
   }
   const bool legacy = true;   // the descriptor interpreter: staging buffers per op-lane
   uint32_t budget_words = smem_limit / 4u;
-  if ((ctx->opt.flags & RTLSIM_F_JIT) && !ctx->opt.smem_limit &&
+  if ((ctx->opt.flags & RTLSIM_F_JIT) && !ctx->opt.smem_limit && !tmem &&
       (ctx->prog.smem_words + 64u) * 4u > smem_limit / 2u) {
     // JIT kernels are instruction-fetch bound: two tiles per CTA (the warps
     // of one op-lane share every fetched instruction) beat one tile with the
@@ -258,7 +265,7 @@ extern "C" int rtlsim_load(const rtlsim_ir *ir, const rtlsim_options *opt, rtlsi
       budget_words = (smem_limit / 2u - 1024u) / 4u;
     }
   }
-  if ((ctx->opt.flags & RTLSIM_F_JIT) && !ctx->opt.op_lanes && ctx->prog.L == kJitMaxLanes) {
+  if ((ctx->opt.flags & RTLSIM_F_JIT) && !ctx->opt.op_lanes && !tmem && ctx->prog.L == kJitMaxLanes) {
     // Occupancy: as many warps per SM as a 1024-thread CTA holds. K tiles fit
     // the shared memory; more op-lanes per tile fill the CTA when K is small
     // (measured round 2, profiles/r02_sweep_*.log: config 4 (K = 2) 4 / 8 /
@@ -448,7 +455,9 @@ static int bind_common(rtlsim_ctx *ctx, uint64_t N, uint64_t T) {
   free_binding(ctx);
   ctx->N = N;
   ctx->T = T;
-  ctx->N_pad = (uint32_t)((N + 31) / 32 * 32);
+  // (r2) TMEM kernels run exactly four tiles per CTA: N_pad in 128s
+  const uint64_t padq = ctx->prog.tmem_cols ? 128u : 32u;
+  ctx->N_pad = (uint32_t)((N + padq - 1) / padq * padq);
   Program &G = ctx->prog;
   ctx->Tc = ctx->opt.chunk_cycles ? ctx->opt.chunk_cycles : 64;
   if (T) ctx->Tc = (uint32_t)std::min<uint64_t>(ctx->Tc, T);
@@ -597,6 +606,7 @@ static uint32_t jit_tiles_per_cta(rtlsim_ctx *ctx, const JitKernels &JK, uint32_
   // the kernel set being launched (the check-mode variant may have been built
   // with another RTLSIM_JIT_TMAX than the plain one): its .maxntid bound; the
   // partition's own shared memory per tile (compacted kernels differ)
+  if (ctx->prog.tmem_cols) return 4u;   // one tile per TMEM lane quarter
   uint32_t m = std::min<uint32_t>(JK.tmax, ((uint32_t)optin - 16u) / std::max<uint32_t>(jit_tile_smem(ctx, JK, q), 1u));
   if (const char *e = getenv("RTLSIM_JIT_TPC")) m = std::min<uint32_t>(m, (uint32_t)atoi(e));
   m = std::max<uint32_t>(m, 1u);
@@ -760,7 +770,7 @@ static int launch_chunk(rtlsim_ctx *ctx, int b, uint64_t cycle0, uint32_t nc, bo
           jp.tpc = jit_tiles_per_cta(ctx, JK, q);
           void *args[] = {&jp};
           e = cudaLaunchKernel((const void *)JK.kern[q], dim3(ctx->N_pad / 32u / jp.tpc),
-                               dim3(32u * G.L * jp.tpc), args, jit_tile_smem(ctx, JK, q) * jp.tpc + 16u, sq);
+                               dim3(32u * G.L * jp.tpc), args, jit_tile_smem(ctx, JK, q) * jp.tpc + 32u, sq);
         } else {
           EvalParams p = eval_params(ctx, b, (cycle0 & 1ull) + c, 1, digest);
           p.step_begin = G.part_steps[q];
@@ -1185,6 +1195,7 @@ extern "C" int rtlsim_stats(const rtlsim_ctx *cctx, rtlsim_stats_t *st) {
   st->jit_cubin_bytes = ctx->jit.cubin_bytes;
   st->jit_sass_instructions = ctx->jit.sass_instructions;
   st->jit_tiles_per_cta = 0;
+  st->tmem_cols = ctx->prog.tmem_cols;
   if (!ctx->jit.kern.empty() && ctx->N_pad)
     for (uint32_t q = 0; q < ctx->jit.kern.size(); q++)
       if (ctx->jit.kern[q]) st->jit_tiles_per_cta = std::max(st->jit_tiles_per_cta, jit_tiles_per_cta(ctx, ctx->jit, q));

@@ -79,7 +79,7 @@ class Stats(ctypes.Structure):
                 ("n_ld", ctypes.c_uint64), ("n_st", ctypes.c_uint64), ("b_spill", ctypes.c_double),
                 ("n_live_ops", ctypes.c_uint64), ("live_word_ops", ctypes.c_uint64),
                 ("jit_sass_instructions", ctypes.c_uint64), ("jit_tiles_per_cta", ctypes.c_uint32),
-                ("pad0", ctypes.c_uint32)]
+                ("tmem_cols", ctypes.c_uint32)]
 
 
 PRODUCER = ctypes.CFUNCTYPE(ctypes.c_int, ctypes.c_void_p, ctypes.c_uint64, ctypes.c_uint64,
