@@ -384,6 +384,9 @@ def run_ours(a):
                 "warp_instructions_per_live_op": (st["jit_sass_instructions"] / max(1, st["n_live_ops"])
                                                   if st["jit_sass_instructions"] else None),
                 "warps_sharing_each_fetched_instruction": st["jit_tiles_per_cta"] or None,
+                "tmem_cols_per_tile": st["tmem_cols"],
+                "value_tiers": ("shared memory + TMEM (computed U32 values, tcgen05.ld/st)" if st["tmem_cols"]
+                                else "shared memory"),
                 "design_seed": hex(stim.DESIGN_SEED_BASE + cid), "stim_seed": hex(seed),
                 "parallelism": f"contiguous stimulus shards x{world} (parallel.run_sharded)",
                 "schedule": "jit per-(cycle, partition) kernels, graph-launched" if a.backend == "jit"

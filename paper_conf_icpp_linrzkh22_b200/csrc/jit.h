@@ -45,10 +45,11 @@ constexpr uint32_t kJitMaxTiles = 16;
 // overrides, up to kJitMaxTiles and 1024 threads per CTA).
 uint32_t jit_default_tiles(bool compact = false);
 // Bytes of shared memory per tile in a JIT CTA (16-byte aligned).
-// (r2) RTLSIM_JIT_TMEM=1: computed U32 values in tensor memory (four tiles per CTA)
-inline bool jit_tmem_env() {
+// (r2) TMEM schedules (computed U32 values in tensor memory, four tiles per
+// CTA): RTLSIM_JIT_TMEM unset = auto (-1), 0 = off, 1 = whenever it fits
+inline int jit_tmem_mode() {
   const char *e = getenv("RTLSIM_JIT_TMEM");
-  return e && atoi(e) != 0;
+  return e ? (atoi(e) != 0 ? 1 : 0) : -1;
 }
 inline uint32_t jit_tile_bytes(const Program &G) { return ((G.smem_words * 4u) + 15u) & ~15u; }
 

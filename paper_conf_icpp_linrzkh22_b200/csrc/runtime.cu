@@ -216,15 +216,9 @@ extern "C" int rtlsim_load(const rtlsim_ir *ir, const rtlsim_options *opt, rtlsi
   const bool dce = (ctx->opt.flags & RTLSIM_F_NO_DCE) == 0;
   const bool fold = (ctx->opt.flags & RTLSIM_F_JIT) != 0 && !getenv("RTLSIM_NO_FOLD");   // JIT-only store-with-conversion descriptors
   if (!lanes && (ctx->opt.flags & RTLSIM_F_JIT)) lanes = kJitMaxLanes;
-  // (r2) RTLSIM_JIT_TMEM=1: U32 values computed by ops live in tensor memory;
-  // four tiles per CTA (one per TMEM lane quarter / SMSP), up to 8 op-lanes
-  const bool tmem = (ctx->opt.flags & RTLSIM_F_JIT) && jit_tmem_env();
-  if (tmem) lanes = std::min<uint32_t>(ctx->opt.op_lanes ? ctx->opt.op_lanes : 8u, 8u);
-  int rc = tmem ? compile_program(ir, lanes, (smem_limit - 256u) / 4u / 4u, &ctx->prog, &err, dce, fold, 512u)
-                : compile_program(ir, lanes, smem_limit / 4u, &ctx->prog, &err, dce, fold);
-  if (rc == RTLSIM_OK && tmem) {
-    // no recompiles below: the TMEM schedule's budget is fixed
-  } else if (rc == RTLSIM_OK && !ctx->opt.op_lanes && (ctx->opt.flags & RTLSIM_F_JIT) && ctx->prog.L > 1) {
+  const bool tmem = false;   // the TMEM schedule is chosen below, after the classic one
+  int rc = compile_program(ir, lanes, smem_limit / 4u, &ctx->prog, &err, dce, fold);
+  if (rc == RTLSIM_OK && !ctx->opt.op_lanes && (ctx->opt.flags & RTLSIM_F_JIT) && ctx->prog.L > 1) {
     // keep the auto choice when it is smaller than the cap
     rtlsim::Program probe;
     std::string e2;
@@ -282,6 +276,24 @@ extern "C" int rtlsim_load(const rtlsim_ir *ir, const rtlsim_options *opt, rtlsi
       if (compile_program(ir, want, budget_words, &wide, &e2, dce, fold) == RTLSIM_OK &&
           wide.smem_words <= ctx->prog.smem_words)
         ctx->prog = std::move(wide);
+    }
+  }
+  // (r2) TMEM schedule (JIT): U32 values computed by ops live in tensor
+  // memory, four tiles per CTA (one per TMEM lane quarter / SMSP), up to 8
+  // op-lanes. The JIT kernels are instruction-fetch bound:
+  // four warps sharing each fetched instruction instead of two measured
+  // config 4 at 55.6 vs 76.2 ms/cycle; designs whose classic working set
+  // already fits four tiles gain nothing (config 3: 1.59 vs 1.47). Auto:
+  // when fewer than four classic tiles fit; RTLSIM_JIT_TMEM=1 / 0 forces.
+  if ((ctx->opt.flags & RTLSIM_F_JIT) && !ctx->opt.smem_limit && jit_tmem_mode() != 0) {
+    const bool want = jit_tmem_mode() == 1 || jit_tile_bytes(ctx->prog) * 4u + 256u > smem_limit;
+    if (want) {
+      rtlsim::Program tp;
+      std::string e2;
+      const uint32_t tl = std::min<uint32_t>(ctx->opt.op_lanes ? ctx->opt.op_lanes : 8u, 8u);
+      if (compile_program(ir, tl, (smem_limit - 256u) / 16u, &tp, &e2, dce, fold, 512u) == RTLSIM_OK &&
+          tp.tmem_cols > 0 && jit_tile_bytes(tp) * 4u + 256u <= smem_limit)
+        ctx->prog = std::move(tp);
     }
   }
   // bytes: slots and, for the interpreter, one 512-byte descriptor staging
