@@ -81,6 +81,9 @@ def main():
     ap.add_argument("config", type=int, choices=sorted(CONFIGS))
     ap.add_argument("--threads", type=int, default=6)
     ap.add_argument("--block", type=int, default=48)
+    ap.add_argument("--reverse", action="store_true", help="work from the end of the sample (a second host)")
+    ap.add_argument("--out", default=None, help="append to this file instead (merged into tests/golden later)")
+    ap.add_argument("--limit", type=int, default=0, help="stop after this many stimuli")
     a = ap.parse_args()
     cid = a.config
     N, T, n, b, want_regs = CONFIGS[cid]
@@ -91,7 +94,11 @@ def main():
     idx = sample(cid)
     done = read(cid)
     todo = [int(i) for i in idx if int(i) not in done]
-    p = path(cid)
+    if a.reverse:
+        todo = todo[::-1]
+    if a.limit:
+        todo = todo[:a.limit]
+    p = a.out or path(cid)
     if not os.path.exists(p):
         with open(p, "w") as f:
             f.write("\n".join(header(cid)) + "\n")
