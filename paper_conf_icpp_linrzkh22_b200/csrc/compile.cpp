@@ -74,11 +74,12 @@ struct Value {
 struct SlotAlloc {
   std::map<uint32_t, uint32_t> free_;   // offset -> size
   uint32_t top = 0, peak = 0;
-  explicit SlotAlloc(uint32_t base) : top(base), peak(base) {}
+  bool align4 = true;
+  explicit SlotAlloc(uint32_t base, bool a4 = true) : top(base), peak(base), align4(a4) {}
   // slots of 4+ words start on a 16-byte boundary (16-byte cp.async row
-  // copies, program.h uop loads / stores)
+  // copies, program.h uop loads / stores); TMEM columns need no alignment
   uint32_t alloc(uint32_t n) {
-    const uint32_t al = n >= 4 ? 4u : 1u;
+    const uint32_t al = (n >= 4 && align4) ? 4u : 1u;
     for (auto it = free_.begin(); it != free_.end(); ++it) {
       const uint32_t off = it->first, sz = it->second;
       const uint32_t a = (off + al - 1) & ~(al - 1);
@@ -495,7 +496,8 @@ int compile_program(const rtlsim_ir *ir, uint32_t op_lanes, uint32_t smem_limit_
   for (int c = 0; c < 4; c++) xnet_rows[c] = G.xrows[c];
   // spill target: the limit minus the descriptor staging buffers (128 words
   // per op-lane warp; the lane count is not known yet, assume the maximum)
-  const uint32_t stage_words = (op_lanes ? std::min<uint32_t>(op_lanes, 16) : 16) * 128u;
+  // (TMEM schedules are JIT-only: no interpreter staging buffers)
+  const uint32_t stage_words = tmem_cols ? 0u : (op_lanes ? std::min<uint32_t>(op_lanes, 16) : 16) * 128u;
   const uint32_t step_cap = getenv("RTLSIM_STEP_CAP") ? (uint32_t)atoi(getenv("RTLSIM_STEP_CAP")) : 0;
   const uint32_t slot_budget =
       smem_limit_words > stage_words ? smem_limit_words - stage_words : (smem_limit_words ? 1u : 0xFFFFFFFFu);

@@ -1498,6 +1498,103 @@ void emit_bit_batch(Em &e, const std::vector<BitDesc> &ops, uint32_t lut) {
   for (const BitDesc &q : ops) opaque_write(e, SP_S, q.y & 0xFFFFu);
 }
 
+// (r2) Lane-parallel bit ops with a truth table per lane (RTLSIM_JIT_BITANY=k,
+// default 8; 0 = off): the step's 1-bit ops are dealt to the warps in chunks
+// of up to 32 (chunk c to op-lane c mod L) instead of one by one; lane i of
+// the chunk evaluates op i — operand / result offsets and its own truth table
+// (immediates folded in) from one LDG.128 of a per-partition table — as the
+// OR of the minterms its table selects: one LOP3 per minterm any op of the
+// chunk uses, masked by a BFE of the lane's table bit where the ops differ.
+// A chunk of n ops costs ~12-30 warp instructions instead of ~5 n (every lane
+// computing the same packed word, one op after another); chunks smaller
+// than k keep the per-op code. The JIT is instruction-fetch bound
+// (DESIGN.md §5.2b), so the total code is what counts.
+uint32_t jit_bitany() {
+  const char *e = getenv("RTLSIM_JIT_BITANY");
+  return e ? (uint32_t)atoi(e) : 8u;
+}
+// the bit ops warp w evaluates in step s (indices into G.bitdesc), in chunks
+void warp_bits(const Program &G, uint32_t s, uint32_t w, std::vector<std::vector<uint32_t>> &out) {
+  out.clear();
+  const uint32_t b0 = G.bit_ptr[s], b1 = G.bit_ptr[s + 1], n = b1 - b0, k = jit_bitany();
+  if (k && n >= k && jit_split() == 0 && jit_bitbatch() == 0) {
+    const uint32_t nch = (n + 31u) / 32u, sz = (n + nch - 1u) / nch;
+    for (uint32_t c = w; c < nch; c += G.L) {
+      std::vector<uint32_t> ch;
+      for (uint32_t i = b0 + c * sz; i < std::min(b1, b0 + (c + 1u) * sz); i++) ch.push_back(i);
+      if (!ch.empty()) out.push_back(std::move(ch));
+    }
+    return;
+  }
+  for (uint32_t i = b0 + w; i < b1; i += G.L) out.push_back({i});
+}
+void emit_bit_batch_any(Em &e, const Program &G, const std::vector<uint32_t> &idx) {
+  const uint32_t n = (uint32_t)idx.size();
+  for (uint32_t i : idx) begin_value(e, SP_S, G.bitdesc[i].y & 0xFFFFu, 1, true);
+  const uint32_t base = e.bittab ? (uint32_t)(e.bittab->size() / 4) : 0;
+  uint32_t any = 0, all = 0xFFu, used = 0;
+  for (uint32_t i : idx) {
+    const BitDesc &q = G.bitdesc[i];
+    const uint32_t lut = bit_fold_lut(q), d = q.y & 0xFFFFu;
+    const uint32_t f[3] = {q.y >> 16, q.z & 0xFFFFu, q.z >> 16};
+    any |= lut;
+    all &= lut;
+    uint32_t ent[4];
+    for (uint32_t k = 0; k < 3; k++) {
+      if (lut_uses(lut, k)) {
+        used |= 1u << k;
+        note_read(e, SP_S, f[k]);
+        ent[k] = xoff(e, SP_S, f[k]) * 4;
+      } else {
+        ent[k] = xoff(e, SP_S, d) * 4;   // ignored input: the lane's own result word
+      }
+    }
+    ent[3] = xoff(e, SP_S, d) * 4 | (lut << 24);
+    if (e.bittab && !e.dry) e.bittab->insert(e.bittab->end(), ent, ent + 4);
+  }
+  std::string p = e.P(), t[4], a[4], v[3], L = e.R(), dd = e.R();
+  for (int k = 0; k < 4; k++) { t[k] = e.R(); a[k] = e.R(); }
+  e.l(fmt("setp.lt.u32 %s, %%lane, %u", p.c_str(), n));
+  e.l(fmt("@%s ld.global.nc.v4.u32 {%s, %s, %s, %s}, [%%bitl+%u]", p.c_str(), t[0].c_str(), t[1].c_str(),
+          t[2].c_str(), t[3].c_str(), base * 16));
+  e.l(fmt("shr.u32 %s, %s, 24", L.c_str(), t[3].c_str()));
+  e.l(fmt("and.b32 %s, %s, 16777215", dd.c_str(), t[3].c_str()));
+  e.l(fmt("add.u32 %s, %s, %%smb", a[3].c_str(), dd.c_str()));
+  for (int k = 0; k < 3; k++) {
+    v[k] = e.R();
+    if (!(used & (1u << k))) {
+      e.l(fmt("mov.u32 %s, 0", v[k].c_str()));   // no op of the chunk reads it
+      continue;
+    }
+    e.l(fmt("add.u32 %s, %s, %%smb", a[k].c_str(), t[k].c_str()));
+    e.l(fmt("@%s ld.shared.u32 %s, [%s]", p.c_str(), v[k].c_str(), a[k].c_str()));
+  }
+  std::string r;
+  for (uint32_t j = 0; j < 8; j++) {
+    if (!((any >> j) & 1u)) continue;
+    if (j & ~used) continue;   // an input no op reads is 0 here: minterms needing it are 0
+    const uint32_t mt = ((j & 1u) ? 0xF0u : 0x0Fu) & ((j & 2u) ? 0xCCu : 0x33u) & ((j & 4u) ? 0xAAu : 0x55u);
+    std::string m = e.R(), nr = e.R();
+    e.l(fmt("lop3.b32 %s, %s, %s, %s, 0x%02x", m.c_str(), v[0].c_str(), v[1].c_str(), v[2].c_str(), mt));
+    if ((all >> j) & 1u) {
+      if (r.empty()) r = m;
+      else { e.l(fmt("or.b32 %s, %s, %s", nr.c_str(), r.c_str(), m.c_str())); r = nr; }
+    } else {
+      std::string M = e.R();
+      e.l(fmt("bfe.s32 %s, %s, %u, 1", M.c_str(), L.c_str(), j));
+      if (r.empty()) e.l(fmt("and.b32 %s, %s, %s", nr.c_str(), m.c_str(), M.c_str()));
+      else e.l(fmt("lop3.b32 %s, %s, %s, %s, 0xf8", nr.c_str(), r.c_str(), m.c_str(), M.c_str()));   // r | (m & M)
+      r = nr;
+    }
+  }
+  if (r.empty()) {
+    r = e.R();
+    e.l(fmt("mov.u32 %s, 0", r.c_str()));
+  }
+  e.l(fmt("@%s st.shared.u32 [%s], %s", p.c_str(), a[3].c_str(), r.c_str()));
+  for (uint32_t i : idx) opaque_write(e, SP_S, G.bitdesc[i].y & 0xFFFFu);
+}
+
 // RTLSIM_JIT_STATS: PTX instruction lines per descriptor kind (stderr at exit)
 struct EmitStats {
   std::mutex mu;
@@ -1734,7 +1831,12 @@ std::string step_function(const Program &G, const std::string &name, uint32_t s0
       for (uint32_t s = s0; s < s1; s++) {
         d.warp = w;
         d.step = (int32_t)s;
-        for (uint32_t k = G.bit_ptr[s] + w; k < G.bit_ptr[s + 1]; k += G.L) emit_bit(d, G.bitdesc[k]);
+        std::vector<std::vector<uint32_t>> wb;
+        warp_bits(G, s, w, wb);
+        for (auto &ch : wb) {
+          if (ch.size() >= std::max<uint32_t>(jit_bitany(), 2u)) emit_bit_batch_any(d, G, ch);
+          else for (uint32_t k : ch) emit_bit(d, G.bitdesc[k]);
+        }
         for (uint32_t k = G.step_ptr[s * G.L + w]; k < G.step_ptr[s * G.L + w + 1]; k++) emit_desc(d, G, G.desc[k]);
       }
   }
@@ -1909,6 +2011,21 @@ std::string step_function(const Program &G, const std::string &name, uint32_t s0
         for (uint32_t k = G.bit_ptr[s] + w; k < G.bit_ptr[s + 1]; k += G.L) {
           if (bb) groups[bit_fold_lut(G.bitdesc[k])].push_back(G.bitdesc[k]);
           else single.push_back(G.bitdesc[k]);
+        }
+        if (!bb && jit_bitany()) {   // per-lane truth tables (jit_bitany)
+          std::vector<std::vector<uint32_t>> wb;
+          warp_bits(G, s, w, wb);
+          single.clear();
+          for (auto &ch : wb) {
+            if (ch.size() >= std::max<uint32_t>(jit_bitany(), 2u)) {
+              const size_t from = e.s.size();
+              e.opn += ch.size();
+              emit_bit_batch_any(e, G, ch);
+              note_kind(e, "bitany", from);
+            } else {
+              for (uint32_t k : ch) single.push_back(G.bitdesc[k]);
+            }
+          }
         }
         for (auto &g : groups) {
           if (g.second.size() < bb) {
