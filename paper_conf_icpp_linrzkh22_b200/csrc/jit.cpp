@@ -170,6 +170,7 @@ struct Em {
   // IADD3.X per access). Windows live within one basic block (cleared at
   // every label) so each use is dominated by its definition.
   uint32_t nspec = 0;
+  bool used_v = false;         // (r2) 16-byte wide-register loads used (prologue sets %vsm / %vdl)
   std::map<std::string, std::pair<std::string, int64_t>> win;   // base -> (reg, row)
   std::string R() { return fmt("%%r%u", nr++); }
   std::string RD() { return fmt("%%rd%u", nrd++); }
@@ -1219,14 +1220,47 @@ void emit_wide(Em &e, const WideRec &w, uint32_t idx) {
 // ----------------------------------------------------------- loads / stores --
 const char *kArenaTag[4] = {"c", "n", "x", "i"};   // cur, nxt, xnet, in
 
+// (r2) source address of a cp.async: LDGSTS has only a ~2 KB immediate on
+// the global side, so an [window + immediate] address costs IADD3 + IMAD.X
+// per row anyway; one IMAD.WIDE (row x stride + base) is shorter and keeps
+// no window register live
+std::string ldaddr(Em &e, const char *sreg, uint32_t row, const char *base) {
+  if (!e.nspec || getenv("RTLSIM_JIT_LDWIN")) return gaddr(e, sreg, row, base);
+  std::string a = e.RD();
+  e.l(fmt("mad.wide.u32 %s, %%%s, %u, %%%s", a.c_str(), sreg, row, base));
+  return a;
+}
+bool jit_ld16() {
+  const char *e = getenv("RTLSIM_JIT_LD16");
+  return e ? atoi(e) != 0 : true;
+}
+
 void emit_ld(Em &e, uint32_t arena, uint32_t cls, uint32_t row, uint32_t slot, uint32_t nw) {
   const char *A = kArenaTag[arena];
   std::string addr;
+  if (cls == CLS_U32 && nw >= 2 && jit_ld16() && !jit_vwide() && !e.compact) {
+    // (r2) a wide register's nw consecutive rows, four per 16-byte cp.async:
+    // lane l copies bytes 16 (l & 7) .. +15 of row r0 + (l >> 3) of the tile
+    // into word row (l >> 3) of the slot (%vsm, %vdl: the per-lane offsets)
+    e.used_v = true;
+    begin_value(e, SP_W, slot, nw, true);
+    std::string tb = e.RD();
+    e.l(fmt("add.s64 %s, %%tb_%s3, %%vdl", tb.c_str(), A));
+    for (uint32_t g = 0; g < nw; g += 4) {
+      std::string a = e.RD();
+      e.l(fmt("mad.wide.u32 %s, %%N4, %u, %s", a.c_str(), row + g, tb.c_str()));
+      const uint32_t k = std::min<uint32_t>(4u, nw - g);
+      const char *pr = k == 1 ? "@%pl8 " : k == 2 ? "@%pl16 " : k == 3 ? "@%pl24 " : "";
+      e.l(fmt("%scp.async.cg.shared.global [%%vsm+%u], [%s], 16", pr, (slot + 32u * g) * 4u, a.c_str()));
+    }
+    for (uint32_t i = 0; i < nw; i++) opaque_write(e, SP_W, slot + 32 * i);
+    return;
+  }
   switch (cls) {
     case CLS_U32:
       begin_value(e, SP_W, slot, nw, true);
       for (uint32_t i = 0; i < nw; i++) {
-        std::string ai = gaddr(e, "N4", row + i, fmt("tb_%s3", A).c_str());
+        std::string ai = ldaddr(e, "N4", row + i, fmt("tb_%s3", A).c_str());
         if (nw >= 2 && jit_vwide())   // into the word's place in its group
           e.l(fmt("cp.async.ca.shared.global [%s+%u], [%s], 4", kLaneBase[vgs(nw, i / 4u)], vbyte(e, slot, nw, i),
                   ai.c_str()));
@@ -1237,19 +1271,19 @@ void emit_ld(Em &e, uint32_t arena, uint32_t cls, uint32_t row, uint32_t slot, u
       break;
     case CLS_U16:
       begin_value(e, SP_H, slot, 1, true);
-      addr = gaddr(e, "N2", row, fmt("tb_%s2", A).c_str());
+      addr = ldaddr(e, "N2", row, fmt("tb_%s2", A).c_str());
       e.l(fmt("@%%pl16 cp.async.ca.shared.global [%%rw+%u], [%s], 4", xoff(e, SP_H, slot) * 4, addr.c_str()));
       opaque_write(e, SP_H, slot);
       break;
     case CLS_U8:
       begin_value(e, SP_B, slot, 1, true);
-      addr = gaddr(e, "N", row, fmt("tb_%s1", A).c_str());
+      addr = ldaddr(e, "N", row, fmt("tb_%s1", A).c_str());
       e.l(fmt("@%%pl8 cp.async.ca.shared.global [%%rw+%u], [%s], 4", xoff(e, SP_B, slot) * 4, addr.c_str()));
       opaque_write(e, SP_B, slot);
       break;
     default:
       begin_value(e, SP_S, slot, 1, true);
-      addr = gaddr(e, "Nb", row, fmt("tb_%s0", A).c_str());
+      addr = ldaddr(e, "Nb", row, fmt("tb_%s0", A).c_str());
       e.l(fmt("@%%pl0 cp.async.ca.shared.global [%%smb+%u], [%s], 4", xoff(e, SP_S, slot) * 4, addr.c_str()));
       opaque_write(e, SP_S, slot);
       break;
@@ -1499,7 +1533,8 @@ void emit_bit_batch(Em &e, const std::vector<BitDesc> &ops, uint32_t lut) {
 }
 
 // (r2) Lane-parallel bit ops with a truth table per lane (RTLSIM_JIT_BITANY=k,
-// default 8; 0 = off): the step's 1-bit ops are dealt to the warps in chunks
+// default 0 = off: config 4 TMEM 59.1 ms/cycle with k = 8 vs 55.4 without —
+// 3 % less code, but the table load sits on every step's critical path): the step's 1-bit ops are dealt to the warps in chunks
 // of up to 32 (chunk c to op-lane c mod L) instead of one by one; lane i of
 // the chunk evaluates op i — operand / result offsets and its own truth table
 // (immediates folded in) from one LDG.128 of a per-partition table — as the
@@ -1511,7 +1546,7 @@ void emit_bit_batch(Em &e, const std::vector<BitDesc> &ops, uint32_t lut) {
 // (DESIGN.md §5.2b), so the total code is what counts.
 uint32_t jit_bitany() {
   const char *e = getenv("RTLSIM_JIT_BITANY");
-  return e ? (uint32_t)atoi(e) : 8u;
+  return e ? (uint32_t)atoi(e) : 0u;
 }
 // the bit ops warp w evaluates in step s (indices into G.bitdesc), in chunks
 void warp_bits(const Program &G, uint32_t s, uint32_t w, std::vector<std::vector<uint32_t>> &out) {
@@ -2144,7 +2179,7 @@ std::string step_function(const Program &G, const std::string &name, uint32_t s0
   out += "\t.reg .b32 %rq2, %rq3, %rq4;\n";
   out += "\t.reg .b32 %smb, %lane, %wl, %N, %tbar, %mbar, %tmt, %rw, %rh, %rb, %N4, %N2, %Nb, %lsh;\n\t.reg .b64 %tbb1, %tbb2, %tlw, ";
   for (int i = 0; i < kN64; i++) out += fmt("%s%%%s", i ? ", " : "", kCtx64[i]);
-  out += ";\n\t.reg .pred %pl0, %pl8, %pl16, %pdig;\n";
+  out += ";\n\t.reg .pred %pl0, %pl8, %pl16, %pl24, %pdig;\n\t.reg .b32 %vsm;\n\t.reg .b64 %vdl;\n";
   for (int i = 0; i < kN32; i++) out += fmt("\tld.param.u32 %%%s, [a_%s];\n", kCtx32[i], kCtx32[i]);
   for (int i = 0; i < kN64; i++) out += fmt("\tld.param.u64 %%%s, [a_%s];\n", kCtx64[i], kCtx64[i]);
   out += "\tmad.lo.u32 %rq2, %lane, 8, %smb;\n\tmad.lo.u32 %rq3, %lane, 12, %smb;\n\tmad.lo.u32 %rq4, %lane, 16, %smb;\n";
@@ -2154,6 +2189,12 @@ std::string step_function(const Program &G, const std::string &name, uint32_t s0
          "\tsetp.ne.u64 %pdig, %dig, 0;\n\tsub.u32 %lsh, 31, %lane;\n"
          "\tmul.wide.u32 %tlw, %lane, 3;\n\tsub.s64 %tbb1, %tb_n1, %tlw;\n"
          "\tmul.wide.u32 %tlw, %lane, 2;\n\tsub.s64 %tbb2, %tb_n2, %tlw;\n";
+  if (e.used_v)   // 16-byte wide loads: smem / global offsets of lane l (row l >> 3, bytes 16 (l & 7))
+    out += "\tsetp.lt.u32 %pl24, %lane, 24;\n\t{\n\t.reg .b32 %vq, %vr;\n\t.reg .b64 %vw;\n"
+           "\tshr.u32 %vq, %lane, 3;\n\tand.b32 %vr, %lane, 7;\n"
+           "\tmad.lo.u32 %vsm, %vq, 128, %smb;\n\tmad.lo.u32 %vsm, %vr, 16, %vsm;\n"
+           "\tmul.wide.u32 %vdl, %vq, %N4;\n\tmul.wide.u32 %vw, %vr, 16;\n\tadd.s64 %vdl, %vdl, %vw;\n"
+           "\tmul.wide.u32 %vw, %lane, 4;\n\tsub.s64 %vdl, %vdl, %vw;\n\t}\n";
   out += e.s;
   out += "\tret;\n}\n";
   return out;
