@@ -1224,15 +1224,19 @@ const char *kArenaTag[4] = {"c", "n", "x", "i"};   // cur, nxt, xnet, in
 // the global side, so an [window + immediate] address costs IADD3 + IMAD.X
 // per row anyway; one IMAD.WIDE (row x stride + base) is shorter and keeps
 // no window register live
+// (measured config 4 TMEM: 55.3 ms/cycle with windows vs 55.9 with IMAD.WIDE:
+// windows stay the default, RTLSIM_JIT_LDMAD=1 for A/B)
 std::string ldaddr(Em &e, const char *sreg, uint32_t row, const char *base) {
-  if (!e.nspec || getenv("RTLSIM_JIT_LDWIN")) return gaddr(e, sreg, row, base);
+  if (!e.nspec || !getenv("RTLSIM_JIT_LDMAD")) return gaddr(e, sreg, row, base);
   std::string a = e.RD();
   e.l(fmt("mad.wide.u32 %s, %%%s, %u, %%%s", a.c_str(), sreg, row, base));
   return a;
 }
+// (r2, RTLSIM_JIT_LD16=1, default off: config 4 TMEM 55.8 vs 55.3 ms/cycle —
+// 40 % fewer LDGSTS but two more live registers and more spills)
 bool jit_ld16() {
   const char *e = getenv("RTLSIM_JIT_LD16");
-  return e ? atoi(e) != 0 : true;
+  return e ? atoi(e) != 0 : false;
 }
 
 void emit_ld(Em &e, uint32_t arena, uint32_t cls, uint32_t row, uint32_t slot, uint32_t nw) {
@@ -1849,7 +1853,8 @@ uint64_t jit_fwd_ops(bool compact) {
 
 std::string step_function(const Program &G, const std::string &name, uint32_t s0, uint32_t s1, bool dig,
                           uint32_t nspec, bool to_end, uint32_t *tile_words = nullptr,
-                          std::vector<WideRec> *wrec_out = nullptr, std::vector<uint32_t> *bittab_out = nullptr) {
+                          std::vector<WideRec> *wrec_out = nullptr, std::vector<uint32_t> *bittab_out = nullptr,
+                          bool inline_body = false) {
   t_prog = &G;
   const bool compact = jit_compact_env(G) && to_end && tile_words;
   std::vector<Em::Inst> insts;
@@ -2173,15 +2178,23 @@ std::string step_function(const Program &G, const std::string &name, uint32_t s0
   } else {
     emit_real(e, false, false);
   }
-  std::string out = func_proto(name) + "\n{\n";
+  // (r2) inline_body: the same code as a block of the kernel (no call: no
+  // parameter passing, no caller stack frame, one register allocation)
+  std::string out = inline_body ? std::string("\t{\n") : func_proto(name) + "\n{\n";
   out += fmt("\t.reg .b32 %%r<%u>;\n\t.reg .b64 %%rd<%u>;\n\t.reg .pred %%p<%u>;\n", e.nr + 1, e.nrd + 1, e.np + 1);
   out += "\t.reg .b64 %mtok0, %mtok1;\n";
   out += "\t.reg .b32 %rq2, %rq3, %rq4;\n";
-  out += "\t.reg .b32 %smb, %lane, %wl, %N, %tbar, %mbar, %tmt, %rw, %rh, %rb, %N4, %N2, %Nb, %lsh;\n\t.reg .b64 %tbb1, %tbb2, %tlw, ";
-  for (int i = 0; i < kN64; i++) out += fmt("%s%%%s", i ? ", " : "", kCtx64[i]);
+  if (inline_body) {
+    out += "\t.reg .b32 %rw, %rh, %rb, %N4, %N2, %Nb, %lsh;\n\t.reg .b64 %tbb1, %tbb2, %tlw";
+  } else {
+    out += "\t.reg .b32 %smb, %lane, %wl, %N, %tbar, %mbar, %tmt, %rw, %rh, %rb, %N4, %N2, %Nb, %lsh;\n\t.reg .b64 %tbb1, %tbb2, %tlw, ";
+    for (int i = 0; i < kN64; i++) out += fmt("%s%%%s", i ? ", " : "", kCtx64[i]);
+  }
   out += ";\n\t.reg .pred %pl0, %pl8, %pl16, %pl24, %pdig;\n\t.reg .b32 %vsm;\n\t.reg .b64 %vdl;\n";
-  for (int i = 0; i < kN32; i++) out += fmt("\tld.param.u32 %%%s, [a_%s];\n", kCtx32[i], kCtx32[i]);
-  for (int i = 0; i < kN64; i++) out += fmt("\tld.param.u64 %%%s, [a_%s];\n", kCtx64[i], kCtx64[i]);
+  if (!inline_body) {
+    for (int i = 0; i < kN32; i++) out += fmt("\tld.param.u32 %%%s, [a_%s];\n", kCtx32[i], kCtx32[i]);
+    for (int i = 0; i < kN64; i++) out += fmt("\tld.param.u64 %%%s, [a_%s];\n", kCtx64[i], kCtx64[i]);
+  }
   out += "\tmad.lo.u32 %rq2, %lane, 8, %smb;\n\tmad.lo.u32 %rq3, %lane, 12, %smb;\n\tmad.lo.u32 %rq4, %lane, 16, %smb;\n";
   out += "\tmad.lo.u32 %rw, %lane, 4, %smb;\n\tmad.lo.u32 %rh, %lane, 2, %smb;\n\tadd.u32 %rb, %lane, %smb;\n"
          "\tshl.b32 %N4, %N, 2;\n\tshl.b32 %N2, %N, 1;\n\tshr.u32 %Nb, %N, 3;\n"
@@ -2196,8 +2209,12 @@ std::string step_function(const Program &G, const std::string &name, uint32_t s0
            "\tmul.wide.u32 %vdl, %vq, %N4;\n\tmul.wide.u32 %vw, %vr, 16;\n\tadd.s64 %vdl, %vdl, %vw;\n"
            "\tmul.wide.u32 %vw, %lane, 4;\n\tsub.s64 %vdl, %vdl, %vw;\n\t}\n";
   out += e.s;
-  out += "\tret;\n}\n";
+  out += inline_body ? "\t}\n" : "\tret;\n}\n";
   return out;
+}
+bool jit_inline() {
+  const char *e = getenv("RTLSIM_JIT_INLINE");
+  return e ? atoi(e) != 0 : false;
 }
 
 }  // namespace
@@ -2241,10 +2258,15 @@ std::string jit_partition_ptx(const Program &G, uint32_t q, const std::string &r
   uint32_t tile_words = 0;
   JitPartInfo local;
   if (!info) info = &local;
-  for (size_t g = 0; g < groups.size(); g++)
-    mod += step_function(G, fmt("rtl_steps_%zu", g), groups[g].first, groups[g].second, dig, nspec,
-                         groups[g].second == s1, compact ? &tile_words : nullptr,
-                         compact ? &info->wide : nullptr, &info->bittab) + "\n";
+  const bool inl = jit_inline();
+  std::vector<std::string> bodies;
+  for (size_t g = 0; g < groups.size(); g++) {
+    std::string f = step_function(G, fmt("rtl_steps_%zu", g), groups[g].first, groups[g].second, dig, nspec,
+                                  groups[g].second == s1, compact ? &tile_words : nullptr,
+                                  compact ? &info->wide : nullptr, &info->bittab, inl);
+    if (inl) bodies.push_back(std::move(f));
+    else mod += f + "\n";
+  }
   // shared memory per tile: the compacted extent, or the schedule's slots
   const uint32_t tbytes = compact ? std::max<uint32_t>(16u, ((tile_words * 4u) + 15u) & ~15u) : jit_tile_bytes(G);
   info->tile_bytes = tbytes;
@@ -2324,6 +2346,10 @@ std::string jit_partition_ptx(const Program &G, uint32_t q, const std::string &r
   mod += "\t{\n\t.reg .b32 %cyc, %ncy;\n\t.reg .b64 %tsw, %stp;\n\t.reg .pred %pcy;\n";
   mod += fmt("\tld.param.u32 %%ncy, [prm+%zu];\n\tmov.u32 %%cyc, 0;\n$CYC:\n", offsetof(JitParams, nc));
   for (size_t g = 0; g < groups.size(); g++) {
+    if (inl) {
+      mod += bodies[g];
+      continue;
+    }
     mod += "\t{\n";
     std::string args;
     int pi = 0;
