@@ -261,3 +261,25 @@ def test_memory_validation_host_only(R):
     with pytest.raises(R.RtlsimError) as ei:
         R.Simulator(b.build(), flags=R.F_HOST_ONLY | R.F_JIT)
     assert ei.value.code == -4
+
+
+def test_tmem_schedule_host_only(R, tmp_path, monkeypatch):
+    """TMEM schedules compile host-only: computed U32 values
+    get TMEM columns (slot = 0x8000 + 32 col), the shared-memory slot area
+    shrinks, and the generated PTX allocates / frees TMEM and moves values
+    with tcgen05.ld / tcgen05.st under the step-barrier fences."""
+    ir = designs.random_dag(502, n_ops=300, n_regs=24, n_partitions=3, input_widths=(7, 33, 1, 64, 100),
+                            max_width=1024)
+    monkeypatch.setenv("RTLSIM_JIT_CACHE", "")
+    monkeypatch.setenv("RTLSIM_JIT_SAVE", str(tmp_path))
+    monkeypatch.setenv("RTLSIM_JIT_TMEM", "0")
+    classic = R.Simulator(ir, flags=R.F_HOST_ONLY | R.F_JIT).stats()
+    monkeypatch.setenv("RTLSIM_JIT_TMEM", "1")
+    st = R.Simulator(ir, flags=R.F_HOST_ONLY | R.F_JIT).stats()
+    assert classic["tmem_cols"] == 0 and 0 < st["tmem_cols"] <= 512
+    assert st["smem_words"] < classic["smem_words"]
+    assert st["op_lanes"] <= 8 and st["jit_sass_instructions"] > 0
+    ptx = "".join(p.read_text() for p in tmp_path.glob("part*.ptx"))
+    for needle in ("tcgen05.alloc", "tcgen05.dealloc", "tcgen05.ld.sync.aligned.32x32b", "tcgen05.st.sync.aligned.32x32b",
+                   "tcgen05.wait::st", "tcgen05.fence::before_thread_sync", "tcgen05.fence::after_thread_sync"):
+        assert needle in ptx, needle
