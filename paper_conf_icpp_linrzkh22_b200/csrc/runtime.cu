@@ -291,7 +291,11 @@ extern "C" int rtlsim_load(const rtlsim_ir *ir, const rtlsim_options *opt, rtlsi
       rtlsim::Program tp;
       std::string e2;
       const uint32_t tl = std::min<uint32_t>(ctx->opt.op_lanes ? ctx->opt.op_lanes : 8u, 8u);
-      if (compile_program(ir, tl, (smem_limit - 256u) / 16u, &tp, &e2, dce, fold, 512u) == RTLSIM_OK &&
+      // RTLSIM_JIT_TMEM_SMEM_KB: CTA shared-memory budget (the rest of the
+      // 256 KB is L1, where register spills land)
+      uint32_t cta = smem_limit;
+      if (const char *e = getenv("RTLSIM_JIT_TMEM_SMEM_KB")) cta = std::min<uint32_t>(cta, 1024u * (uint32_t)atoi(e));
+      if (compile_program(ir, tl, (cta - 256u) / 16u, &tp, &e2, dce, fold, 512u) == RTLSIM_OK &&
           tp.tmem_cols > 0 && jit_tile_bytes(tp) * 4u + 256u <= smem_limit)
         ctx->prog = std::move(tp);
     }
