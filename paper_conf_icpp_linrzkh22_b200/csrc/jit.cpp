@@ -53,6 +53,7 @@ const char *kCtx64[] = {"tb_c0", "tb_c1", "tb_c2", "tb_c3", "tb_n0", "tb_n1", "t
                         "tb_x0", "tb_x1", "tb_x2", "tb_x3", "tb_i0", "tb_i1", "tb_i2", "tb_i3",
                         "outb", "dig", "wide", "smg", "bitl", "memb", "portb"};
 constexpr int kN32 = 7, kN64 = 23;
+constexpr uint64_t kTmemFwdOps = 8;   // forwarding budget of TMEM schedules (jit_fwd_ops)
 
 // Split-phase step barrier (RTLSIM_JIT_SPLIT=1; default off, see below):
 // instead of bar.sync at every step end, a warp arrives on an mbarrier (two,
@@ -1845,10 +1846,15 @@ bool jit_compact_env(const Program &G) {
   const char *e = getenv("RTLSIM_JIT_COMPACT");
   return G.L == 1 && (e ? atoi(e) != 0 : true);
 }
-uint64_t jit_fwd_ops(bool compact) {
+// forwarding register budget: a slot value is taken from a register only
+// within this many descriptors of its write / read. TMEM schedules run 32
+// warps at 64 registers and spill; budgets of 4 / 8 / 16
+// measured config 4 at 52.8 / 53.0 / 52.9 ms/cycle vs 55.9 unbounded
+// (profiles/r02_t_probe_fwd.log, r02_u_probe.log)
+uint64_t jit_fwd_ops(bool compact, bool tmem = false) {
   const char *e = getenv("RTLSIM_JIT_FWDOPS");
   if (e) return (uint64_t)atoll(e);
-  return compact ? 64u : UINT64_MAX;
+  return compact ? 64u : tmem ? kTmemFwdOps : UINT64_MAX;
 }
 
 std::string step_function(const Program &G, const std::string &name, uint32_t s0, uint32_t s1, bool dig,
@@ -1983,7 +1989,7 @@ std::string step_function(const Program &G, const std::string &name, uint32_t s0
   e.nspec = nspec;
   e.log = &log;
   e.fwd_max = compact ? INT32_MAX / 2 : jit_fwd_steps();
-  e.fwd_ops = jit_fwd_ops(compact);
+  e.fwd_ops = jit_fwd_ops(compact, G.tmem_cols != 0);
   e.compact = compact;
   e.inst = &insts;
   e.wrec = probe ? &wrec_probe : &wrec_final;
