@@ -41,4 +41,5 @@ for cid in cfgs:
     print(json.dumps({"cfg": cid, "env": {k: os.environ.get(k) for k in ("JIT","LANES","SMEM_KB","RTLSIM_JIT_OPT","RTLSIM_JIT_TMAX","RTLSIM_JIT_TPC","N")}, "tpc_max_smem": 232448 // max(1, st["smem_words"]*4), "jit_s": s1["jit_compile_s"], "cubin": s1["jit_cubin_bytes"], "tpc_used": None, "gen_s": round(tg,1), "load_s": round(tl,2), "L": st['op_lanes'], "smem_KB": st['smem_words']*4/1024,
           "steps": st['n_steps'], "desc": st['n_desc'], "b_floor": st['b_floor'], "b_state": st['b_state'],
           "ms_per_cycle_total": ms / (3*Tc), "ms_per_cycle_eval": ems / (3*Tc),
-          "stim_cyc_per_s": stc / (ms/1e3), "eval_GBps_floor": st['b_floor'] * stc / (ems/1e3) / 1e9}))
+          "stim_cyc_per_s": stc / (ms/1e3), "sass": s1["jit_sass_instructions"], "tmem_cols": s1["tmem_cols"],
+          "warp_instr_per_s": s1["jit_sass_instructions"] * (N / 32) / (ems / (3*Tc) / 1e3) if s1["jit_sass_instructions"] else None, "eval_GBps_floor": st['b_floor'] * stc / (ems/1e3) / 1e9}))
