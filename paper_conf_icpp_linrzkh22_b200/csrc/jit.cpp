@@ -172,6 +172,7 @@ struct Em {
   // every label) so each use is dominated by its definition.
   uint32_t nspec = 0;
   bool used_v = false;         // (r2) 16-byte wide-register loads used (prologue sets %vsm / %vdl)
+  bool ubase = false;          // (r2) arena windows from the kernel's params + %to<k> (inline bodies)
   std::map<std::string, std::pair<std::string, int64_t>> win;   // base -> (reg, row)
   std::string R() { return fmt("%%r%u", nr++); }
   std::string RD() { return fmt("%%rd%u", nrd++); }
@@ -213,7 +214,17 @@ std::string gaddr(Em &e, const char *sreg, uint32_t row, const char *base) {
   // new window: this row plus the rows up to ~12 MB above and ~4 MB below it
   const int64_t wrow = (int64_t)row + std::max<int64_t>(0, ((int64_t)1 << 22) / stride);
   std::string a = e.RD();
-  e.l(fmt("add.s64 %s, %%%s, %lld", a.c_str(), base, (long long)(wrow * stride)));
+  if (e.ubase && !strncmp(base, "tb_", 3) && strlen(base) == 5 && strchr("cnxi", base[3])) {
+    // (r2) uniform arena base from the kernel parameters (constant bank) plus
+    // the thread's 64-bit class offset: no per-arena base register stays live
+    const uint32_t ai = (uint32_t)(strchr("cnxi", base[3]) - "cnxi"), k = (uint32_t)(base[4] - '0');
+    std::string u = e.RD(), t = e.RD();
+    e.l(fmt("ld.param.u64 %s, [prm+%u]", u.c_str(), 32u * ai + 8u * k));
+    e.l(fmt("add.s64 %s, %s, %%to%u", t.c_str(), u.c_str(), k));
+    e.l(fmt("add.s64 %s, %s, %lld", a.c_str(), t.c_str(), (long long)(wrow * stride)));
+  } else {
+    e.l(fmt("add.s64 %s, %%%s, %lld", a.c_str(), base, (long long)(wrow * stride)));
+  }
   e.win[base] = {a, wrow};
   return off_str(a, ((int64_t)row - wrow) * stride);
 }
@@ -1857,6 +1868,16 @@ uint64_t jit_fwd_ops(bool compact, bool tmem = false) {
   return compact ? 64u : tmem ? kTmemFwdOps : UINT64_MAX;
 }
 
+// (r2) RTLSIM_JIT_UBASE=1: inline step bodies address the state arenas from
+// the kernel parameters (uniform, constant bank) plus one 64-bit per-class
+// thread offset %to<k>, instead of 16 per-arena 64-bit base registers — the
+// registers the 64-per-thread budget of 32-warp TMEM CTAs spills
+static_assert(offsetof(JitParams, cur) == 0 && offsetof(JitParams, nxt) == 32 && offsetof(JitParams, xnet) == 64 &&
+                  offsetof(JitParams, in) == 96, "jit_ubase reads the arena bases at prm + 32 * arena + 8 * class");
+bool jit_ubase() {
+  const char *e = getenv("RTLSIM_JIT_UBASE");
+  return e && atoi(e) != 0;
+}
 std::string step_function(const Program &G, const std::string &name, uint32_t s0, uint32_t s1, bool dig,
                           uint32_t nspec, bool to_end, uint32_t *tile_words = nullptr,
                           std::vector<WideRec> *wrec_out = nullptr, std::vector<uint32_t> *bittab_out = nullptr,
@@ -1990,6 +2011,7 @@ std::string step_function(const Program &G, const std::string &name, uint32_t s0
   e.log = &log;
   e.fwd_max = compact ? INT32_MAX / 2 : jit_fwd_steps();
   e.fwd_ops = jit_fwd_ops(compact, G.tmem_cols != 0);
+  e.ubase = inline_body && jit_ubase() && nspec != 0 && G.part_steps.size() > 2;
   e.compact = compact;
   e.inst = &insts;
   e.wrec = probe ? &wrec_probe : &wrec_final;
@@ -2220,7 +2242,7 @@ std::string step_function(const Program &G, const std::string &name, uint32_t s0
 }
 bool jit_inline() {
   const char *e = getenv("RTLSIM_JIT_INLINE");
-  return e ? atoi(e) != 0 : false;
+  return e ? atoi(e) != 0 : jit_ubase();
 }
 
 }  // namespace
@@ -2300,6 +2322,16 @@ std::string jit_partition_ptx(const Program &G, uint32_t q, const std::string &r
   mod += fmt("\tld.param.u32 %%N, [prm+%zu];\n", offsetof(JitParams, N));
   if (nspec)   // row offsets are immediates for this N_pad: refuse any other
     mod += fmt("\t{\n\t.reg .pred %%pn;\n\tsetp.ne.u32 %%pn, %%N, %u;\n\t@%%pn trap;\n\t}\n", nspec);
+  // per-class 64-bit thread offsets into an arena (tile * row bytes + lane
+  // * 4; bit rows: tile * 4) for the parameter-based addressing (jit_ubase)
+  mod += "\t.reg .b64 %to0, %to1, %to2, %to3;\n";
+  {
+    const uint32_t tm[4] = {4, 32, 64, 128};
+    for (int k = 0; k < 4; k++) {
+      mod += fmt("\tmul.wide.u32 %%to%d, %%tile, %u;\n", k, tm[k]);
+      if (k > 0) mod += fmt("\tmul.wide.u32 %%t64, %%lane, 4;\n\tadd.u64 %%to%d, %%to%d, %%t64;\n", k, k);
+    }
+  }
   const size_t aoff[4] = {offsetof(JitParams, cur), offsetof(JitParams, nxt), offsetof(JitParams, xnet),
                           offsetof(JitParams, in)};
   const char *tag[4] = {"c", "n", "x", "i"};
