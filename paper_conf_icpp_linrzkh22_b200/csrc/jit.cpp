@@ -1679,7 +1679,7 @@ void desc_keys(const Program &G, const Desc &q, std::vector<uint64_t> &src, std:
 // is loaded up front — runs of consecutive columns as vector tcgen05.ld
 // (.x2 .. .x32), one tcgen05.wait::ld for all — and handed to the emitter as
 // forwarded registers (lds() then finds them)
-void tm_prefetch(Em &e, const Program &G, const Desc &q) {
+void tm_cols_of(Em &e, const Program &G, const Desc &q, std::vector<uint32_t> &cols) {
   std::vector<uint64_t> src, dst;
   bool ld = false;
   desc_keys(G, q, src, dst, &ld);
@@ -1690,7 +1690,6 @@ void tm_prefetch(Em &e, const Program &G, const Desc &q) {
     lo = r.imm / 32u;
     hi = (r.imm + r.wd - 1u) / 32u;
   }
-  std::vector<uint32_t> cols;
   for (uint64_t k : src) {
     const uint32_t off = (uint32_t)k;
     if ((k >> 32) != SP_W || !in_tmem(off) || !fwd_get(e, k).empty()) continue;
@@ -1700,6 +1699,20 @@ void tm_prefetch(Em &e, const Program &G, const Desc &q) {
     }
     cols.push_back((off - kTmemBase) / 32u);
   }
+}
+// RTLSIM_JIT_TMGROUP=g: the TMEM operands of g consecutive descriptors of a
+// warp's step are loaded together (one wait); default 1
+uint32_t jit_tmgroup() {
+  const char *e = getenv("RTLSIM_JIT_TMGROUP");
+  return e ? std::max(1, atoi(e)) : 1u;
+}
+void tm_prefetch_cols(Em &e, std::vector<uint32_t> &cols);
+void tm_prefetch(Em &e, const Program &G, const Desc &q) {
+  std::vector<uint32_t> cols;
+  tm_cols_of(e, G, q, cols);
+  tm_prefetch_cols(e, cols);
+}
+void tm_prefetch_cols(Em &e, std::vector<uint32_t> &cols) {
   if (cols.empty()) return;
   std::sort(cols.begin(), cols.end());
   cols.erase(std::unique(cols.begin(), cols.end()), cols.end());
@@ -2115,7 +2128,16 @@ std::string step_function(const Program &G, const std::string &name, uint32_t s0
           note_kind(e, "bit", from);
         }
       }
-      for (uint32_t k = G.step_ptr[s * G.L + w]; k < G.step_ptr[s * G.L + w + 1]; k++) emit_desc(e, G, G.desc[k]);
+      for (uint32_t k0 = G.step_ptr[s * G.L + w], k = k0; k < G.step_ptr[s * G.L + w + 1]; k++) {
+        const uint32_t g = jit_tmgroup();
+        if (G.tmem_cols && g > 1 && e.fwd_max > 0 && (k - k0) % g == 0) {
+          std::vector<uint32_t> cols;
+          for (uint32_t j = k; j < std::min<uint32_t>(k + g, G.step_ptr[s * G.L + w + 1]); j++)
+            tm_cols_of(e, G, G.desc[j], cols);
+          tm_prefetch_cols(e, cols);
+        }
+        emit_desc(e, G, G.desc[k]);
+      }
       e.l("cp.async.commit_group");
       e.l(fmt("cp.async.wait_group %u", G.step_wait[s]));
       // The per-warp code blocks each hold their own copy of the step
